@@ -1,0 +1,190 @@
+"""CPU oracle for the Jigsaw hot path -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` leg may import this package.  The product path
+(``paper_conf_icpp_zhanglyfyllq24_b200``) never imports it, and this package
+never imports the product: the two share no code.  The only module both use is
+``synth`` (seeded input generators, none of the method's arithmetic).
+
+Thin ctypes marshalling around ``oracle/oracle.c`` (O1 SpMM, O2 canonical
+reorder CR1) plus re-exports of the independent numpy checker ``check.py`` (O3).
+Citations are to /root/reference/PAPER.md lines (P:NNN) and to the readings
+R-Qn listed in DESIGN.md §3.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+PAD = -1
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c into liboracle.so with gcc (plain C11, -O2, no SIMD flags)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-shared", "-fPIC",
+                               "-o", _LIB, _SRC])
+    return _LIB
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_LIB)
+        i64, p = ctypes.c_int64, ctypes.c_void_p
+        L.orc_half_to_double.restype = ctypes.c_double
+        L.orc_half_to_double.argtypes = [ctypes.c_uint16]
+        L.orc_spmm.restype = ctypes.c_int
+        L.orc_spmm.argtypes = [p, i64, i64, p, i64, p, i64, p, p]
+        L.orc_tile_reorder.restype = ctypes.c_int
+        L.orc_tile_reorder.argtypes = [p, ctypes.c_int, ctypes.c_int, ctypes.c_int, p, p, p, p]
+        L.orc_reorder_range.restype = p
+        L.orc_reorder_range.argtypes = [p, i64, i64, ctypes.c_int, ctypes.c_int,
+                                        ctypes.c_int, ctypes.c_int]
+        L.orc_format_sizes.restype = None
+        L.orc_format_sizes.argtypes = [p, p]
+        L.orc_format_copy.restype = None
+        L.orc_format_copy.argtypes = [p] * 11
+        L.orc_format_free.restype = None
+        L.orc_format_free.argtypes = [p]
+        _lib = L
+    return _lib
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _bits(x: np.ndarray) -> np.ndarray:
+    x = np.ascontiguousarray(x)
+    if x.dtype == np.float16:
+        x = x.view(np.uint16)
+    if x.dtype != np.uint16:
+        raise TypeError("expected fp16 values or uint16 fp16 bit patterns")
+    return x
+
+
+def half_to_double(h: int) -> float:
+    return lib().orc_half_to_double(int(h) & 0xFFFF)
+
+
+def spmm(A, B, rows=None):
+    """O1: C = A.B over the nonzeros of A, fp64 accumulation, plus
+    Mabs = |A|.|B| for the parity tolerance |C - C_ref| <= 1e-2*Mabs + 1e-3.
+    ``rows`` (optional) restricts the computation to those rows of A."""
+    A, B = _bits(A), _bits(B)
+    M, K = A.shape
+    K2, N = B.shape
+    assert K == K2
+    if rows is None:
+        r, nr, rp = None, M, None
+    else:
+        r = np.ascontiguousarray(np.asarray(rows, dtype=np.int64))
+        nr, rp = len(r), _ptr(r)
+    C = np.empty((nr, N), dtype=np.float64)
+    Mabs = np.empty((nr, N), dtype=np.float64)
+    rc = lib().orc_spmm(_ptr(A), M, K, _ptr(B), N, rp, nr, _ptr(C), _ptr(Mabs))
+    if rc:
+        raise ValueError(f"orc_spmm failed ({rc})")
+    return C, Mabs
+
+
+def tile_reorder(masks, cols, W=16, G=4, Z=2):
+    """Alg. 1 + reorder retry on one tile.
+
+    masks: W python ints (row bitmasks, row r = bit r, P <= 128 rows)
+    cols : W column ids (PAD = -1)
+    Returns (perm, cols_after, evicted)."""
+    m = np.zeros(2 * W, dtype=np.uint64)
+    for j, x in enumerate(masks):
+        m[2 * j] = np.uint64(int(x) & ((1 << 64) - 1))
+        m[2 * j + 1] = np.uint64(int(x) >> 64)
+    c = np.ascontiguousarray(np.asarray(cols, dtype=np.int32))
+    perm = np.zeros(W, dtype=np.uint8)
+    ev = np.zeros(16, dtype=np.int32)
+    nev = ctypes.c_int(0)
+    rc = lib().orc_tile_reorder(_ptr(m), W, G, Z, _ptr(c), _ptr(perm), _ptr(ev),
+                                ctypes.byref(nev))
+    if rc:
+        raise ValueError(f"orc_tile_reorder failed ({rc})")
+    return perm.tolist(), c.tolist(), ev[: nev.value].tolist()
+
+
+@dataclass
+class Format:
+    """Canonical CR1 arrays.  Tiles of all panels are stored
+    consecutively; panel p owns tiles tile_off[p] : tile_off[p] + T[p]."""
+    M: int
+    K: int
+    P: int
+    mode: int
+    panels: range
+    T: np.ndarray          # [npanels] int64
+    D: np.ndarray          # [npanels] int64
+    col_idx: np.ndarray    # [ntiles, 16] int32, PAD = -1
+    perm: np.ndarray       # [ntiles, 16] uint8
+    vals: np.ndarray       # [ntiles, P, 8] uint16 (fp16 bits)
+    meta: np.ndarray       # [ntiles, P] uint16 (nibble q = i0 + 4*i1 at bits 4q)
+    kind: np.ndarray       # [ntiles] uint8 (0 MAIN, 1 OVERFLOW)
+    nevict: np.ndarray     # [ntiles] uint8
+    rcol: np.ndarray       # [ndtiles, 16] int32 (DENSE mode)
+    dvals: np.ndarray      # [ndtiles, P, 16] uint16 (DENSE mode)
+
+    @property
+    def tile_off(self):
+        return np.concatenate([[0], np.cumsum(self.T)]).astype(np.int64)
+
+    @property
+    def dtile_off(self):
+        return np.concatenate([[0], np.cumsum(self.D)]).astype(np.int64)
+
+    @property
+    def gather(self):
+        """gather[t][j] = col_idx[t][perm[t][j]]."""
+        return np.take_along_axis(self.col_idx, self.perm.astype(np.int64), axis=1)
+
+
+def reorder(A, P=128, mode=0, panels=None) -> Format:
+    """O2: canonical reorder CR1 of A (M x K fp16), panels of P rows.
+    mode 0 = SPTC (paper), 1 = DENSE residual.  ``panels`` = (p0, p1) restricts
+    the work to a contiguous panel range (panels are independent)."""
+    A = _bits(A)
+    M, K = A.shape
+    npan = (M + P - 1) // P
+    p0, p1 = (0, npan) if panels is None else panels
+    h = lib().orc_reorder_range(_ptr(A), M, K, P, mode, p0, p1)
+    if not h:
+        raise ValueError("orc_reorder_range failed")
+    try:
+        sz = np.zeros(4, dtype=np.int64)
+        lib().orc_format_sizes(h, _ptr(sz))
+        npn, nt, nd, P_ = (int(x) for x in sz)
+        T = np.zeros(npn, np.int64)
+        D = np.zeros(npn, np.int64)
+        col_idx = np.zeros((nt, 16), np.int32)
+        perm = np.zeros((nt, 16), np.uint8)
+        vals = np.zeros((nt, P, 8), np.uint16)
+        meta = np.zeros((nt, P), np.uint16)
+        kind = np.zeros(nt, np.uint8)
+        nevict = np.zeros(nt, np.uint8)
+        rcol = np.zeros((nd, 16), np.int32)
+        dvals = np.zeros((nd, P, 16), np.uint16)
+        lib().orc_format_copy(h, _ptr(T), _ptr(D), _ptr(col_idx), _ptr(perm), _ptr(vals),
+                              _ptr(meta), _ptr(kind), _ptr(nevict), _ptr(rcol), _ptr(dvals))
+    finally:
+        lib().orc_format_free(h)
+    return Format(M, K, P, mode, range(p0, p1), T, D, col_idx, perm, vals, meta, kind,
+                  nevict, rcol, dvals)
+
+
+from .check import check_format, decode, format_bytes, canon  # noqa: E402,F401
