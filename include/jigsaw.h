@@ -1,0 +1,172 @@
+/*
+ * jigsaw.h -- C ABI of libjigsaw.so, the B200 (sm_100a) hot path of
+ *   "Jigsaw: Accelerating SpMM with Vector Sparsity on Sparse Tensor Core"
+ *   (Zhang, Liu et al., ICPP '24).
+ *
+ * Problem statement: C = A x B, where A (M x K) is a
+ * vector-pruned sparse fp16 matrix (1-D column vectors of width v) and
+ * B (K x N) is a dense fp16 matrix.  A is prepared once by the
+ * multi-granularity sparsity reorder (Alg. 1) into the reorder-aware
+ * storage format; the product then runs on the sm_100a sparse tensor
+ * cores (tcgen05.mma.sp, 2:4).
+ *
+ * Conventions for every call:
+ *   - Plain C99 types only.  Device pointers are CUDA device addresses on the
+ *     CURRENT device; host pointers are ordinary (pageable or pinned) memory.
+ *   - Matrices are row-major fp16 (IEEE binary16) with the leading dimension
+ *     equal to the column count: A has ld = K, B has ld = N, C has ld = N.
+ *   - Errors never abort: a call returns a status (or NULL) and records it in a
+ *     thread-local slot readable with jigsaw_last_status() /
+ *     jigsaw_last_error_string().
+ *   - Zero test (DESIGN.md R-Q3): an fp16 entry is a nonzero iff
+ *     (bits & 0x7FFF) != 0; -0 and +0 are zeros.  Non-finite values are carried
+ *     but are outside the numerical tolerance contract.
+ */
+#ifndef JIGSAW_H_
+#define JIGSAW_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define JIGSAW_API __attribute__((visibility("default")))
+#else
+#define JIGSAW_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct jigsaw_handle_s* jigsaw_handle_t; /* opaque, immutable after creation */
+typedef struct CUstream_st* jigsaw_stream_t;     /* a cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+  JIGSAW_SUCCESS = 0,
+  JIGSAW_ERROR_INVALID_VALUE = 1, /* null pointer, bad size, misaligned buffer, bad option */
+  JIGSAW_ERROR_UNSUPPORTED = 2,   /* no sm_100 device, or an option not built into this library */
+  JIGSAW_ERROR_OUT_OF_MEMORY = 3, /* device allocation failed */
+  JIGSAW_ERROR_CUDA = 4,          /* a CUDA runtime/driver call failed (message attached) */
+  JIGSAW_ERROR_WRONG_DEVICE = 5,  /* current device differs from the handle's device */
+  JIGSAW_ERROR_INTERNAL = 6       /* a builder invariant failed (bug) */
+} jigsaw_status_t;
+
+/* Residual handling for columns evicted by the reorder retry. */
+typedef enum {
+  JIGSAW_RESIDUAL_SPTC = 0, /* paper: evicted columns re-queued into later 2:4 tiles (default) */
+  JIGSAW_RESIDUAL_DENSE = 1 /* evicted columns form a dense tail run on dense tensor cores */
+} jigsaw_residual_mode_t;
+
+typedef struct {
+  int panel_rows;    /* rows per panel (the BLOCK_TILE analogue, R-Q5/R-Q6); 128 */
+  int residual_mode; /* jigsaw_residual_mode_t */
+  int reserved[6];   /* must be zero */
+} jigsaw_options_t;
+
+/* Statistics of a prepared matrix (jigsaw_get_info). */
+typedef struct {
+  int64_t M, K;            /* shape of A */
+  int32_t v;               /* vector width given at reorder (recorded, not used: R-Q22) */
+  int32_t panel_rows;      /* P */
+  int32_t residual_mode;   /* jigsaw_residual_mode_t */
+  int32_t device;          /* CUDA ordinal the handle lives on */
+  int64_t npanels;         /* ceil(M / P) */
+  int64_t ntiles;          /* sum_p T_p: 2:4 tiles of 16 logical columns */
+  int64_t ndtiles;         /* sum_p D_p: dense residual tiles (DENSE mode) */
+  int64_t overflow_tiles;  /* tiles beyond ceil(K_p/16) per panel (SPTC mode) */
+  int64_t evictions;       /* total columns moved by the reorder retry */
+  int64_t nnz;             /* nonzero entries of A */
+  int64_t kp_total;        /* sum_p K_p (non-zero columns per panel) */
+  int64_t max_tiles;       /* max_p T_p */
+  int64_t nksteps;         /* sum_p ceil(T_p/2): sparse MMA k-steps (32 logical columns) */
+  int64_t format_bytes;    /* canonical format size: per tile 16P + 2P + 64 B (DESIGN.md R-Q19) */
+  int64_t device_bytes;    /* device memory held by the handle */
+  double reorder_ms;       /* device time of the reorder/format build */
+} jigsaw_info_t;
+
+/* Caller-allocated host buffers for jigsaw_export_format; any member may be
+ * NULL (skipped).  Sizes come from jigsaw_get_info (P = panel_rows). */
+typedef struct {
+  int64_t* T;        /* [npanels]          2:4 tiles per panel */
+  int64_t* D;        /* [npanels]          dense residual tiles per panel */
+  int32_t* col_idx;  /* [ntiles][16]       columns in pop order; -1 = PAD (col_idx_array) */
+  uint8_t* perm;     /* [ntiles][16]       MMA_TILE column order (block_col_idx_array) */
+  int32_t* gather;   /* [ntiles][16]       col_idx[perm[j]], read back from the device layout */
+  uint16_t* vals;    /* [ntiles][P][8]     kept fp16 bits, decoded from the device layout */
+  uint16_t* meta;    /* [ntiles][P]        2:4 metadata, nibble q = i0+4*i1 (sptc_col_idx_array) */
+  uint8_t* kind;     /* [ntiles]           0 = main tile, 1 = overflow tile */
+  uint8_t* nevict;   /* [ntiles]           evictions performed while building that tile */
+  int32_t* rcol;     /* [ndtiles][16]      DENSE mode residual columns, -1 = PAD */
+  uint16_t* dvals;   /* [ndtiles][P][16]   DENSE mode residual fp16 bits */
+} jigsaw_format_host_t;
+
+/* ---------------------------------------------------------------- north-star calls */
+
+/* Multi-granularity sparsity reorder + reorder-aware format, with the
+ * default options (P = 128, SPTC residual).
+ *   A : device pointer, fp16 row-major M x K (ld = K), read-only, borrowed for the
+ *       duration of the call (the handle keeps no reference to it).
+ *   M, K > 0;  v in {1, 2, 4, 8} with M % v == 0 (v is validated and recorded).
+ * Runs on the current device, synchronously (returns after the build finished).
+ * Returns a new handle, or NULL on error (see jigsaw_last_status()). */
+JIGSAW_API jigsaw_handle_t jigsaw_reorder(const void* A, int64_t M, int64_t K, int v);
+
+/* C = A x B on sparse tensor cores, beta = 0: every element of C is written
+ * (rows of an all-zero panel are written as zeros).
+ *   B : device pointer, fp16 row-major K x N (ld = N), 16-byte aligned.
+ *   C : device pointer, fp16 row-major M x N (ld = N), 16-byte aligned; overwritten.
+ *   N > 0, N % 8 == 0 (TMA needs 16-byte rows).
+ * Asynchronous on `stream`; no host synchronisation and no allocation.  The handle
+ * is immutable, so calls may run concurrently on several streams.  C must not
+ * alias B. */
+JIGSAW_API jigsaw_status_t jigsaw_spmm(jigsaw_handle_t h, const void* B, int64_t N, void* C,
+                            jigsaw_stream_t stream);
+
+/* Releases the handle's device memory (synchronises the handle's device first).
+ * NULL is a no-op. */
+JIGSAW_API void jigsaw_free(jigsaw_handle_t h);
+
+/* ---------------------------------------------------------------- support calls */
+
+JIGSAW_API jigsaw_status_t jigsaw_last_status(void);       /* thread-local, last call's status */
+JIGSAW_API const char* jigsaw_last_error_string(void);     /* thread-local, valid until the next call */
+JIGSAW_API const char* jigsaw_version(void);               /* static string */
+
+/* jigsaw_reorder with explicit options and stream (opt == NULL: defaults).
+ * Synchronous like jigsaw_reorder; *out receives the handle (NULL on error). */
+JIGSAW_API jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v,
+                                  const jigsaw_options_t* opt, jigsaw_stream_t stream,
+                                  jigsaw_handle_t* out);
+
+/* Same as jigsaw_reorder_ex but A is a HOST pointer (copied to the device inside). */
+JIGSAW_API jigsaw_status_t jigsaw_reorder_host(const void* A_host, int64_t M, int64_t K, int v,
+                                    const jigsaw_options_t* opt, jigsaw_stream_t stream,
+                                    jigsaw_handle_t* out);
+
+JIGSAW_API jigsaw_status_t jigsaw_get_info(jigsaw_handle_t h, jigsaw_info_t* out);
+
+/* Copies the canonical format to caller-allocated host buffers (synchronous).
+ * gather/vals/meta are reconstructed from the DEVICE layout the kernel consumes,
+ * so a layout bug shows up as a mismatch against the oracle. */
+JIGSAW_API jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* out);
+
+/* C = A x B with B and C in HOST memory (end-to-end path): copies B in, runs
+ * jigsaw_spmm, copies C out, all on `stream`, then synchronises `stream`.
+ * Device staging buffers are taken from the stream-ordered allocator. */
+JIGSAW_API jigsaw_status_t jigsaw_spmm_host(jigsaw_handle_t h, const void* B_host, int64_t N, void* C_host,
+                                 jigsaw_stream_t stream);
+
+/* `count` independent products Cs[i] = A_i x Bs[i] (handles on the same device),
+ * issued back to back on `stream` (the batch of independent matrices, C5a). */
+JIGSAW_API jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const* Bs,
+                                    const int64_t* Ns, void* const* Cs, int count,
+                                    jigsaw_stream_t stream);
+
+/* Number of kernels the last successful jigsaw_spmm issued per call (for launch
+ * accounting in benchmarks); reorder kernels are not counted. */
+JIGSAW_API int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* JIGSAW_H_ */

@@ -1,0 +1,230 @@
+"""Python binding of libjigsaw.so (include/jigsaw.h) -- argument marshalling only.
+
+Every step of the hot path (reorder R1..R5, SpMM S1) runs in the CUDA kernels of
+``csrc/``; this module only passes pointers, sizes and streams through ctypes.
+PyTorch is used for device memory and streams.  There is no CPU fallback: if the
+library is missing or the device is not sm_100a, the calls raise.
+
+Names follow the paper's problem statement and the north-star
+calls: ``reorder(A, v)`` -> Handle (jigsaw_reorder), ``Handle.spmm(B)``
+(jigsaw_spmm), ``Handle.free()`` (jigsaw_free).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import _build
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libjigsaw.so")
+
+STATUS = {0: "SUCCESS", 1: "INVALID_VALUE", 2: "UNSUPPORTED", 3: "OUT_OF_MEMORY", 4: "CUDA",
+          5: "WRONG_DEVICE", 6: "INTERNAL"}
+
+# Every symbol include/jigsaw.h declares (tests check the library exports all of them).
+ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_status",
+               "jigsaw_last_error_string", "jigsaw_version", "jigsaw_reorder_ex",
+               "jigsaw_reorder_host", "jigsaw_get_info", "jigsaw_export_format",
+               "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_launches_per_call"]
+
+
+class JigsawError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"jigsaw error {STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class Options(ctypes.Structure):
+    _fields_ = [("panel_rows", ctypes.c_int), ("residual_mode", ctypes.c_int),
+                ("reserved", ctypes.c_int * 6)]
+
+
+class Info(ctypes.Structure):
+    _fields_ = [("M", ctypes.c_int64), ("K", ctypes.c_int64), ("v", ctypes.c_int32),
+                ("panel_rows", ctypes.c_int32), ("residual_mode", ctypes.c_int32),
+                ("device", ctypes.c_int32), ("npanels", ctypes.c_int64), ("ntiles", ctypes.c_int64),
+                ("ndtiles", ctypes.c_int64), ("overflow_tiles", ctypes.c_int64),
+                ("evictions", ctypes.c_int64), ("nnz", ctypes.c_int64), ("kp_total", ctypes.c_int64),
+                ("max_tiles", ctypes.c_int64), ("nksteps", ctypes.c_int64),
+                ("format_bytes", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
+                ("reorder_ms", ctypes.c_double)]
+
+
+class FormatHost(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_void_p) for n in
+                ("T", "D", "col_idx", "perm", "gather", "vals", "meta", "kind", "nevict", "rcol", "dvals")]
+
+
+_lib = None
+
+
+def lib(build_if_missing: bool = True):
+    """Load libjigsaw.so (building it with nvcc first if it is absent or stale)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if build_if_missing:
+        try:
+            _build.build()
+        except Exception:
+            if not os.path.exists(LIB_PATH):
+                raise
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"libjigsaw.so not built ({LIB_PATH}); run __graft_entry__.build()")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, i64, ci = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+    sig = {
+        "jigsaw_reorder": (vp, [vp, i64, i64, ci]),
+        "jigsaw_spmm": (ci, [vp, vp, i64, vp, vp]),
+        "jigsaw_free": (None, [vp]),
+        "jigsaw_last_status": (ci, []),
+        "jigsaw_last_error_string": (ctypes.c_char_p, []),
+        "jigsaw_version": (ctypes.c_char_p, []),
+        "jigsaw_reorder_ex": (ci, [vp, i64, i64, ci, ctypes.POINTER(Options), vp, ctypes.POINTER(vp)]),
+        "jigsaw_reorder_host": (ci, [vp, i64, i64, ci, ctypes.POINTER(Options), vp, ctypes.POINTER(vp)]),
+        "jigsaw_get_info": (ci, [vp, ctypes.POINTER(Info)]),
+        "jigsaw_export_format": (ci, [vp, ctypes.POINTER(FormatHost)]),
+        "jigsaw_spmm_host": (ci, [vp, vp, i64, vp, vp]),
+        "jigsaw_spmm_batched": (ci, [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(i64),
+                                     ctypes.POINTER(vp), ci, vp]),
+        "jigsaw_spmm_launches_per_call": (ci, [vp, i64]),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(L, name)
+        fn.restype = res
+        fn.argtypes = args
+    _lib = L
+    return L
+
+
+def _raise_if(status: int):
+    if status != 0:
+        raise JigsawError(status, lib().jigsaw_last_error_string().decode())
+
+
+def version() -> str:
+    return lib().jigsaw_version().decode()
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return ctypes.c_void_p(stream)
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _check_fp16_cuda(t, name):
+    import torch
+    if not isinstance(t, torch.Tensor) or t.dtype != torch.float16 or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA float16 tensor")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous (row-major)")
+
+
+class Handle:
+    """A prepared matrix (jigsaw_handle_t): the reorder-aware format on the device."""
+
+    def __init__(self, ptr: int):
+        self._h = ctypes.c_void_p(ptr)
+
+    @property
+    def ptr(self):
+        return self._h
+
+    def info(self) -> dict:
+        out = Info()
+        _raise_if(lib().jigsaw_get_info(self._h, ctypes.byref(out)))
+        return {n: getattr(out, n) for n, _ in Info._fields_}
+
+    def spmm(self, B, C=None, stream=None):
+        """C = A x B (jigsaw_spmm); B: CUDA fp16 K x N; returns C (M x N fp16)."""
+        import torch
+        _check_fp16_cuda(B, "B")
+        inf = self.info()
+        K, N = B.shape
+        if K != inf["K"]:
+            raise ValueError(f"B has {K} rows, A has K = {inf['K']}")
+        if C is None:
+            C = torch.empty((inf["M"], N), dtype=torch.float16, device=B.device)
+        else:
+            _check_fp16_cuda(C, "C")
+        _raise_if(lib().jigsaw_spmm(self._h, ctypes.c_void_p(B.data_ptr()), N,
+                                    ctypes.c_void_p(C.data_ptr()), _stream_ptr(stream)))
+        return C
+
+    def spmm_host(self, B: np.ndarray, stream=None) -> np.ndarray:
+        """End-to-end path (jigsaw_spmm_host): host B in, host C out."""
+        B = np.ascontiguousarray(B)
+        if B.dtype == np.float16:
+            B = B.view(np.uint16)
+        inf = self.info()
+        C = np.empty((inf["M"], B.shape[1]), dtype=np.uint16)
+        _raise_if(lib().jigsaw_spmm_host(self._h, B.ctypes.data_as(ctypes.c_void_p), B.shape[1],
+                                         C.ctypes.data_as(ctypes.c_void_p),
+                                         _stream_ptr(stream) if stream is not None else None))
+        return C
+
+    def export(self) -> dict:
+        """Canonical format (jigsaw_export_format) as numpy arrays."""
+        inf = self.info()
+        npan, nt, nd, P = inf["npanels"], inf["ntiles"], inf["ndtiles"], inf["panel_rows"]
+        arr = dict(T=np.zeros(npan, np.int64), D=np.zeros(npan, np.int64),
+                   col_idx=np.zeros((nt, 16), np.int32), perm=np.zeros((nt, 16), np.uint8),
+                   gather=np.zeros((nt, 16), np.int32), vals=np.zeros((nt, P, 8), np.uint16),
+                   meta=np.zeros((nt, P), np.uint16), kind=np.zeros(nt, np.uint8),
+                   nevict=np.zeros(nt, np.uint8), rcol=np.zeros((nd, 16), np.int32),
+                   dvals=np.zeros((nd, P, 16), np.uint16))
+        fh = FormatHost(**{k: v.ctypes.data for k, v in arr.items()})
+        _raise_if(lib().jigsaw_export_format(self._h, ctypes.byref(fh)))
+        return arr
+
+    def free(self):
+        if self._h is not None and self._h.value:
+            lib().jigsaw_free(self._h)
+        self._h = ctypes.c_void_p(0)
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, stream=None) -> Handle:
+    """jigsaw_reorder_ex: multi-granularity reorder + format build of A (CUDA fp16 M x K)."""
+    _check_fp16_cuda(A, "A")
+    M, K = A.shape
+    opt = Options(panel_rows, residual_mode)
+    out = ctypes.c_void_p(0)
+    _raise_if(lib().jigsaw_reorder_ex(ctypes.c_void_p(A.data_ptr()), M, K, v, ctypes.byref(opt),
+                                      _stream_ptr(stream), ctypes.byref(out)))
+    return Handle(out.value)
+
+
+def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: int = 0) -> Handle:
+    """jigsaw_reorder_host: A given as a host array (fp16 or uint16 bits)."""
+    A = np.ascontiguousarray(A)
+    if A.dtype == np.float16:
+        A = A.view(np.uint16)
+    M, K = A.shape
+    opt = Options(panel_rows, residual_mode)
+    out = ctypes.c_void_p(0)
+    _raise_if(lib().jigsaw_reorder_host(A.ctypes.data_as(ctypes.c_void_p), M, K, v,
+                                        ctypes.byref(opt), None, ctypes.byref(out)))
+    return Handle(out.value)
+
+
+def spmm_batched(handles, Bs, Cs, stream=None):
+    """jigsaw_spmm_batched: independent products issued back to back on one stream."""
+    n = len(handles)
+    hs = (ctypes.c_void_p * n)(*[h.ptr.value for h in handles])
+    bp = (ctypes.c_void_p * n)(*[b.data_ptr() for b in Bs])
+    cp = (ctypes.c_void_p * n)(*[c.data_ptr() for c in Cs])
+    ns = (ctypes.c_int64 * n)(*[b.shape[1] for b in Bs])
+    _raise_if(lib().jigsaw_spmm_batched(hs, bp, ns, cp, n, _stream_ptr(stream)))
+    return Cs

@@ -1,0 +1,305 @@
+// api.cu -- the C ABI of libjigsaw.so (include/jigsaw.h): validation, handle
+// lifetime, status reporting, export of the canonical format, launches.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "internal.h"
+
+struct jigsaw_handle_s {
+  jig::Format f;
+};
+
+namespace jig {
+
+namespace {
+thread_local jigsaw_status_t t_status = JIGSAW_SUCCESS;
+thread_local std::string t_msg;
+}  // namespace
+
+jigsaw_status_t set_status(jigsaw_status_t s, const std::string& msg) {
+  t_status = s;
+  t_msg = msg;
+  return s;
+}
+
+jigsaw_status_t cuda_status(cudaError_t e, const char* what) {
+  cudaGetLastError();  // clear sticky-free errors
+  return set_status(JIGSAW_ERROR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+namespace {
+
+jigsaw_status_t check_device(int* dev_out) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_status(JIGSAW_ERROR_UNSUPPORTED, std::string("no CUDA device: ") + cudaGetErrorString(e));
+  }
+  int major = 0, minor = 0;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+  cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+  if (major != 10 || minor != 0)
+    return set_status(JIGSAW_ERROR_UNSUPPORTED, "libjigsaw is built for sm_100a (B200); device " +
+                                                    std::to_string(dev) + " is sm_" + std::to_string(major) +
+                                                    std::to_string(minor));
+  *dev_out = dev;
+  return JIGSAW_SUCCESS;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, const jigsaw_options_t* opt) {
+  if (!A) return set_status(JIGSAW_ERROR_INVALID_VALUE, "A is NULL");
+  if (M <= 0 || K <= 0) return set_status(JIGSAW_ERROR_INVALID_VALUE, "M and K must be positive");
+  if (K > (int64_t)1 << 30 || M > (int64_t)1 << 31)
+    return set_status(JIGSAW_ERROR_INVALID_VALUE, "M or K too large");
+  if (!(v == 1 || v == 2 || v == 4 || v == 8)) return set_status(JIGSAW_ERROR_INVALID_VALUE, "v must be 1, 2, 4 or 8");
+  if (M % v) return set_status(JIGSAW_ERROR_INVALID_VALUE, "M must be a multiple of v");
+  if (opt) {
+    if (opt->panel_rows != kPanelRows)
+      return set_status(opt->panel_rows == 64 ? JIGSAW_ERROR_UNSUPPORTED : JIGSAW_ERROR_INVALID_VALUE,
+                        "panel_rows must be 128 (64 is not built in this version)");
+    if (opt->residual_mode == JIGSAW_RESIDUAL_DENSE)
+      return set_status(JIGSAW_ERROR_UNSUPPORTED, "DENSE residual mode is not built in this version");
+    if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC)
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
+    for (int i = 0; i < 6; ++i)
+      if (opt->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved options must be zero");
+  }
+  return JIGSAW_SUCCESS;
+}
+
+jigsaw_status_t validate_spmm(jigsaw_handle_t h, const void* B, int64_t N, const void* C, bool device_ptrs) {
+  if (!h) return set_status(JIGSAW_ERROR_INVALID_VALUE, "handle is NULL");
+  if (!B || !C) return set_status(JIGSAW_ERROR_INVALID_VALUE, "B or C is NULL");
+  if (N <= 0 || N % 8) return set_status(JIGSAW_ERROR_INVALID_VALUE, "N must be a positive multiple of 8");
+  if (N > (int64_t)1 << 30) return set_status(JIGSAW_ERROR_INVALID_VALUE, "N too large");
+  if (device_ptrs && (!aligned16(B) || !aligned16(C)))
+    return set_status(JIGSAW_ERROR_INVALID_VALUE, "B and C must be 16-byte aligned");
+  int dev = -1;
+  cudaGetDevice(&dev);
+  if (dev != h->f.device) return set_status(JIGSAW_ERROR_WRONG_DEVICE, "current device differs from the handle's");
+  return JIGSAW_SUCCESS;
+}
+
+}  // namespace
+}  // namespace jig
+
+using namespace jig;
+
+extern "C" {
+
+jigsaw_status_t jigsaw_last_status(void) { return t_status; }
+const char* jigsaw_last_error_string(void) { return t_msg.c_str(); }
+const char* jigsaw_version(void) { return "jigsaw-b200 0.1 (sm_100a, tcgen05.mma.sp)"; }
+
+jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, const jigsaw_options_t* opt,
+                                  jigsaw_stream_t stream, jigsaw_handle_t* out) {
+  if (!out) return set_status(JIGSAW_ERROR_INVALID_VALUE, "out is NULL");
+  *out = nullptr;
+  jigsaw_status_t s = validate_reorder(A, M, K, v, opt);
+  if (s != JIGSAW_SUCCESS) return s;
+  if (!aligned16(A)) return set_status(JIGSAW_ERROR_INVALID_VALUE, "A must be 16-byte aligned");
+  int dev = 0;
+  if ((s = check_device(&dev)) != JIGSAW_SUCCESS) return s;
+  jigsaw_handle_s* h = new (std::nothrow) jigsaw_handle_s();
+  if (!h) return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "host allocation failed");
+  set_status(JIGSAW_SUCCESS);
+  s = build_format(static_cast<const uint16_t*>(A), M, K, v, kPanelRows, JIGSAW_RESIDUAL_SPTC,
+                   reinterpret_cast<cudaStream_t>(stream), &h->f);
+  if (s != JIGSAW_SUCCESS) {
+    delete h;
+    return s;
+  }
+  *out = h;
+  return set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_handle_t jigsaw_reorder(const void* A, int64_t M, int64_t K, int v) {
+  jigsaw_handle_t h = nullptr;
+  jigsaw_reorder_ex(A, M, K, v, nullptr, nullptr, &h);
+  return h;
+}
+
+jigsaw_status_t jigsaw_reorder_host(const void* A_host, int64_t M, int64_t K, int v, const jigsaw_options_t* opt,
+                                    jigsaw_stream_t stream, jigsaw_handle_t* out) {
+  if (!out) return set_status(JIGSAW_ERROR_INVALID_VALUE, "out is NULL");
+  *out = nullptr;
+  jigsaw_status_t s = validate_reorder(A_host, M, K, v, opt);
+  if (s != JIGSAW_SUCCESS) return s;
+  int dev = 0;
+  if ((s = check_device(&dev)) != JIGSAW_SUCCESS) return s;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  void* dA = nullptr;
+  const size_t bytes = (size_t)M * K * 2;
+  cudaError_t e = cudaMallocAsync(&dA, bytes, st);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "cudaMallocAsync(A) failed");
+  }
+  e = cudaMemcpyAsync(dA, A_host, bytes, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) {
+    cudaFreeAsync(dA, st);
+    return cuda_status(e, "copy A to device");
+  }
+  s = jigsaw_reorder_ex(dA, M, K, v, opt, stream, out);
+  cudaFreeAsync(dA, st);
+  cudaStreamSynchronize(st);
+  return s;
+}
+
+jigsaw_status_t jigsaw_spmm(jigsaw_handle_t h, const void* B, int64_t N, void* C, jigsaw_stream_t stream) {
+  jigsaw_status_t s = validate_spmm(h, B, N, C, true);
+  if (s != JIGSAW_SUCCESS) return s;
+  s = launch_spmm(h->f, B, N, C, reinterpret_cast<cudaStream_t>(stream));
+  if (s != JIGSAW_SUCCESS) return s;
+  return set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_status_t jigsaw_spmm_host(jigsaw_handle_t h, const void* B_host, int64_t N, void* C_host,
+                                 jigsaw_stream_t stream) {
+  jigsaw_status_t s = validate_spmm(h, B_host, N, C_host, false);
+  if (s != JIGSAW_SUCCESS) return s;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const size_t bbytes = (size_t)h->f.K * N * 2, cbytes = (size_t)h->f.M * N * 2;
+  void *dB = nullptr, *dC = nullptr;
+  cudaError_t e = cudaMallocAsync(&dB, bbytes, st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&dC, cbytes, st);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    if (dB) cudaFreeAsync(dB, st);
+    return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "cudaMallocAsync(B/C) failed");
+  }
+  e = cudaMemcpyAsync(dB, B_host, bbytes, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) {
+    s = launch_spmm(h->f, dB, N, dC, st);
+    if (s == JIGSAW_SUCCESS) e = cudaMemcpyAsync(C_host, dC, cbytes, cudaMemcpyDeviceToHost, st);
+  }
+  cudaFreeAsync(dB, st);
+  cudaFreeAsync(dC, st);
+  cudaError_t e2 = cudaStreamSynchronize(st);
+  if (s != JIGSAW_SUCCESS) return s;
+  if (e != cudaSuccess) return cuda_status(e, "jigsaw_spmm_host copies");
+  if (e2 != cudaSuccess) return cuda_status(e2, "jigsaw_spmm_host");
+  return set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const* Bs, const int64_t* Ns,
+                                    void* const* Cs, int count, jigsaw_stream_t stream) {
+  if (count < 0 || (count > 0 && (!hs || !Bs || !Ns || !Cs)))
+    return set_status(JIGSAW_ERROR_INVALID_VALUE, "bad batch arguments");
+  for (int i = 0; i < count; ++i) {
+    jigsaw_status_t s = validate_spmm(hs[i], Bs[i], Ns[i], Cs[i], true);
+    if (s != JIGSAW_SUCCESS) return s;
+  }
+  for (int i = 0; i < count; ++i) {
+    jigsaw_status_t s = launch_spmm(hs[i]->f, Bs[i], Ns[i], Cs[i], reinterpret_cast<cudaStream_t>(stream));
+    if (s != JIGSAW_SUCCESS) return s;
+  }
+  return set_status(JIGSAW_SUCCESS);
+}
+
+int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N) {
+  (void)h;
+  (void)N;
+  return 1;
+}
+
+void jigsaw_free(jigsaw_handle_t h) {
+  if (!h) return;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  if (cur != h->f.device) cudaSetDevice(h->f.device);
+  cudaDeviceSynchronize();
+  free_format(&h->f);
+  if (cur != h->f.device) cudaSetDevice(cur);
+  delete h;
+  set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_status_t jigsaw_get_info(jigsaw_handle_t h, jigsaw_info_t* out) {
+  if (!h || !out) return set_status(JIGSAW_ERROR_INVALID_VALUE, "NULL argument");
+  const Format& f = h->f;
+  memset(out, 0, sizeof *out);
+  out->M = f.M;
+  out->K = f.K;
+  out->v = f.v;
+  out->panel_rows = f.P;
+  out->residual_mode = f.mode;
+  out->device = f.device;
+  out->npanels = f.npanels;
+  out->ntiles = f.ntiles;
+  out->ndtiles = f.ndtiles;
+  out->overflow_tiles = f.overflow_tiles;
+  out->evictions = f.evictions;
+  out->nnz = f.nnz;
+  out->kp_total = f.kp_total;
+  out->max_tiles = f.max_tiles;
+  out->nksteps = f.nksteps;
+  out->format_bytes = (int64_t)(16 * f.P + 2 * f.P + 64) * f.ntiles + (int64_t)(32 * f.P + 64) * f.ndtiles;
+  out->device_bytes = f.device_bytes;
+  out->reorder_ms = f.reorder_ms;
+  return set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* out) {
+  if (!h || !out) return set_status(JIGSAW_ERROR_INVALID_VALUE, "NULL argument");
+  const Format& f = h->f;
+  int cur = -1;
+  cudaGetDevice(&cur);
+  if (cur != f.device) return set_status(JIGSAW_ERROR_WRONG_DEVICE, "current device differs from the handle's");
+  const int64_t nt = f.ntiles, P = f.P;
+  if (out->T)
+    for (int64_t p = 0; p < f.npanels; ++p) out->T[p] = f.T[p];
+  if (out->D)
+    for (int64_t p = 0; p < f.npanels; ++p) out->D[p] = f.D.empty() ? 0 : f.D[p];
+  cudaError_t e = cudaSuccess;
+  if (nt && out->col_idx && e == cudaSuccess) e = cudaMemcpy(out->col_idx, f.d_colidx, nt * 16 * 4, cudaMemcpyDeviceToHost);
+  if (nt && out->perm && e == cudaSuccess) e = cudaMemcpy(out->perm, f.d_perm, nt * 16, cudaMemcpyDeviceToHost);
+  if (nt && out->kind && e == cudaSuccess) e = cudaMemcpy(out->kind, f.d_kind, nt, cudaMemcpyDeviceToHost);
+  if (nt && out->nevict && e == cudaSuccess) e = cudaMemcpy(out->nevict, f.d_nevict, nt, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_status(e, "export copy");
+  if (nt && (out->gather || out->vals || out->meta)) {
+    // read back the device layout and invert it
+    std::vector<uint8_t> A((size_t)f.nksteps * kKStepBytesA);
+    std::vector<uint32_t> E((size_t)f.nkblocks * 512);
+    std::vector<int32_t> G((size_t)f.nksteps * 32);
+    e = cudaMemcpy(A.data(), f.d_Aimg, A.size(), cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess) e = cudaMemcpy(E.data(), f.d_Eimg, E.size() * 4, cudaMemcpyDeviceToHost);
+    if (e == cudaSuccess) e = cudaMemcpy(G.data(), f.d_G, G.size() * 4, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return cuda_status(e, "export copy (device layout)");
+    for (int64_t p = 0; p < f.npanels; ++p) {
+      for (int t = 0; t < f.T[p]; ++t) {
+        const int64_t ft = f.tile_off[p] + t;
+        const int64_t gks = f.ks_off[p] + t / 2;
+        const int h2 = t & 1;
+        const int64_t kb = f.kb_off[p] + (t / 2) / kStepsPerBlock;
+        const int col = (t / 2) % kStepsPerBlock;
+        if (out->gather)
+          for (int j = 0; j < 16; ++j) {
+            const int32_t g = G[gks * 32 + h2 * 16 + j];
+            out->gather[ft * 16 + j] = g >= f.K ? kPad : g;
+          }
+        for (int r = 0; r < P; ++r) {
+          if (out->vals)
+            memcpy(out->vals + (ft * P + r) * 8, &A[gks * kKStepBytesA + (r >> 3) * 256 + h2 * 128 + (r & 7) * 16], 16);
+          if (out->meta) {
+            const int m2 = r >> 4, m0 = r & 7, hi = (r >> 3) & 1;
+            const int L = m0 + 8 * h2 + 16 * m2;
+            const uint32_t w = E[(kb * 128 + L) * 4 + col];
+            out->meta[ft * P + r] = (uint16_t)(hi ? (w >> 16) : (w & 0xFFFF));
+          }
+        }
+      }
+    }
+  }
+  return set_status(JIGSAW_SUCCESS);
+}
+
+}  // extern "C"

@@ -1,0 +1,62 @@
+// internal.h -- shared declarations of libjigsaw.so (host side + kernel launchers).
+// Not part of the ABI (include/jigsaw.h is).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/jigsaw.h"
+
+namespace jig {
+
+constexpr int kTileCols = 16;     // logical columns per tile (the paper's MMA_TILE width)
+constexpr int kPanelRows = 128;   // P = tcgen05 M (R-Q5)
+constexpr int kKStepBytesA = 4096;  // 128 rows x 16 halves (compressed 32 logical) per k-step
+constexpr int kStepsPerBlock = 4;   // k-steps per E block (tcgen05.cp 128x128b = 4 TMEM columns)
+constexpr int kEBlockBytes = 2048;  // 128 lanes x 16 B
+constexpr int kPad = -1;
+
+// Device-resident prepared matrix (the reorder-aware format).
+struct Format {
+  int64_t M = 0, K = 0;
+  int v = 0, P = kPanelRows, mode = 0, device = 0;
+  int64_t npanels = 0, ntiles = 0, nksteps = 0, nkblocks = 0, ndtiles = 0;
+  // host copies of per-panel counts / offsets
+  std::vector<int32_t> T, D, tile_off, ks_off, kb_off;
+  // device per-panel arrays
+  int32_t* d_ksn = nullptr;    // [npanels]   k-steps of the panel = ceil(T_p / 2)
+  int32_t* d_ksoff = nullptr;  // [npanels]   first k-step of the panel
+  int32_t* d_kboff = nullptr;  // [npanels]   first E block of the panel
+  // canonical arrays (device)
+  int32_t* d_colidx = nullptr;  // [ntiles][16]
+  uint8_t* d_perm = nullptr;    // [ntiles][16]
+  uint8_t* d_kind = nullptr;    // [ntiles]
+  uint8_t* d_nevict = nullptr;  // [ntiles]
+  // device layout consumed by the SpMM kernel
+  uint8_t* d_Aimg = nullptr;  // [nksteps][4096]: UMMA K-major no-swizzle core matrices
+  uint8_t* d_Eimg = nullptr;  // [nkblocks][128][4] u32: TMEM metadata lanes
+  int32_t* d_G = nullptr;     // [nksteps][32]: B row per logical column (PAD -> K, TMA zero fill)
+  // stats
+  int64_t nnz = 0, kp_total = 0, evictions = 0, overflow_tiles = 0, max_tiles = 0;
+  int64_t device_bytes = 0;
+  double reorder_ms = 0;
+  std::vector<void*> allocs;
+};
+
+// status plumbing (api.cu)
+jigsaw_status_t set_status(jigsaw_status_t s, const std::string& msg = "");
+jigsaw_status_t cuda_status(cudaError_t e, const char* what);
+
+// reorder.cu: builds *f from device A (M x K fp16) on `stream`; synchronous.
+jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
+                             cudaStream_t stream, Format* f);
+void free_format(Format* f);
+
+// spmm.cu
+jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s);
+int spmm_num_sms();
+
+}  // namespace jig

@@ -1,0 +1,603 @@
+// reorder.cu -- GPU builder of the reorder-aware format (R1..R5).
+//
+//   R1 k_colmask     per panel and column: the P-bit row mask of nonzeros
+//                    (BLOCK_TILE granularity)
+//   R2 k_compact     S_p = ascending list of the panel's nonzero columns
+//                    (col_idx_array; R-Q4)
+//   R3 k_main_tiles  one warp per full 16-column tile of S_p: Alg. 1
+//                    + reorder retry -- tiles are independent
+//   R4 k_overflow    one warp per panel: the remainder of S_p and the evicted
+//                    columns, re-tiled in FIFO order (R-Q12)
+//   R5 k_emit        2:4 compression straight into the device
+//                    layout the SpMM kernel consumes (A image, TMEM metadata
+//                    lanes, B gather rows) + the canonical col_idx / perm
+//
+// The tile search returns the lexicographically first cover (R-Q8) and evicts
+// the real column in the fewest compatible groups, ties to the smallest slot
+// (R-Q11) -- the definition the oracle (oracle/oracle.c) implements
+// independently; tests/test_gpu_parity.py compares the two bit for bit.
+#include <climits>
+#include <cstdio>
+#include <cstring>
+
+#include "internal.h"
+
+namespace jig {
+
+namespace {
+
+constexpr int kNumSubsets = 1820;  // C(16, 4)
+constexpr int kNumG0 = 455;        // 4-subsets containing slot 0 = C(15, 3)
+constexpr unsigned kFull = 0xFFFFFFFFu;
+
+__device__ uint16_t g_subs[kNumSubsets];  // all 4-subsets of 16 slots, lexicographic
+
+bool g_tables_ready[64] = {false};
+
+jigsaw_status_t init_tables(int dev) {
+  if (dev >= 0 && dev < 64 && g_tables_ready[dev]) return JIGSAW_SUCCESS;
+  uint16_t subs[kNumSubsets];
+  int n = 0;
+  for (int a = 0; a < 16; ++a)
+    for (int b = a + 1; b < 16; ++b)
+      for (int c = b + 1; c < 16; ++c)
+        for (int d = c + 1; d < 16; ++d)
+          subs[n++] = (uint16_t)((1u << a) | (1u << b) | (1u << c) | (1u << d));
+  cudaError_t e = cudaMemcpyToSymbol(g_subs, subs, sizeof subs);
+  if (e != cudaSuccess) return cuda_status(e, "cudaMemcpyToSymbol(subsets)");
+  if (dev >= 0 && dev < 64) g_tables_ready[dev] = true;
+  return JIGSAW_SUCCESS;
+}
+
+// ------------------------------------------------------------------ R1
+__global__ void k_colmask(const uint16_t* __restrict__ A, int64_t M, int64_t K, int P,
+                          uint4* __restrict__ masks, unsigned long long* __restrict__ nnz) {
+  const int p = blockIdx.y;
+  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t w[4] = {0, 0, 0, 0};
+  int cnt = 0;
+  if (c < K) {
+    const int64_t row0 = (int64_t)p * P;
+    const int nr = (int)min((int64_t)P, M - row0);
+#pragma unroll 8
+    for (int r = 0; r < nr; ++r) {
+      const uint16_t x = A[(row0 + r) * K + c];
+      if (x & 0x7FFFu) {  // R-Q3: +-0 are zeros
+        w[r >> 5] |= 1u << (r & 31);
+        ++cnt;
+      }
+    }
+    masks[(int64_t)p * K + c] = make_uint4(w[0], w[1], w[2], w[3]);
+  }
+  for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
+  if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(nnz, (unsigned long long)cnt);
+}
+
+// ------------------------------------------------------------------ R2
+__global__ void k_compact(const uint4* __restrict__ masks, int64_t K, int32_t* __restrict__ S,
+                          int32_t* __restrict__ Kp) {
+  __shared__ int wsum[32];
+  __shared__ int total;
+  const int p = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nw = blockDim.x >> 5;
+  int base = 0;
+  for (int64_t c0 = 0; c0 < K; c0 += blockDim.x) {
+    const int64_t c = c0 + tid;
+    bool flag = false;
+    if (c < K) {
+      const uint4 m = masks[(int64_t)p * K + c];
+      flag = (m.x | m.y | m.z | m.w) != 0;
+    }
+    const unsigned b = __ballot_sync(kFull, flag);
+    const int lpre = __popc(b & ((1u << lane) - 1u));
+    if (lane == 0) wsum[warp] = __popc(b);
+    __syncthreads();
+    if (warp == 0) {
+      int x = lane < nw ? wsum[lane] : 0;
+      int incl = x;
+      for (int o = 1; o < 32; o <<= 1) {
+        int y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+      }
+      if (lane < nw) wsum[lane] = incl - x;  // exclusive
+      if (lane == 31) total = incl;
+    }
+    __syncthreads();
+    if (flag) S[(int64_t)p * K + base + wsum[warp] + lpre] = (int32_t)c;
+    base += total;
+    __syncthreads();
+  }
+  if (tid == 0) Kp[p] = base;
+}
+
+// ------------------------------------------------------------------ tile search
+struct TileSmem {
+  uint32_t bitmap[2048];  // compat[S] for every 4-subset S, indexed by the 16-bit slot mask
+  uint4 m[16];            // row masks per slot (PAD: 0)
+  int32_t cols[16];       // column per slot (kPad = -1)
+  int32_t ev[16];         // evicted columns, in eviction order
+  uint8_t perm[16];
+  int nev;
+};
+
+__device__ __forceinline__ bool compat(const TileSmem& s, uint32_t sub) {
+  return (s.bitmap[sub >> 5] >> (sub & 31)) & 1u;
+}
+
+// Lexicographically first completion of the cover given g0 (R-Q8): g1 holds the
+// smallest uncovered slot, candidates tried in lexicographic order; then g2; g3
+// is the rest.
+__device__ bool complete_cover(const TileSmem& s, uint32_t used, uint32_t& o1, uint32_t& o2,
+                               uint32_t& o3) {
+  const int lo1 = __ffs(~used & 0xFFFFu) - 1;
+  const uint32_t av1 = ~used & 0xFFFFu & ~(1u << lo1);
+  for (uint32_t x = av1; x; x &= x - 1) {
+    const int b = __ffs(x) - 1;
+    for (uint32_t y = x & (x - 1); y; y &= y - 1) {
+      const int c = __ffs(y) - 1;
+      for (uint32_t z = y & (y - 1); z; z &= z - 1) {
+        const int d = __ffs(z) - 1;
+        const uint32_t s1 = (1u << lo1) | (1u << b) | (1u << c) | (1u << d);
+        if (!compat(s, s1)) continue;
+        const uint32_t u2 = used | s1;
+        const int lo2 = __ffs(~u2 & 0xFFFFu) - 1;
+        const uint32_t av2 = ~u2 & 0xFFFFu & ~(1u << lo2);
+        for (uint32_t x2 = av2; x2; x2 &= x2 - 1) {
+          const int b2 = __ffs(x2) - 1;
+          for (uint32_t y2 = x2 & (x2 - 1); y2; y2 &= y2 - 1) {
+            const int c2 = __ffs(y2) - 1;
+            for (uint32_t z2 = y2 & (y2 - 1); z2; z2 &= z2 - 1) {
+              const int d2 = __ffs(z2) - 1;
+              const uint32_t s2 = (1u << lo2) | (1u << b2) | (1u << c2) | (1u << d2);
+              if (!compat(s, s2)) continue;
+              const uint32_t s3 = ~(u2 | s2) & 0xFFFFu;
+              if (compat(s, s3)) {
+                o1 = s1; o2 = s2; o3 = s3;
+                return true;
+              }
+            }
+          }
+        }
+      }
+    }
+  }
+  return false;
+}
+
+// Alg. 1 + reorder retry on one tile, executed by one full warp.  On entry
+// s.cols / s.m hold the 16 popped columns; on exit s.cols has evicted slots set
+// to PAD, s.perm the new column order g0||g1||g2||g3, s.ev[0..s.nev) the evictions.
+__device__ void tile_search(TileSmem& s, int lane) {
+  if (lane == 0) s.nev = 0;
+  __syncwarp();
+  uint32_t realset = __ballot_sync(kFull, lane < 16 && s.cols[lane] != kPad) & 0xFFFFu;
+  for (;;) {
+    // Alg. 1 lines 1-8: compatibility of all 1820 4-column groups; a group is
+    // compatible iff no row has >= 3 nonzeros among its 4 columns.
+    for (int i = lane; i < 2048; i += 32) s.bitmap[i] = 0;
+    __syncwarp();
+    int fr = 0, hmax = 0;
+    for (int k0 = 0; k0 < kNumSubsets; k0 += 32) {
+      const int k = k0 + lane;
+      bool ok = false;
+      uint32_t sub = 0;
+      if (k < kNumSubsets) {
+        sub = g_subs[k];
+        uint32_t r = sub;
+        const int a = __ffs(r) - 1; r &= r - 1;
+        const int b = __ffs(r) - 1; r &= r - 1;
+        const int c = __ffs(r) - 1; r &= r - 1;
+        const int d = __ffs(r) - 1;
+        const uint4 ma = s.m[a], mb = s.m[b], mc = s.m[c], md = s.m[d];
+        const uint32_t bad = ((ma.x & mb.x & (mc.x | md.x)) | (mc.x & md.x & (ma.x | mb.x))) |
+                             ((ma.y & mb.y & (mc.y | md.y)) | (mc.y & md.y & (ma.y | mb.y))) |
+                             ((ma.z & mb.z & (mc.z | md.z)) | (mc.z & md.z & (ma.z | mb.z))) |
+                             ((ma.w & mb.w & (mc.w | md.w)) | (mc.w & md.w & (ma.w | mb.w)));
+        ok = bad == 0;
+        if (ok) {
+          atomicOr(&s.bitmap[sub >> 5], 1u << (sub & 31));
+          hmax = max(hmax, __popc(sub & realset));
+        }
+      }
+      // freq[j] = number of compatible groups containing slot j
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const unsigned bj = __ballot_sync(kFull, ok && ((sub >> j) & 1u));
+        if (lane == j) fr += __popc(bj);
+      }
+    }
+    for (int o = 16; o; o >>= 1) hmax = max(hmax, __shfl_xor_sync(kFull, hmax, o));
+    __syncwarp();
+    // Necessary conditions for a cover (they only skip searches that must fail):
+    // every slot lies in some compatible group; 4 groups can hold all real columns.
+    const bool coverable = __all_sync(kFull, lane >= 16 || fr > 0) && hmax * 4 >= __popc(realset);
+    // Alg. 1 lines 9-17: lanes try the candidates for g0 (groups containing slot 0)
+    // in lexicographic order, 32 at a time; the lowest successful one wins.
+    if (coverable) {
+      for (int k0 = 0; k0 < kNumG0; k0 += 32) {
+        const int k = k0 + lane;
+        uint32_t g0 = 0, a1 = 0, a2 = 0, a3 = 0;
+        bool ok = false;
+        if (k < kNumG0) {
+          g0 = g_subs[k];
+          ok = compat(s, g0) && complete_cover(s, g0, a1, a2, a3);
+        }
+        const unsigned b = __ballot_sync(kFull, ok);
+        if (b) {
+          const int w = __ffs(b) - 1;
+          g0 = __shfl_sync(kFull, g0, w);
+          a1 = __shfl_sync(kFull, a1, w);
+          a2 = __shfl_sync(kFull, a2, w);
+          a3 = __shfl_sync(kFull, a3, w);
+          if (lane == 0) {
+            int o = 0;
+            const uint32_t gs[4] = {g0, a1, a2, a3};
+            for (int g = 0; g < 4; ++g)
+              for (uint32_t x = gs[g]; x; x &= x - 1) s.perm[o++] = (uint8_t)(__ffs(x) - 1);
+          }
+          __syncwarp();
+          return;
+        }
+      }
+    }
+    // Reorder retry: evict the least frequent real column (ties: smallest slot).
+    const int key = (lane < 16 && ((realset >> lane) & 1u)) ? (fr << 5) | lane : INT_MAX;
+    int best = key;
+    for (int o = 16; o; o >>= 1) best = min(best, __shfl_xor_sync(kFull, best, o));
+    const int e = best & 31;
+    if (lane == 0) {
+      s.ev[s.nev++] = s.cols[e];
+      s.cols[e] = kPad;
+      s.m[e] = make_uint4(0, 0, 0, 0);
+    }
+    realset &= ~(1u << e);
+    __syncwarp();
+  }
+}
+
+struct Scratch {
+  int32_t* tcols;  // [npan][cap][16]
+  uint8_t* tperm;  // [npan][cap][16]
+  int32_t* tev;    // [npan][cap][16]
+  uint8_t* tnev;   // [npan][cap]
+  int cap;
+};
+
+__device__ void store_tile(const TileSmem& s, const Scratch& sc, int p, int t, int lane) {
+  const int64_t o = ((int64_t)p * sc.cap + t) * 16;
+  if (lane < 16) {
+    sc.tcols[o + lane] = s.cols[lane];
+    sc.tperm[o + lane] = s.perm[lane];
+    sc.tev[o + lane] = lane < s.nev ? s.ev[lane] : kPad;
+  }
+  if (lane == 0) sc.tnev[(int64_t)p * sc.cap + t] = (uint8_t)s.nev;
+}
+
+// ------------------------------------------------------------------ R3
+constexpr int kR3Warps = 4;
+__global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const uint4* __restrict__ masks,
+                                                              const int32_t* __restrict__ S,
+                                                              const int32_t* __restrict__ Kp,
+                                                              int64_t K, Scratch sc) {
+  __shared__ TileSmem sm[kR3Warps];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int p = blockIdx.y;
+  const int t = blockIdx.x * kR3Warps + warp;
+  if (t >= Kp[p] / 16) return;  // only full tiles of S_p (warp-uniform)
+  TileSmem& s = sm[warp];
+  if (lane < 16) {
+    const int32_t c = S[(int64_t)p * K + 16 * t + lane];
+    s.cols[lane] = c;
+    s.m[lane] = masks[(int64_t)p * K + c];
+  }
+  __syncwarp();
+  tile_search(s, lane);
+  store_tile(s, sc, p, t, lane);
+}
+
+// ------------------------------------------------------------------ R4
+__global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks,
+                                                 const int32_t* __restrict__ S,
+                                                 const int32_t* __restrict__ Kp, int64_t K,
+                                                 Scratch sc, int32_t* __restrict__ queue,
+                                                 int64_t qcap, int32_t* __restrict__ T,
+                                                 int* __restrict__ err) {
+  __shared__ TileSmem s;
+  const int p = blockIdx.x, lane = threadIdx.x;
+  const int kp = Kp[p], nfull = kp / 16, rem = kp - 16 * nfull;
+  int32_t* q = queue + (int64_t)p * qcap;
+  // FIFO contents after the full tiles: the rest of S_p, then the columns the full
+  // tiles evicted, in tile order and eviction order (exactly CR1's sequential queue).
+  for (int i = lane; i < rem; i += 32) q[i] = S[(int64_t)p * K + 16 * nfull + i];
+  int64_t tail = rem;
+  for (int t = 0; t < nfull; ++t) {
+    const int n = sc.tnev[(int64_t)p * sc.cap + t];
+    if (lane < n) q[tail + lane] = sc.tev[((int64_t)p * sc.cap + t) * 16 + lane];
+    tail += n;
+  }
+  __syncwarp();
+  int64_t head = 0;
+  int t = nfull;
+  while (head < tail) {
+    if (t >= sc.cap || tail + 16 > qcap) {
+      if (lane == 0) atomicExch(err, 1);
+      break;
+    }
+    if (lane < 16) {
+      const int32_t c = head + lane < tail ? q[head + lane] : kPad;
+      s.cols[lane] = c;
+      s.m[lane] = c == kPad ? make_uint4(0, 0, 0, 0) : masks[(int64_t)p * K + c];
+    }
+    head = min(head + 16, tail);
+    __syncwarp();
+    tile_search(s, lane);
+    store_tile(s, sc, p, t, lane);
+    if (lane < s.nev) q[tail + lane] = s.ev[lane];
+    tail += s.nev;
+    ++t;
+    __syncwarp();
+  }
+  if (lane == 0) T[p] = t;
+}
+
+// ------------------------------------------------------------------ R5
+// One CTA (128 threads = rows) per (panel, k-step): compresses the two tiles of
+// the k-step (R-Q15, R-Q16) and writes
+//   A image : 4096 B = [row group 16][tile 2][row 8][8 halves]  (UMMA K-major,
+//             no swizzle: LBO = 128 B between the two tiles, SBO = 256 B)
+//   E lanes : TMEM metadata layout of tcgen05.mma.sp kind::f16 -- lane
+//             L = m0 + 8*h + 16*m2 holds rows r = 16*m2 + m0 and r + 8 of tile half h
+//   G rows  : B row per logical column, PAD -> K (TMA zero fill)
+__global__ void __launch_bounds__(128) k_emit(const uint16_t* __restrict__ A, int64_t M, int64_t K,
+                                              Scratch sc, const int32_t* __restrict__ T,
+                                              const int32_t* __restrict__ tile_off,
+                                              const int32_t* __restrict__ ksoff,
+                                              const int32_t* __restrict__ kboff,
+                                              uint8_t* __restrict__ Aimg, uint32_t* __restrict__ Eimg,
+                                              int32_t* __restrict__ G, int32_t* __restrict__ colidx,
+                                              uint8_t* __restrict__ perm, uint8_t* __restrict__ kind,
+                                              uint8_t* __restrict__ nevict, const int32_t* __restrict__ Kp) {
+  __shared__ int32_t gat[2][16];
+  __shared__ uint16_t smeta[2][128];
+  const int p = blockIdx.y, ks = blockIdx.x, tid = threadIdx.x;
+  const int Tp = T[p];
+  const int nks = (Tp + 1) / 2;
+  if (ks >= nks) return;
+  const int64_t gks = ksoff[p] + ks;
+  if (tid < 32) {
+    const int h = tid >> 4, j = tid & 15, t = 2 * ks + h;
+    int32_t g = kPad;
+    if (t < Tp) {
+      const int64_t o = ((int64_t)p * sc.cap + t) * 16;
+      g = sc.tcols[o + sc.tperm[o + j]];
+      const int64_t ft = (int64_t)tile_off[p] + t;
+      colidx[ft * 16 + j] = sc.tcols[o + j];
+      perm[ft * 16 + j] = sc.tperm[o + j];
+      if (j == 0) {
+        kind[ft] = t < (Kp[p] + 15) / 16 ? 0 : 1;
+        nevict[ft] = sc.tnev[(int64_t)p * sc.cap + t];
+      }
+    }
+    gat[h][j] = g;
+    G[gks * 32 + tid] = g == kPad ? (int32_t)K : g;
+  }
+  __syncthreads();
+  const int r = tid;
+  const int64_t row = (int64_t)p * 128 + r;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    uint16_t v[8];
+    uint16_t meta = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      uint16_t bits[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int32_t c = gat[h][4 * q + i];
+        bits[i] = (c == kPad || row >= M) ? (uint16_t)0 : A[row * K + c];
+      }
+      int keep[2], nk = 0;
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+        if (nk < 2 && (bits[i] & 0x7FFFu)) keep[nk++] = i;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        if (nk >= 2) break;
+        if (bits[i] & 0x7FFFu) continue;
+        if (nk == 1 && keep[0] == i) continue;
+        keep[nk++] = i;
+      }
+      if (keep[0] > keep[1]) { const int x = keep[0]; keep[0] = keep[1]; keep[1] = x; }
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        const uint16_t b = bits[keep[k]];
+        v[2 * q + k] = (b & 0x7FFFu) ? b : (uint16_t)0;
+      }
+      meta |= (uint16_t)((keep[0] + 4 * keep[1]) << (4 * q));
+    }
+    uint4 pk;
+    pk.x = v[0] | ((uint32_t)v[1] << 16);
+    pk.y = v[2] | ((uint32_t)v[3] << 16);
+    pk.z = v[4] | ((uint32_t)v[5] << 16);
+    pk.w = v[6] | ((uint32_t)v[7] << 16);
+    *reinterpret_cast<uint4*>(Aimg + gks * kKStepBytesA + (r >> 3) * 256 + h * 128 + (r & 7) * 16) = pk;
+    smeta[h][r] = meta;
+  }
+  __syncthreads();
+  {
+    const int L = tid, m0 = L & 7, h = (L >> 3) & 1, m2 = L >> 4;
+    const int rr = 16 * m2 + m0;
+    const uint32_t w = (uint32_t)smeta[h][rr] | ((uint32_t)smeta[h][rr + 8] << 16);
+    Eimg[((int64_t)(kboff[p] + ks / kStepsPerBlock) * 128 + L) * 4 + (ks % kStepsPerBlock)] = w;
+  }
+}
+
+template <class T>
+jigsaw_status_t dalloc(T** p, size_t bytes, std::vector<void*>& list) {
+  *p = nullptr;
+  if (bytes == 0) bytes = 16;
+  cudaError_t e = cudaMalloc((void**)p, bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, std::string("cudaMalloc failed: ") + cudaGetErrorString(e));
+  }
+  list.push_back(*p);
+  return JIGSAW_SUCCESS;
+}
+
+}  // namespace
+
+void free_format(Format* f) {
+  for (void* p : f->allocs) cudaFree(p);
+  f->allocs.clear();
+}
+
+#define JIG_TRY(x)                          \
+  do {                                      \
+    jigsaw_status_t _s = (x);               \
+    if (_s != JIGSAW_SUCCESS) goto fail;    \
+  } while (0)
+#define JIG_CU(x, what)                                   \
+  do {                                                    \
+    cudaError_t _e = (x);                                 \
+    if (_e != cudaSuccess) { cuda_status(_e, what); goto fail; } \
+  } while (0)
+
+jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
+                             cudaStream_t stream, Format* f) {
+  std::vector<void*> scratch;
+  int dev = 0;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  jigsaw_status_t st = JIGSAW_SUCCESS;
+  const int npan = (int)((M + P - 1) / P);
+  const int cap = (int)(K / 8 + 2);
+  const int64_t qcap = 2 * K + 64;
+  uint4* masks = nullptr;
+  int32_t *S = nullptr, *Kp = nullptr, *T = nullptr, *queue = nullptr, *tile_off = nullptr;
+  int* err = nullptr;
+  unsigned long long* nnz = nullptr;
+  Scratch sc{};
+  std::vector<int32_t> hKp(npan), hT(npan);
+  unsigned long long hnnz = 0;
+  int herr = 0;
+  int maxks = 0;
+
+  cudaGetDevice(&dev);
+  f->M = M; f->K = K; f->v = v; f->P = P; f->mode = mode; f->device = dev;
+  f->npanels = npan;
+  if ((st = init_tables(dev)) != JIGSAW_SUCCESS) return st;
+
+  JIG_TRY(dalloc(&masks, sizeof(uint4) * npan * K, scratch));
+  JIG_TRY(dalloc(&S, sizeof(int32_t) * npan * K, scratch));
+  JIG_TRY(dalloc(&Kp, sizeof(int32_t) * npan, scratch));
+  JIG_TRY(dalloc(&T, sizeof(int32_t) * npan, scratch));
+  JIG_TRY(dalloc(&err, sizeof(int), scratch));
+  JIG_TRY(dalloc(&nnz, sizeof(unsigned long long), scratch));
+  JIG_TRY(dalloc(&queue, sizeof(int32_t) * npan * qcap, scratch));
+  JIG_TRY(dalloc(&sc.tcols, sizeof(int32_t) * npan * cap * 16, scratch));
+  JIG_TRY(dalloc(&sc.tperm, (size_t)npan * cap * 16, scratch));
+  JIG_TRY(dalloc(&sc.tev, sizeof(int32_t) * npan * cap * 16, scratch));
+  JIG_TRY(dalloc(&sc.tnev, (size_t)npan * cap, scratch));
+  sc.cap = cap;
+
+  JIG_CU(cudaEventCreate(&ev0), "cudaEventCreate");
+  JIG_CU(cudaEventCreate(&ev1), "cudaEventCreate");
+  JIG_CU(cudaEventRecord(ev0, stream), "cudaEventRecord");
+  JIG_CU(cudaMemsetAsync(err, 0, sizeof(int), stream), "memset");
+  JIG_CU(cudaMemsetAsync(nnz, 0, sizeof(unsigned long long), stream), "memset");
+  k_colmask<<<dim3((unsigned)((K + 127) / 128), npan), 128, 0, stream>>>(dA, M, K, P, masks, nnz);
+  k_compact<<<npan, 1024, 0, stream>>>(masks, K, S, Kp);
+  k_main_tiles<<<dim3((unsigned)((K / 16 + kR3Warps - 1) / kR3Warps), npan), 32 * kR3Warps, 0, stream>>>(
+      masks, S, Kp, K, sc);
+  k_overflow<<<npan, 32, 0, stream>>>(masks, S, Kp, K, sc, queue, qcap, T, err);
+  JIG_CU(cudaGetLastError(), "reorder kernels launch");
+  JIG_CU(cudaMemcpyAsync(hKp.data(), Kp, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy Kp");
+  JIG_CU(cudaMemcpyAsync(hT.data(), T, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy T");
+  JIG_CU(cudaMemcpyAsync(&hnnz, nnz, sizeof hnnz, cudaMemcpyDeviceToHost, stream), "copy nnz");
+  JIG_CU(cudaMemcpyAsync(&herr, err, sizeof herr, cudaMemcpyDeviceToHost, stream), "copy err");
+  JIG_CU(cudaStreamSynchronize(stream), "reorder R1-R4");
+  if (herr) {
+    st = set_status(JIGSAW_ERROR_INTERNAL, "reorder: tile or queue capacity exceeded");
+    goto fail;
+  }
+  // offsets (host): tiles, k-steps (ceil(T_p/2)), E blocks (ceil(ksteps/4))
+  f->T = hT;
+  f->D.assign(npan, 0);
+  f->tile_off.assign(npan + 1, 0);
+  f->ks_off.assign(npan + 1, 0);
+  f->kb_off.assign(npan + 1, 0);
+  f->kp_total = 0;
+  f->max_tiles = 0;
+  f->overflow_tiles = 0;
+  for (int p = 0; p < npan; ++p) {
+    const int nks = (hT[p] + 1) / 2;
+    f->tile_off[p + 1] = f->tile_off[p] + hT[p];
+    f->ks_off[p + 1] = f->ks_off[p] + nks;
+    f->kb_off[p + 1] = f->kb_off[p] + (nks + kStepsPerBlock - 1) / kStepsPerBlock;
+    f->kp_total += hKp[p];
+    f->max_tiles = std::max<int64_t>(f->max_tiles, hT[p]);
+    f->overflow_tiles += hT[p] - (hKp[p] + 15) / 16;
+    maxks = std::max(maxks, nks);
+  }
+  f->ntiles = f->tile_off[npan];
+  f->nksteps = f->ks_off[npan];
+  f->nkblocks = f->kb_off[npan];
+  f->nnz = (int64_t)hnnz;
+  f->evictions = f->ntiles * 16 - f->kp_total - 0;  // placeholder, replaced below
+  {
+    std::vector<int32_t> ksn(npan);
+    for (int p = 0; p < npan; ++p) ksn[p] = (hT[p] + 1) / 2;
+    JIG_TRY(dalloc(&f->d_ksn, sizeof(int32_t) * npan, f->allocs));
+    JIG_TRY(dalloc(&f->d_ksoff, sizeof(int32_t) * (npan + 1), f->allocs));
+    JIG_TRY(dalloc(&f->d_kboff, sizeof(int32_t) * (npan + 1), f->allocs));
+    JIG_TRY(dalloc(&tile_off, sizeof(int32_t) * (npan + 1), scratch));
+    JIG_TRY(dalloc(&f->d_colidx, sizeof(int32_t) * 16 * f->ntiles, f->allocs));
+    JIG_TRY(dalloc(&f->d_perm, (size_t)16 * f->ntiles, f->allocs));
+    JIG_TRY(dalloc(&f->d_kind, (size_t)f->ntiles, f->allocs));
+    JIG_TRY(dalloc(&f->d_nevict, (size_t)f->ntiles, f->allocs));
+    JIG_TRY(dalloc(&f->d_Aimg, (size_t)kKStepBytesA * f->nksteps, f->allocs));
+    JIG_TRY(dalloc(&f->d_Eimg, (size_t)kEBlockBytes * f->nkblocks, f->allocs));
+    JIG_TRY(dalloc(&f->d_G, sizeof(int32_t) * 32 * f->nksteps, f->allocs));
+    JIG_CU(cudaMemcpyAsync(f->d_ksn, ksn.data(), sizeof(int32_t) * npan, cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemcpyAsync(f->d_ksoff, f->ks_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemcpyAsync(f->d_kboff, f->kb_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemcpyAsync(tile_off, f->tile_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemsetAsync(f->d_Eimg, 0, (size_t)kEBlockBytes * f->nkblocks, stream), "memset E");
+    if (maxks > 0)
+      k_emit<<<dim3(maxks, npan), 128, 0, stream>>>(dA, M, K, sc, T, tile_off, f->d_ksoff, f->d_kboff,
+                                                  f->d_Aimg, reinterpret_cast<uint32_t*>(f->d_Eimg), f->d_G,
+                                                  f->d_colidx, f->d_perm, f->d_kind, f->d_nevict, Kp);
+    JIG_CU(cudaGetLastError(), "k_emit launch");
+    JIG_CU(cudaEventRecord(ev1, stream), "cudaEventRecord");
+    // total evictions = sum of per-tile counts
+    std::vector<uint8_t> hnev(f->ntiles);
+    if (f->ntiles)
+      JIG_CU(cudaMemcpyAsync(hnev.data(), f->d_nevict, f->ntiles, cudaMemcpyDeviceToHost, stream), "copy nevict");
+    JIG_CU(cudaStreamSynchronize(stream), "reorder R5");
+    f->evictions = 0;
+    for (uint8_t x : hnev) f->evictions += x;
+  }
+  {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, ev0, ev1);
+    f->reorder_ms = ms;
+  }
+  f->device_bytes = 0;
+  f->device_bytes += (int64_t)f->nksteps * (kKStepBytesA + 128) + (int64_t)f->nkblocks * kEBlockBytes +
+                     (int64_t)f->ntiles * (16 * 4 + 16 + 2) + (int64_t)npan * 12;
+  for (void* p : scratch) cudaFree(p);
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  return JIGSAW_SUCCESS;
+fail:
+  for (void* p : scratch) cudaFree(p);
+  if (ev0) cudaEventDestroy(ev0);
+  if (ev1) cudaEventDestroy(ev1);
+  free_format(f);
+  {
+    jigsaw_status_t s = jigsaw_last_status();
+    return s == JIGSAW_SUCCESS ? set_status(JIGSAW_ERROR_INTERNAL, "reorder failed") : s;
+  }
+}
+
+}  // namespace jig

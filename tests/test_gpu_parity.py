@@ -1,0 +1,206 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+  * reorder / format: BIT-EXACT against oracle O2 (CR1) -- T_p, col_idx, perm,
+    gather, vals, meta, kind, evictions -- and valid under checker O3;
+  * SpMM: |C - C_ref| <= 1e-2 * (|A|.|B|) + 1e-3 element-wise (north_star
+    tolerance), and bit-exact on integer-valued inputs.
+Small cases span several tiles and a ragged tail; full-size cases (BASELINE
+configs C2/C4) are checked on sampled panels and rows."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import check
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import paper_conf_icpp_zhanglyfyllq24_b200 as jig  # noqa: E402
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    torch.cuda.set_device(0)
+
+
+def _dev(x: np.ndarray):
+    return torch.from_numpy(np.ascontiguousarray(x).view(np.int16)).cuda().view(torch.float16)
+
+
+def _host(t) -> np.ndarray:
+    return t.view(torch.int16).cpu().numpy().view(np.uint16)
+
+
+def assert_format_equal(gpu: dict, ref: oracle.Format, panels=None):
+    if panels is None:
+        assert np.array_equal(gpu["T"], ref.T)
+        sl = slice(None)
+    else:
+        p0, p1 = panels
+        toff = np.concatenate([[0], np.cumsum(gpu["T"])])
+        assert np.array_equal(gpu["T"][p0:p1], ref.T)
+        sl = slice(int(toff[p0]), int(toff[p1]))
+    for k in ("col_idx", "perm", "vals", "meta", "kind", "nevict"):
+        a, b = gpu[k][sl], getattr(ref, k)
+        assert a.shape == b.shape, k
+        bad = np.argwhere(a != b)
+        assert bad.size == 0, f"{k} differs at {bad[:5].tolist()}"
+    assert np.array_equal(gpu["gather"][sl], ref.gather)
+
+
+def spmm_check(C_gpu: np.ndarray, A, B, rows=None):
+    C_ref, Mabs = oracle.spmm(A, B, rows=rows)
+    C = C_gpu.view(np.float16).astype(np.float64)
+    if rows is not None:
+        C = C[rows]
+    err = np.abs(C - C_ref)
+    tol = 1e-2 * Mabs + 1e-3
+    worst = np.unravel_index(np.argmax(err - tol), err.shape)
+    assert np.all(err <= tol), f"max excess at {worst}: err {err[worst]} tol {tol[worst]}"
+    return float((err / (Mabs + 1e-30)).max())
+
+
+CASES = [
+    # M, K, v, s, N, kind, seed
+    (256, 256, 4, 0.80, 64, "uniform", 1),     # C1
+    (384, 512, 8, 0.90, 256, "uniform", 2),
+    (200, 300, 4, 0.85, 136, "uniform", 3),    # ragged M, K % 16 != 0, N % 128 != 0
+    (512, 1024, 2, 0.70, 128, "skewed", 4),
+    (256, 512, 8, 0.50, 128, "uniform", 5),    # residual-heavy (many evictions)
+    (128, 64, 1, 0.0, 64, "uniform", 6),       # fully dense panel
+    (256, 2048, 8, 0.98, 256, "uniform", 7),
+]
+
+
+@pytest.mark.parametrize("M,K,v,s,N,kind,seed", CASES)
+def test_reorder_bit_exact_and_spmm(M, K, v, s, N, kind, seed):
+    A = synth.vector_sparse(M, K, v, s, seed, kind=kind)
+    B = synth.dense_b(K, N, seed)
+    h = jig.reorder(_dev(A), v)
+    g = h.export()
+    ref = oracle.reorder(A, P=128)
+    assert_format_equal(g, ref)
+    check.check_format(A, 128, g["T"], g["gather"], g["vals"], g["meta"], perm=g["perm"])
+    info = h.info()
+    assert info["ntiles"] == int(ref.T.sum())
+    assert info["evictions"] == int(ref.nevict.sum())
+    assert info["nnz"] == int(((A & 0x7FFF) != 0).sum())
+    assert info["format_bytes"] == check.format_bytes(ref.T, 128)
+    C = h.spmm(_dev(B))
+    torch.cuda.synchronize()
+    spmm_check(_host(C), A, B)
+    h.free()
+
+
+@pytest.mark.parametrize("seed", [11, 12])
+def test_spmm_integer_inputs_bit_exact(seed):
+    """Integer-valued A in {+-1,+-2}, B in {-2..2}, |C| <= 2048: every fp32 partial
+    sum is exact, so the GPU result must equal the oracle bit for bit."""
+    M, K, N = 384, 640, 192
+    A = synth.vector_sparse(M, K, 4, 0.9, seed, kind="int")
+    B = synth.dense_b(K, N, seed, kind="int")
+    h = jig.reorder(_dev(A), 4)
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    C_ref, _ = oracle.spmm(A, B)
+    assert np.abs(C_ref).max() <= 2048
+    assert np.array_equal(C.view(np.float16).astype(np.float64), C_ref)
+
+
+def test_all_zero_panel_and_empty_matrix():
+    A = np.zeros((384, 96), np.uint16)
+    A[130:138, 5] = np.float16(1.0).view(np.uint16)   # only panel 1 has nonzeros
+    B = synth.dense_b(96, 64, 1)
+    h = jig.reorder(_dev(A), 8)
+    g = h.export()
+    assert g["T"].tolist() == [0, 1, 0]
+    Cd = torch.full((384, 64), 7.0, dtype=torch.float16, device="cuda")
+    h.spmm(_dev(B), C=Cd)
+    C = _host(Cd)
+    spmm_check(C, A, B)
+    assert np.all(C[:128] == 0) and np.all(C[256:] == 0)
+    Z = np.zeros((128, 64), np.uint16)
+    hz = jig.reorder(_dev(Z), 1)
+    assert hz.info()["ntiles"] == 0
+    Cz = hz.spmm(_dev(synth.dense_b(64, 32, 2)))
+    assert int(torch.count_nonzero(Cz)) == 0
+
+
+def test_already_24_and_v_independence():
+    A = synth.nm24(256, 256, 3)
+    h = jig.reorder(_dev(A), 1)
+    g = h.export()
+    assert int(g["nevict"].sum()) == 0
+    assert all(g["perm"][t].tolist() == list(range(16)) for t in range(len(g["perm"])))
+    A8 = synth.vector_sparse(256, 256, 8, 0.9, 9)
+    g1, g8 = jig.reorder(_dev(A8), 1).export(), jig.reorder(_dev(A8), 8).export()
+    for k in g1:
+        assert np.array_equal(g1[k], g8[k]), k     # R-Q22: the format ignores v
+
+
+def test_negative_zero_and_host_paths():
+    A = synth.vector_sparse(256, 128, 4, 0.8, 5)
+    A[3, :] = np.where(A[3, :] == 0, np.uint16(0x8000), A[3, :])   # -0 entries are zeros
+    B = synth.dense_b(128, 64, 5)
+    h = jig.reorder_host(A, 4)
+    assert_format_equal(h.export(), oracle.reorder(A, P=128))
+    C = h.spmm_host(B)
+    spmm_check(C, A, B)
+
+
+def test_spmm_batched_and_streams():
+    mats = [synth.vector_sparse(256, 384, 8, 0.9, 20 + i) for i in range(3)]
+    Bs = [synth.dense_b(384, 128, 30 + i) for i in range(3)]
+    hs = [jig.reorder(_dev(a), 8) for a in mats]
+    dB = [_dev(b) for b in Bs]
+    dC = [torch.empty((256, 128), dtype=torch.float16, device="cuda") for _ in range(3)]
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        jig.spmm_batched(hs, dB, dC, stream=s)
+    s.synchronize()
+    for a, b, c in zip(mats, Bs, dC):
+        spmm_check(_host(c), a, b)
+
+
+def test_abi_errors_on_gpu():
+    A = synth.vector_sparse(128, 64, 4, 0.8, 1)
+    h = jig.reorder(_dev(A), 4)
+    B = _dev(synth.dense_b(64, 64, 1))
+    with pytest.raises(jig.JigsawError) as e:
+        h.spmm(B[:, :60].contiguous())      # N % 8 != 0
+    assert e.value.status == 1
+    L = jig.lib()
+    Cd = torch.empty((128, 64), dtype=torch.float16, device="cuda")
+    import ctypes
+    st = L.jigsaw_spmm(h.ptr, ctypes.c_void_p(B.data_ptr() + 2), 64, ctypes.c_void_p(Cd.data_ptr()), None)
+    assert st == 1                            # misaligned B
+    with pytest.raises(jig.JigsawError):
+        jig.reorder(_dev(synth.vector_sparse(8, 8, 1, 0.5, 1)), 3)
+
+
+# ---------------------------------------------------------------- full sizes
+@pytest.mark.parametrize("M,K,v,s,N", [
+    (2048, 512, 8, 0.95, 256),      # C2
+    (512, 2048, 2, 0.80, 256),      # C2
+    (4096, 4096, 8, 0.90, 2048),    # C4
+    (11008, 4096, 8, 0.70, 2048),   # C4
+])
+def test_full_size_sampled(M, K, v, s, N):
+    """BASELINE sizes in the launch configuration bench.py times: format
+    bit-exact on two sampled panels, C checked on 24 sampled rows."""
+    A = synth.vector_sparse(M, K, v, s, 1)
+    B = synth.dense_b(K, N, 1)
+    h = jig.reorder(_dev(A), v)
+    g = h.export()
+    npan = (M + 127) // 128
+    for p in sorted({0, npan // 2, npan - 1}):
+        ref = oracle.reorder(A, P=128, panels=(p, p + 1))
+        assert_format_equal(g, ref, panels=(p, p + 1))
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(0)
+    rows = np.sort(rng.choice(M, size=24, replace=False))
+    spmm_check(C, A, B, rows=rows)
