@@ -1,22 +1,28 @@
 // spmm.cu -- S1: the SpMM mainloop C = A x B on sm_100a sparse tensor cores
-// (DESIGN.md §5.2).  PAPER.md P:120-128 (CTA per C tile, B gathered by the
+// (DESIGN.md §5.2).  PAPER.md P:120-128 (CTA per C tile, B gathered through the
 // reorder indices, C written straight from the accumulators)
-// (deepened pipeline: gather indices are read >= one stage ahead of the MMA),
-// re-designed for tcgen05:
+// (deepened pipeline: gather indices fetched ahead of the B copies), re-designed
+// for tcgen05:
 //
-//   persistent CTA per SM, 6 warps, warp-specialised:
-//     warp 0  producer : per k-block (4 k-steps = 128 logical columns)
-//                        cp.async.bulk of the compressed A image (16 KB) and the
-//                        metadata block (2 KB), and 2 x 32 TMA tile::gather4 of
-//                        the B rows named by the gather list (SW128, MN-major)
-//     warp 1  MMA      : tcgen05.cp metadata -> TMEM, then per k-step one
-//                        tcgen05.mma.sp.kind::f16  M=128 N=128 K=32 (logical)
-//                        into a double-buffered fp32 TMEM accumulator
-//     warps 2-5 epilogue: tcgen05.ld -> fp16 (RN) -> C rows < M
-//   work unit = (panel p of 128 rows, 128-column slice of C); units are
-//   scheduled round-robin, panels fastest, so co-resident CTAs share B in L2.
+//   320 threads, warp-specialised, mbarrier ring of kStages k-blocks
+//   (k-block = 4 k-steps = 128 logical columns = 8 tiles):
+//     warp 0      A/E producer : cp.async.bulk of the compressed A image (4 KB per
+//                               k-step) and of the TMEM metadata block (2 KB)
+//     warps 6-9   B producers  : warp w gathers the 32 B rows of k-step w with
+//                               16-byte cp.async straight into the SW128 MN-major
+//                               UMMA layout (PAD rows / columns >= N zero-filled)
+//     warp 1      MMA issuer   : tcgen05.cp metadata -> TMEM, then per k-step one
+//                               tcgen05.mma.sp.kind::f16 M=128 N=NT K=32 (logical)
+//                               into a double-buffered fp32 TMEM accumulator
+//     warps 2-5   epilogue     : tcgen05.ld -> fp16 (RN) -> C rows < M
+//   work unit = (panel of 128 rows, NT columns of C), panels fastest.
+//   Split-K (few units, e.g. the DLMC shapes of BASELINE configs[1]): a cluster
+//   of S CTAs shares one unit, each CTA runs 1/S of the panel's k-blocks, and
+//   the fp32 partial tiles are reduce-scattered through DSMEM with st.async
+//   (owner CTA r sums rows [r*128/S, (r+1)*128/S) and writes them to C).
 #include <cuda_fp16.h>
 
+#include <algorithm>
 #include <cstdio>
 
 #include "internal.h"
@@ -26,18 +32,27 @@ namespace jig {
 
 namespace {
 
-constexpr int kNTile = 128;                         // C columns per unit (UMMA N)
-constexpr int kStages = 4;
+constexpr unsigned kFullMask = 0xFFFFFFFFu;
+constexpr int kThreads = 320;
+constexpr int kBProdWarp0 = 6;
 constexpr int kRowsPerBlock = 32 * kStepsPerBlock;  // B rows per k-block (128)
 constexpr int kChunkB = kRowsPerBlock * 128;        // one 64-column SW128 chunk: 16 KB
-constexpr int kStageB = 2 * kChunkB;                // 32 KB
 constexpr int kStageA = kStepsPerBlock * kKStepBytesA;  // 16 KB
 constexpr int kStageE = kEBlockBytes;               // 2 KB
-constexpr int kThreads = 192;
-constexpr int kTmemCols = 512;
-constexpr int kAccCols = kNTile;                    // fp32 accumulator: 1 column per C column
-constexpr int kEColBase = 2 * kAccCols;             // metadata ring after the two accumulators
-constexpr size_t kSmemBytes = 1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + 256;
+
+template <int NT, bool kSplit>
+struct Cfg {
+  static constexpr int kChunks = NT / 64;
+  static constexpr int kStageB = kChunks * kChunkB;
+  static constexpr int kStages = NT == 128 ? 4 : 5;
+  static constexpr int kAccCols = NT;
+  static constexpr int kEColBase = 2 * NT;
+  static constexpr uint32_t kTmemCols = 2 * NT + 4 * kStages <= 256 ? 256 : 512;
+  static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
+  static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
+  static constexpr size_t kSmem = 1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + kRecvBytes + 256;
+  static_assert(kSmem <= 232448, "shared memory budget");
+};
 
 struct SpmmParams {
   const uint8_t* Aimg;
@@ -46,108 +61,153 @@ struct SpmmParams {
   const int32_t* ksn;
   const int32_t* ksoff;
   const int32_t* kboff;
+  const __half* B;
   __half* C;
-  int64_t M, N;
-  int npanels, nunits;
+  int64_t M, N, K;
+  int npanels, nunits, S;
 };
 
-__global__ void __launch_bounds__(kThreads, 1)
-    k_spmm(const __grid_constant__ CUtensorMap tmB, const SpmmParams prm) {
+__device__ __forceinline__ uint32_t pack_h2(float a, float b) {
+  __half2 h = __floats2half2_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+template <int NT, bool kSplit>
+__global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
+  using C_ = Cfg<NT, kSplit>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* sB = smem;                                // kStages x 32 KB (1024-aligned)
-  uint8_t* sA = sB + kStages * kStageB;              // kStages x 16 KB
-  uint8_t* sE = sA + kStages * kStageA;              // kStages x 2 KB
-  uint64_t* full = reinterpret_cast<uint64_t*>(sE + kStages * kStageE);
-  uint64_t* empty = full + kStages;
-  uint64_t* tfull = empty + kStages;
+  uint8_t* sB = smem;                                   // kStages x kStageB (1024-aligned)
+  uint8_t* sA = sB + C_::kStages * C_::kStageB;         // kStages x 16 KB
+  uint8_t* sE = sA + C_::kStages * kStageA;             // kStages x 2 KB
+  uint8_t* sRecv = sE + C_::kStages * kStageE;          // split-K receive buffer
+  uint64_t* full = reinterpret_cast<uint64_t*>(sRecv + C_::kRecvBytes);
+  uint64_t* empty = full + C_::kStages;
+  uint64_t* tfull = empty + C_::kStages;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* recv_full = tempty + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(recv_full + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int S = kSplit ? prm.S : 1;
+  const uint32_t rank = kSplit ? cluster_ctarank() : 0;
+  const int cluster_id = blockIdx.x / S, nclusters = gridDim.x / S;
+
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kStages; ++s) {
-      mbar_init(&full[s], 1);
+    for (int s = 0; s < C_::kStages; ++s) {
+      mbar_init(&full[s], 1 + 128);  // A/E expect_tx arrival + 128 B-producer cp.async arrivals
       mbar_init(&empty[s], 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);
       mbar_init(&tempty[a], 4);
     }
+    mbar_init(recv_full, 1);
     fence_barrier_init();
   }
-  if (warp == 0 && lane == 0) prefetch_tmap(&tmB);
-  if (warp == 1) tmem_alloc<kTmemCols>(tmem_slot);
-  __syncthreads();
+  if (warp == 1) tmem_alloc<C_::kTmemCols>(tmem_slot);
+  if constexpr (kSplit) {
+    cluster_sync_all();  // peers' barriers are initialised before any st.async targets them
+  } else {
+    __syncthreads();
+  }
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
 
   if (warp == 0) {
-    // ------------------------------------------------------------ producer
+    // ------------------------------------------------------------ A / E producer
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int u = cluster_id; u < prm.nunits; u += nclusters) {
+        const int p = u % prm.npanels;
+        const int nks = prm.ksn[p];
+        const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
+        const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
+        for (int kb = kb_lo; kb < kb_hi; ++kb) {
+          const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
+          const int64_t gks = prm.ksoff[p] + (int64_t)kb * kStepsPerBlock;
+          mbar_wait(&empty[stage], phase ^ 1);
+          mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + kStageE));
+          bulk_g2s(sA + stage * kStageA, prm.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
+          bulk_g2s(sE + stage * kStageE, prm.Eimg + (int64_t)(prm.kboff[p] + kb) * kEBlockBytes, kStageE,
+                   &full[stage]);
+          if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp >= kBProdWarp0) {
+    // ------------------------------------------------------------ B producers
+    const int w = warp - kBProdWarp0;      // k-step within the k-block
+    constexpr int LPR = NT / 8;            // lanes per B row (16-byte chunks per row)
+    constexpr int RPI = 32 / LPR;          // rows per iteration
+    const int c = lane % LPR;
     int stage = 0;
     uint32_t phase = 0;
-    for (int u = blockIdx.x; u < prm.nunits; u += gridDim.x) {
+    for (int u = cluster_id; u < prm.nunits; u += nclusters) {
       const int p = u % prm.npanels;
-      const int n0 = (u / prm.npanels) * kNTile;
+      const int n0 = (u / prm.npanels) * NT;
+      const int col = n0 + 8 * c;
+      const bool colok = col < prm.N;
       const int nks = prm.ksn[p];
-      const int ks0 = prm.ksoff[p];
-      const int kb0 = prm.kboff[p];
-      for (int kb = 0; kb * kStepsPerBlock < nks; ++kb) {
+      const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
+      const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
+      for (int kb = kb_lo; kb < kb_hi; ++kb) {
         const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
-        const int gks = ks0 + kb * kStepsPerBlock;
-        // gather rows for this k-block (issued before waiting: index load latency
-        // overlaps the wait, the P:222 "col_idx one stage ahead" idea)
-        int4 rows = make_int4(0, 0, 0, 0);
-        if (lane < steps * 8) rows = *reinterpret_cast<const int4*>(prm.G + (int64_t)gks * 32 + 4 * lane);
+        const int64_t gks = prm.ksoff[p] + (int64_t)kb * kStepsPerBlock;
+        // gather list of this k-step, read before waiting for the slot
+        const int32_t gidx = w < steps ? prm.G[(gks + w) * 32 + lane] : 0;
         mbar_wait(&empty[stage], phase ^ 1);
-        if (lane == 0) {
-          mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + kStageE + steps * 32 * 128 * 2));
-          bulk_g2s(sA + stage * kStageA, prm.Aimg + (int64_t)gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
-          bulk_g2s(sE + stage * kStageE, prm.Eimg + (int64_t)(kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
-        }
-        __syncwarp();
-        if (lane < steps * 8) {
-          uint8_t* dst = sB + stage * kStageB + lane * 512;
+        if (w < steps) {
+          uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
 #pragma unroll
-          for (int ch = 0; ch < 2; ++ch)
-            tma_gather4(dst + ch * kChunkB, &tmB, n0 + 64 * ch, rows.x, rows.y, rows.z, rows.w, &full[stage]);
+          for (int it = 0; it < 32 / RPI; ++it) {
+            const int j = it * RPI + lane / LPR;
+            const int32_t g = __shfl_sync(kFullMask, gidx, j);
+            const bool ok = colok && g < prm.K;
+            const __half* src = ok ? prm.B + (int64_t)g * prm.N + col : prm.B;
+            cp_async_16(sb + j * 128 + (((c & 7) ^ (j & 7)) << 4), src, ok ? 16u : 0u);
+          }
         }
-        if (++stage == kStages) { stage = 0; phase ^= 1; }
+        cp_async_mbar_arrive_noinc(&full[stage]);
+        if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
       }
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {
-      const uint32_t idesc0 = idesc_f16(128, kNTile, 0, 1, 1, 0);
-      const uint32_t idesc1 = idesc_f16(128, kNTile, 0, 1, 1, 1);
+      const uint32_t idesc0 = idesc_f16(128, NT, 0, 1, 1, 0);
+      const uint32_t idesc1 = idesc_f16(128, NT, 0, 1, 1, 1);
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
-      for (int u = blockIdx.x; u < prm.nunits; u += gridDim.x) {
+      for (int u = cluster_id; u < prm.nunits; u += nclusters) {
         const int p = u % prm.npanels;
         const int nks = prm.ksn[p];
-        if (nks == 0) continue;
+        const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
+        const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
+        if (kb_lo == kb_hi) continue;
         const int a = it & 1;
         const uint32_t use = (uint32_t)(it >> 1);
         mbar_wait(&tempty[a], (use & 1) ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tbase + a * kAccCols;
-        for (int kb = 0; kb * kStepsPerBlock < nks; ++kb) {
+        const uint32_t d_tmem = tbase + a * C_::kAccCols;
+        for (int kb = kb_lo; kb < kb_hi; ++kb) {
           const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
           mbar_wait(&full[stage], phase);
           tc_fence_after();
-          const uint32_t e_tmem = tbase + kEColBase + 4 * stage;
+          const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
           tc_cp_128x128b(e_tmem, smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0));
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
-          const uint32_t b_base = smem_u32(sB + stage * kStageB);
+          const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
           for (int s = 0; s < steps; ++s) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
             const uint64_t bdesc = smem_desc(b_base + s * 32 * 128, kChunkB, 1024, 2);
             tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0,
-                          (kb | s) != 0);
+                          (kb != kb_lo) || (s != 0));
           }
           tc_commit(&empty[stage]);
-          if (++stage == kStages) { stage = 0; phase ^= 1; }
+          if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
         tc_commit(&tfull[a]);
         ++it;
@@ -155,78 +215,145 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     __syncwarp();
   } else {
-    // ------------------------------------------------------------ epilogue
+    // ------------------------------------------------------------ epilogue (warps 2-5)
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     int it = 0;
-    for (int u = blockIdx.x; u < prm.nunits; u += gridDim.x) {
+    for (int u = cluster_id; u < prm.nunits; u += nclusters) {
       const int p = u % prm.npanels;
-      const int n0 = (u / prm.npanels) * kNTile;
+      const int n0 = (u / prm.npanels) * NT;
       const int nks = prm.ksn[p];
-      const int64_t row = (int64_t)p * 128 + q * 32 + lane;
-      __half* crow = prm.C + row * prm.N + n0;
-      if (nks == 0) {  // all-zero panel (R-Q21): C rows are zeros
-        if (row < prm.M)
-          for (int c = 0; c < kNTile && n0 + c < prm.N; c += 8)
-            *reinterpret_cast<uint4*>(crow + c) = make_uint4(0, 0, 0, 0);
-        continue;
-      }
+      const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
+      const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
+      const bool has_acc = kb_hi > kb_lo;
+      const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it & 1;
-      const uint32_t use = (uint32_t)(it >> 1);
-      mbar_wait(&tfull[a], use & 1);
-      tc_fence_after();
+      if (has_acc) {
+        mbar_wait(&tfull[a], (uint32_t)(it >> 1) & 1);
+        tc_fence_after();
+      }
+      if constexpr (!kSplit) {
+        const int64_t row = (int64_t)p * 128 + r;
+        __half* crow = prm.C + row * prm.N + n0;
 #pragma unroll 1
-      for (int c0 = 0; c0 < kNTile; c0 += 32) {
-        uint32_t r[32];
-        tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * kAccCols + c0, r);
-        tc_wait_ld();
-        if (row < prm.M) {
+        for (int c0 = 0; c0 < NT; c0 += 32) {
+          uint32_t v[32];
+          if (has_acc) {
+            tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * C_::kAccCols + c0, v);
+            tc_wait_ld();
+          } else {
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            if (n0 + c0 + 8 * j < prm.N) {
-              uint4 pk;
-              __half2 h0 = __floats2half2_rn(__uint_as_float(r[8 * j + 0]), __uint_as_float(r[8 * j + 1]));
-              __half2 h1 = __floats2half2_rn(__uint_as_float(r[8 * j + 2]), __uint_as_float(r[8 * j + 3]));
-              __half2 h2 = __floats2half2_rn(__uint_as_float(r[8 * j + 4]), __uint_as_float(r[8 * j + 5]));
-              __half2 h3 = __floats2half2_rn(__uint_as_float(r[8 * j + 6]), __uint_as_float(r[8 * j + 7]));
-              pk.x = *reinterpret_cast<uint32_t*>(&h0);
-              pk.y = *reinterpret_cast<uint32_t*>(&h1);
-              pk.z = *reinterpret_cast<uint32_t*>(&h2);
-              pk.w = *reinterpret_cast<uint32_t*>(&h3);
-              *reinterpret_cast<uint4*>(crow + c0 + 8 * j) = pk;
+            for (int j = 0; j < 32; ++j) v[j] = 0;     // all-zero panel (R-Q21)
+          }
+          if (row < prm.M) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              if (n0 + c0 + 8 * j < prm.N) {
+                uint4 pk;
+                pk.x = pack_h2(__uint_as_float(v[8 * j + 0]), __uint_as_float(v[8 * j + 1]));
+                pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
+                pk.z = pack_h2(__uint_as_float(v[8 * j + 4]), __uint_as_float(v[8 * j + 5]));
+                pk.w = pack_h2(__uint_as_float(v[8 * j + 6]), __uint_as_float(v[8 * j + 7]));
+                *reinterpret_cast<uint4*>(crow + c0 + 8 * j) = pk;
+              }
             }
           }
         }
+      } else {
+        // reduce-scatter of the fp32 partial tile through DSMEM
+        const int rpo = 128 / S;                           // rows owned per CTA
+        const uint32_t owner = (uint32_t)(r / rpo);
+        const int lr = r % rpo;
+        if (warp == 2 && lane == 0) mbar_arrive_expect_tx(recv_full, (uint32_t)(128 * NT * 4));
+        const uint32_t dst = mapa_shared(smem_u32(sRecv + (rank * rpo + lr) * C_::kRecvStride), owner);
+        const uint32_t dbar = mapa_shared(smem_u32(recv_full), owner);
+#pragma unroll 1
+        for (int c0 = 0; c0 < NT; c0 += 32) {
+          uint32_t v[32];
+          if (has_acc) {
+            tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * C_::kAccCols + c0, v);
+            tc_wait_ld();
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) v[j] = 0;
+          }
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            st_async_v4(dst + (c0 + 4 * j) * 4, v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3], dbar);
+        }
+        // owner: wait for all S partial slices of its rows, sum, convert, store
+        mbar_wait(recv_full, 0);
+        const int t = threadIdx.x - 64;                    // 0..127
+        constexpr int C8 = NT / 8;                         // 8-column groups per row
+        for (int item = t; item < rpo * C8; item += 128) {
+          const int i = item / C8, c8 = item % C8;
+          float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+          for (int s = 0; s < S; ++s) {
+            const float4* src = reinterpret_cast<const float4*>(sRecv + (s * rpo + i) * C_::kRecvStride + c8 * 32);
+            const float4 x = src[0], y = src[1];
+            acc[0] += x.x; acc[1] += x.y; acc[2] += x.z; acc[3] += x.w;
+            acc[4] += y.x; acc[5] += y.y; acc[6] += y.z; acc[7] += y.w;
+          }
+          const int64_t row = (int64_t)p * 128 + rank * rpo + i;
+          const int64_t colg = n0 + c8 * 8;
+          if (row < prm.M && colg < prm.N) {
+            uint4 pk;
+            pk.x = pack_h2(acc[0], acc[1]);
+            pk.y = pack_h2(acc[2], acc[3]);
+            pk.z = pack_h2(acc[4], acc[5]);
+            pk.w = pack_h2(acc[6], acc[7]);
+            *reinterpret_cast<uint4*>(prm.C + row * prm.N + colg) = pk;
+          }
+        }
       }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[a]);
-      ++it;
+      if (has_acc) {
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[a]);
+        ++it;
+      }
     }
   }
   tc_fence_before();
-  __syncthreads();
-  if (warp == 1) tmem_dealloc<kTmemCols>(tbase);
-}
-
-typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
-                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*,
-                                  CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion,
-                                  CUtensorMapFloatOOBfill);
-
-EncodeTiledFn encode_fn() {
-  static EncodeTiledFn fn = nullptr;
-  if (!fn) {
-    cudaDriverEntryPointQueryResult q;
-    void* p = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<EncodeTiledFn>(p);
+  if constexpr (kSplit) {
+    cluster_sync_all();  // no CTA leaves while peers may still target its shared memory
+  } else {
+    __syncthreads();
   }
-  return fn;
+  if (warp == 1) tmem_dealloc<C_::kTmemCols>(tbase);
 }
 
 int g_num_sms[64] = {0};
-bool g_attr_set[64] = {false};
+bool g_attr_set[64][4] = {};
+
+template <int NT, bool kSplit>
+jigsaw_status_t launch_variant(const SpmmParams& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
+  using C_ = Cfg<NT, kSplit>;
+  auto kern = k_spmm<NT, kSplit>;
+  if (dev >= 0 && dev < 64 && !g_attr_set[dev][vid]) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::kSmem);
+    if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(k_spmm)");
+    if (kSplit) {
+      e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+      if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(cluster)");
+    }
+    g_attr_set[dev][vid] = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = C_::kSmem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = kSplit ? S : 1;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, prm);
+  if (e != cudaSuccess) return cuda_status(e, "k_spmm launch");
+  return JIGSAW_SUCCESS;
+}
 
 }  // namespace
 
@@ -238,18 +365,29 @@ int spmm_num_sms() {
   return g_num_sms[dev];
 }
 
+// Tile / split selection: enough units for every SM -> NT = 128,
+// persistent; otherwise NT = 64 and, when the panels carry enough k-blocks,
+// split-K over a cluster of S = 2/4/8 CTAs.
+void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* grid) {
+  const int64_t u128 = f.npanels * ((N + 127) / 128);
+  if (u128 >= sms) {
+    *NT = 128;
+    *S = 1;
+    *grid = (int)std::min<int64_t>(u128, sms);
+    return;
+  }
+  const int64_t u64 = f.npanels * ((N + 63) / 64);
+  int64_t kb_total = 0;
+  for (int64_t p = 0; p < f.npanels; ++p) kb_total += (f.T[p] + 7) / 8;
+  const double kb_avg = f.npanels ? (double)kb_total / f.npanels : 0.0;
+  int s = 1;
+  while (s < 8 && u64 * (2 * s) <= sms && kb_avg >= 2.0 * s) s *= 2;
+  *NT = 64;
+  *S = s;
+  *grid = s > 1 ? (int)(u64 * s) : (int)std::min<int64_t>(u64, sms);
+}
+
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
-  EncodeTiledFn enc = encode_fn();
-  if (!enc) return set_status(JIGSAW_ERROR_CUDA, "cuTensorMapEncodeTiled unavailable");
-  CUtensorMap tm;
-  cuuint64_t gdim[2] = {(cuuint64_t)N, (cuuint64_t)f.K};
-  cuuint64_t gstr[1] = {(cuuint64_t)N * 2};
-  cuuint32_t box[2] = {64, 1};
-  cuuint32_t estr[2] = {1, 1};
-  CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(dB), gdim, gstr, box, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return set_status(JIGSAW_ERROR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
   SpmmParams prm;
   prm.Aimg = f.d_Aimg;
   prm.Eimg = f.d_Eimg;
@@ -257,23 +395,29 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   prm.ksn = f.d_ksn;
   prm.ksoff = f.d_ksoff;
   prm.kboff = f.d_kboff;
+  prm.B = reinterpret_cast<const __half*>(dB);
   prm.C = reinterpret_cast<__half*>(dC);
   prm.M = f.M;
   prm.N = N;
+  prm.K = f.K;
   prm.npanels = (int)f.npanels;
-  const int64_t ntn = (N + kNTile - 1) / kNTile;
-  prm.nunits = (int)(f.npanels * ntn);
-  int dev = f.device;
-  if (dev >= 0 && dev < 64 && !g_attr_set[dev]) {
-    cudaError_t e = cudaFuncSetAttribute(k_spmm, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
-    if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(k_spmm)");
-    g_attr_set[dev] = true;
+  int NT = 128, S = 1, grid = 1;
+  choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
+  if (const char* e = getenv("JIGSAW_FORCE_SPLIT")) {  // test hook: force NT = 64 with split S
+    const int fs = atoi(e);
+    if (fs == 1 || fs == 2 || fs == 4 || fs == 8) {
+      NT = 64;
+      S = fs;
+      const int64_t u64 = f.npanels * ((N + 63) / 64);
+      grid = S > 1 ? (int)(u64 * S) : (int)std::min<int64_t>(u64, spmm_num_sms());
+    }
   }
-  const int grid = (int)std::min<int64_t>(prm.nunits, spmm_num_sms());
-  k_spmm<<<grid, kThreads, kSmemBytes, s>>>(tm, prm);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return cuda_status(e, "k_spmm launch");
-  return JIGSAW_SUCCESS;
+  prm.S = S;
+  prm.nunits = (int)(f.npanels * ((N + NT - 1) / NT));
+  const int dev = f.device;
+  if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, 0, s);
+  if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, 1, s);
+  return launch_variant<64, true>(prm, grid, S, dev, 2, s);
 }
 
 }  // namespace jig

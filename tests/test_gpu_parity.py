@@ -204,3 +204,26 @@ def test_full_size_sampled(M, K, v, s, N):
     rng = np.random.default_rng(0)
     rows = np.sort(rng.choice(M, size=24, replace=False))
     spmm_check(C, A, B, rows=rows)
+
+
+@pytest.mark.parametrize("force", ["1", "2", "4", "8"])
+@pytest.mark.parametrize("M,K,v,s,N", [(512, 2048, 4, 0.9, 256), (384, 700, 8, 0.8, 200),
+                                       (256, 96, 2, 0.95, 64)])
+def test_spmm_kernel_variants(force, M, K, v, s, N, monkeypatch):
+    """Every k_spmm variant (NT = 64 with split-K S = 1/2/4/8 over a cluster and the
+    DSMEM reduce-scatter) against the oracle, incl. splits that get no k-block."""
+    monkeypatch.setenv("JIGSAW_FORCE_SPLIT", force)
+    A = synth.vector_sparse(M, K, v, s, 3)
+    B = synth.dense_b(K, N, 3)
+    h = jig.reorder(_dev(A), v)
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    spmm_check(C, A, B)
+    Ai = synth.vector_sparse(M, K, v, s, 4, kind="int")
+    Bi = synth.dense_b(K, N, 4, kind="int")
+    hi = jig.reorder(_dev(Ai), v)
+    Ci = _host(hi.spmm(_dev(Bi)))
+    torch.cuda.synchronize()
+    C_ref, _ = oracle.spmm(Ai, Bi)
+    if np.abs(C_ref).max() <= 2048:
+        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
