@@ -131,6 +131,8 @@ class Handle:
 
     def __init__(self, ptr: int):
         self._h = ctypes.c_void_p(ptr)
+        inf = self.info()
+        self.M, self.K = inf["M"], inf["K"]
 
     @property
     def ptr(self):
@@ -145,25 +147,28 @@ class Handle:
         """C = A x B (jigsaw_spmm); B: CUDA fp16 K x N; returns C (M x N fp16)."""
         import torch
         _check_fp16_cuda(B, "B")
-        inf = self.info()
         K, N = B.shape
-        if K != inf["K"]:
-            raise ValueError(f"B has {K} rows, A has K = {inf['K']}")
+        if K != self.K:
+            raise ValueError(f"B has {K} rows, A has K = {self.K}")
         if C is None:
-            C = torch.empty((inf["M"], N), dtype=torch.float16, device=B.device)
+            C = torch.empty((self.M, N), dtype=torch.float16, device=B.device)
         else:
             _check_fp16_cuda(C, "C")
+            if tuple(C.shape) != (self.M, N):
+                raise ValueError("C must be M x N")
         _raise_if(lib().jigsaw_spmm(self._h, ctypes.c_void_p(B.data_ptr()), N,
                                     ctypes.c_void_p(C.data_ptr()), _stream_ptr(stream)))
         return C
 
-    def spmm_host(self, B: np.ndarray, stream=None) -> np.ndarray:
-        """End-to-end path (jigsaw_spmm_host): host B in, host C out."""
+    def spmm_host(self, B: np.ndarray, out: np.ndarray = None, stream=None) -> np.ndarray:
+        """End-to-end path (jigsaw_spmm_host): host B in, host C out (optionally
+        into `out`, e.g. pinned memory)."""
         B = np.ascontiguousarray(B)
         if B.dtype == np.float16:
             B = B.view(np.uint16)
-        inf = self.info()
-        C = np.empty((inf["M"], B.shape[1]), dtype=np.uint16)
+        C = np.empty((self.M, B.shape[1]), dtype=np.uint16) if out is None else out
+        if C.shape != (self.M, B.shape[1]) or not C.flags.c_contiguous or C.itemsize != 2:
+            raise ValueError("out must be a contiguous M x N 16-bit array")
         _raise_if(lib().jigsaw_spmm_host(self._h, B.ctypes.data_as(ctypes.c_void_p), B.shape[1],
                                          C.ctypes.data_as(ctypes.c_void_p),
                                          _stream_ptr(stream) if stream is not None else None))

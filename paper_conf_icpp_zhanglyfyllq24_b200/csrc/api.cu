@@ -54,6 +54,26 @@ jigsaw_status_t check_device(int* dev_out) {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
+// Stream-ordered staging memory for the host-buffer entry points: a private pool
+// per device that keeps its memory (no release to the OS between calls).
+cudaMemPool_t g_pool[64] = {};
+cudaError_t staging_alloc(void** p, size_t bytes, cudaStream_t st) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) return cudaMallocAsync(p, bytes, st);
+  if (!g_pool[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaError_t e = cudaMemPoolCreate(&g_pool[dev], &props);
+    if (e != cudaSuccess) return e;
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(g_pool[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  return cudaMallocFromPoolAsync(p, bytes, g_pool[dev], st);
+}
+
 jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, const jigsaw_options_t* opt) {
   if (!A) return set_status(JIGSAW_ERROR_INVALID_VALUE, "A is NULL");
   if (M <= 0 || K <= 0) return set_status(JIGSAW_ERROR_INVALID_VALUE, "M and K must be positive");
@@ -138,7 +158,7 @@ jigsaw_status_t jigsaw_reorder_host(const void* A_host, int64_t M, int64_t K, in
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   void* dA = nullptr;
   const size_t bytes = (size_t)M * K * 2;
-  cudaError_t e = cudaMallocAsync(&dA, bytes, st);
+  cudaError_t e = staging_alloc(&dA, bytes, st);
   if (e != cudaSuccess) {
     cudaGetLastError();
     return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "cudaMallocAsync(A) failed");
@@ -169,8 +189,8 @@ jigsaw_status_t jigsaw_spmm_host(jigsaw_handle_t h, const void* B_host, int64_t 
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   const size_t bbytes = (size_t)h->f.K * N * 2, cbytes = (size_t)h->f.M * N * 2;
   void *dB = nullptr, *dC = nullptr;
-  cudaError_t e = cudaMallocAsync(&dB, bbytes, st);
-  if (e == cudaSuccess) e = cudaMallocAsync(&dC, cbytes, st);
+  cudaError_t e = staging_alloc(&dB, bbytes, st);
+  if (e == cudaSuccess) e = staging_alloc(&dC, cbytes, st);
   if (e != cudaSuccess) {
     cudaGetLastError();
     if (dB) cudaFreeAsync(dB, st);
@@ -198,17 +218,18 @@ jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const
     jigsaw_status_t s = validate_spmm(hs[i], Bs[i], Ns[i], Cs[i], true);
     if (s != JIGSAW_SUCCESS) return s;
   }
-  for (int i = 0; i < count; ++i) {
-    jigsaw_status_t s = launch_spmm(hs[i]->f, Bs[i], Ns[i], Cs[i], reinterpret_cast<cudaStream_t>(stream));
-    if (s != JIGSAW_SUCCESS) return s;
-  }
+  if (count == 0) return set_status(JIGSAW_SUCCESS);
+  std::vector<const Format*> fs(count);
+  for (int i = 0; i < count; ++i) fs[i] = &hs[i]->f;
+  jigsaw_status_t s = launch_spmm_grouped(fs.data(), Bs, Ns, Cs, count, reinterpret_cast<cudaStream_t>(stream));
+  if (s != JIGSAW_SUCCESS) return s;
   return set_status(JIGSAW_SUCCESS);
 }
 
 int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N) {
   (void)h;
   (void)N;
-  return 1;
+  return 1;  // jigsaw_spmm: one k_spmm launch; jigsaw_spmm_batched: one per 64 products
 }
 
 void jigsaw_free(jigsaw_handle_t h) {

@@ -57,6 +57,8 @@ void free_format(Format* f);
 
 // spmm.cu
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s);
+jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
+                                    void* const* Cs, int count, cudaStream_t s);
 int spmm_num_sms();
 
 }  // namespace jig

@@ -54,7 +54,8 @@ struct Cfg {
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
-struct SpmmParams {
+// One product of a (possibly grouped) launch.
+struct Problem {
   const uint8_t* Aimg;
   const uint8_t* Eimg;
   const int32_t* G;
@@ -64,8 +65,35 @@ struct SpmmParams {
   const __half* B;
   __half* C;
   int64_t M, N, K;
-  int npanels, nunits, S;
+  int npanels;
+  int unit0;  // first global work unit of this problem
 };
+constexpr int kMaxProblems = 64;
+struct SpmmParams {
+  Problem pr[kMaxProblems];
+  int nprob, nunits, S;
+};
+
+// Work unit u -> (problem, panel, first C column, k-block range of this CTA).
+struct Work {
+  const Problem* P;
+  int p, n0, nks, kb_lo, kb_hi;
+};
+template <int NT>
+__device__ __forceinline__ Work decode_unit(const SpmmParams& prm, int u, uint32_t rank, int S) {
+  int i = 0;
+  while (i + 1 < prm.nprob && prm.pr[i + 1].unit0 <= u) ++i;
+  Work w;
+  w.P = &prm.pr[i];
+  const int lu = u - w.P->unit0;
+  w.p = lu % w.P->npanels;
+  w.n0 = (lu / w.P->npanels) * NT;
+  w.nks = w.P->ksn[w.p];
+  const int nkb = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
+  w.kb_lo = (int)(rank * nkb / S);
+  w.kb_hi = (int)((rank + 1) * nkb / S);
+  return w;
+}
 
 __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   __half2 h = __floats2half2_rn(a, b);
@@ -120,58 +148,80 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
       int stage = 0;
       uint32_t phase = 0;
       for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-        const int p = u % prm.npanels;
-        const int nks = prm.ksn[p];
-        const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
-        const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
-        for (int kb = kb_lo; kb < kb_hi; ++kb) {
-          const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
-          const int64_t gks = prm.ksoff[p] + (int64_t)kb * kStepsPerBlock;
+        const Work wk = decode_unit<NT>(prm, u, rank, S);
+        const int64_t ks0 = wk.P->ksoff[wk.p], kb0 = wk.P->kboff[wk.p];
+        for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
+          const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
+          const int64_t gks = ks0 + (int64_t)kb * kStepsPerBlock;
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + kStageE));
-          bulk_g2s(sA + stage * kStageA, prm.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
-          bulk_g2s(sE + stage * kStageE, prm.Eimg + (int64_t)(prm.kboff[p] + kb) * kEBlockBytes, kStageE,
-                   &full[stage]);
+          bulk_g2s(sA + stage * kStageA, wk.P->Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
+          bulk_g2s(sE + stage * kStageE, wk.P->Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
     }
   } else if (warp >= kBProdWarp0) {
     // ------------------------------------------------------------ B producers
+    // The gather list of the NEXT k-block is loaded while the current one is
+    // issued, so the index load never sits in front of the B copies.
     const int w = warp - kBProdWarp0;      // k-step within the k-block
     constexpr int LPR = NT / 8;            // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
     int stage = 0;
     uint32_t phase = 0;
-    for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-      const int p = u % prm.npanels;
-      const int n0 = (u / prm.npanels) * NT;
-      const int col = n0 + 8 * c;
-      const bool colok = col < prm.N;
-      const int nks = prm.ksn[p];
-      const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
-      const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
-      for (int kb = kb_lo; kb < kb_hi; ++kb) {
-        const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
-        const int64_t gks = prm.ksoff[p] + (int64_t)kb * kStepsPerBlock;
-        // gather list of this k-step, read before waiting for the slot
-        const int32_t gidx = w < steps ? prm.G[(gks + w) * 32 + lane] : 0;
-        mbar_wait(&empty[stage], phase ^ 1);
-        if (w < steps) {
-          uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
-#pragma unroll
-          for (int it = 0; it < 32 / RPI; ++it) {
-            const int j = it * RPI + lane / LPR;
-            const int32_t g = __shfl_sync(kFullMask, gidx, j);
-            const bool ok = colok && g < prm.K;
-            const __half* src = ok ? prm.B + (int64_t)g * prm.N + col : prm.B;
-            cp_async_16(sb + j * 128 + (((c & 7) ^ (j & 7)) << 4), src, ok ? 16u : 0u);
-          }
-        }
-        cp_async_mbar_arrive_noinc(&full[stage]);
-        if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
+    // iterator over the (unit, k-block) pairs of this CTA, skipping empty units
+    auto next_nonempty = [&](int start, int& uo, Work& wo) -> bool {
+      for (int uu = start; uu < prm.nunits; uu += nclusters) {
+        wo = decode_unit<NT>(prm, uu, rank, S);
+        if (wo.kb_hi > wo.kb_lo) { uo = uu; return true; }
       }
+      return false;
+    };
+    auto gload = [&](const Work& ww, int kk) -> int32_t {
+      const int steps = min(kStepsPerBlock, ww.nks - kk * kStepsPerBlock);
+      const int64_t gks = ww.P->ksoff[ww.p] + (int64_t)kk * kStepsPerBlock;
+      return w < steps ? ww.P->G[(gks + w) * 32 + lane] : 0;
+    };
+    int u = 0;
+    Work wk{};
+    bool have = next_nonempty(cluster_id, u, wk);
+    int kb = have ? wk.kb_lo : 0;
+    int32_t gcur = have ? gload(wk, kb) : 0;
+    while (have) {
+      int un = u, kbn = kb + 1;
+      Work wn = wk;
+      bool hn = true;
+      if (kbn >= wk.kb_hi) {
+        hn = next_nonempty(u + nclusters, un, wn);
+        kbn = wn.kb_lo;
+      }
+      const int32_t gnext = hn ? gload(wn, kbn) : 0;   // prefetch the next gather list
+      const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
+      const int col = wk.n0 + 8 * c;
+      const bool colok = col < wk.P->N;
+      mbar_wait(&empty[stage], phase ^ 1);
+      if (w < steps) {
+        uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
+        const __half* Bp = wk.P->B;
+        const int64_t ldb = wk.P->N, K = wk.P->K;
+#pragma unroll
+        for (int it = 0; it < 32 / RPI; ++it) {
+          const int j = it * RPI + lane / LPR;
+          const int32_t g = __shfl_sync(kFullMask, gcur, j);
+          const bool ok = colok && g < K;
+          const __half* src = ok ? Bp + (int64_t)g * ldb + col : Bp;
+          cp_async_16(sb + j * 128 + (((c & 7) ^ (j & 7)) << 4), src, ok ? 16u : 0u);
+        }
+      }
+      cp_async_mbar_arrive_noinc(&full[stage]);
+      if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
+      u = un;
+      wk = wn;
+      kb = kbn;
+      have = hn;
+      gcur = gnext;
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
@@ -182,10 +232,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
       uint32_t phase = 0;
       int it = 0;
       for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-        const int p = u % prm.npanels;
-        const int nks = prm.ksn[p];
-        const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
-        const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
+        const Work wk = decode_unit<NT>(prm, u, rank, S);
+        const int nks = wk.nks, kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
         const int a = it & 1;
         const uint32_t use = (uint32_t)(it >> 1);
@@ -219,12 +267,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     int it = 0;
     for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-      const int p = u % prm.npanels;
-      const int n0 = (u / prm.npanels) * NT;
-      const int nks = prm.ksn[p];
-      const int nkb = (nks + kStepsPerBlock - 1) / kStepsPerBlock;
-      const int kb_lo = (int)(rank * nkb / S), kb_hi = (int)((rank + 1) * nkb / S);
-      const bool has_acc = kb_hi > kb_lo;
+      const Work wk = decode_unit<NT>(prm, u, rank, S);
+      const int p = wk.p, n0 = wk.n0;
+      const int64_t M = wk.P->M, N = wk.P->N;
+      __half* const Cm = wk.P->C;
+      const bool has_acc = wk.kb_hi > wk.kb_lo;
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it & 1;
       if (has_acc) {
@@ -233,7 +280,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
       }
       if constexpr (!kSplit) {
         const int64_t row = (int64_t)p * 128 + r;
-        __half* crow = prm.C + row * prm.N + n0;
+        __half* crow = Cm + row * N + n0;
 #pragma unroll 1
         for (int c0 = 0; c0 < NT; c0 += 32) {
           uint32_t v[32];
@@ -244,10 +291,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
 #pragma unroll
             for (int j = 0; j < 32; ++j) v[j] = 0;     // all-zero panel (R-Q21)
           }
-          if (row < prm.M) {
+          if (row < M) {
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
-              if (n0 + c0 + 8 * j < prm.N) {
+              if (n0 + c0 + 8 * j < N) {
                 uint4 pk;
                 pk.x = pack_h2(__uint_as_float(v[8 * j + 0]), __uint_as_float(v[8 * j + 1]));
                 pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
@@ -295,13 +342,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
           }
           const int64_t row = (int64_t)p * 128 + rank * rpo + i;
           const int64_t colg = n0 + c8 * 8;
-          if (row < prm.M && colg < prm.N) {
+          if (row < M && colg < N) {
             uint4 pk;
             pk.x = pack_h2(acc[0], acc[1]);
             pk.y = pack_h2(acc[2], acc[3]);
             pk.z = pack_h2(acc[4], acc[5]);
             pk.w = pack_h2(acc[6], acc[7]);
-            *reinterpret_cast<uint4*>(prm.C + row * prm.N + colg) = pk;
+            *reinterpret_cast<uint4*>(Cm + row * N + colg) = pk;
           }
         }
       }
@@ -387,20 +434,38 @@ void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* gr
   *grid = s > 1 ? (int)(u64 * s) : (int)std::min<int64_t>(u64, sms);
 }
 
+static void fill_problem(Problem& P, const Format& f, const void* dB, int64_t N, void* dC) {
+  P.Aimg = f.d_Aimg;
+  P.Eimg = f.d_Eimg;
+  P.G = f.d_G;
+  P.ksn = f.d_ksn;
+  P.ksoff = f.d_ksoff;
+  P.kboff = f.d_kboff;
+  P.B = reinterpret_cast<const __half*>(dB);
+  P.C = reinterpret_cast<__half*>(dC);
+  P.M = f.M;
+  P.N = N;
+  P.K = f.K;
+  P.npanels = (int)f.npanels;
+}
+
+static jigsaw_status_t launch_params(SpmmParams& prm, int NT, int S, int grid, int dev, cudaStream_t s) {
+  prm.S = S;
+  int u = 0;
+  for (int i = 0; i < prm.nprob; ++i) {
+    prm.pr[i].unit0 = u;
+    u += (int)(prm.pr[i].npanels * ((prm.pr[i].N + NT - 1) / NT));
+  }
+  prm.nunits = u;
+  if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, 0, s);
+  if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, 1, s);
+  return launch_variant<64, true>(prm, grid, S, dev, 2, s);
+}
+
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
-  SpmmParams prm;
-  prm.Aimg = f.d_Aimg;
-  prm.Eimg = f.d_Eimg;
-  prm.G = f.d_G;
-  prm.ksn = f.d_ksn;
-  prm.ksoff = f.d_ksoff;
-  prm.kboff = f.d_kboff;
-  prm.B = reinterpret_cast<const __half*>(dB);
-  prm.C = reinterpret_cast<__half*>(dC);
-  prm.M = f.M;
-  prm.N = N;
-  prm.K = f.K;
-  prm.npanels = (int)f.npanels;
+  thread_local SpmmParams prm;  // large (param space); host-side scratch
+  prm.nprob = 1;
+  fill_problem(prm.pr[0], f, dB, N, dC);
   int NT = 128, S = 1, grid = 1;
   choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
   if (const char* e = getenv("JIGSAW_FORCE_SPLIT")) {  // test hook: force NT = 64 with split S
@@ -412,12 +477,30 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
       grid = S > 1 ? (int)(u64 * S) : (int)std::min<int64_t>(u64, spmm_num_sms());
     }
   }
-  prm.S = S;
-  prm.nunits = (int)(f.npanels * ((N + NT - 1) / NT));
-  const int dev = f.device;
-  if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, 0, s);
-  if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, 1, s);
-  return launch_variant<64, true>(prm, grid, S, dev, 2, s);
+  return launch_params(prm, NT, S, grid, f.device, s);
+}
+
+// Grouped launch: many independent products in ONE persistent kernel (units of
+// all problems are dealt round-robin to the CTAs), up to kMaxProblems per launch.
+jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
+                                    void* const* Cs, int count, cudaStream_t s) {
+  thread_local SpmmParams prm;
+  const int sms = spmm_num_sms();
+  for (int i0 = 0; i0 < count; i0 += kMaxProblems) {
+    const int n = std::min(kMaxProblems, count - i0);
+    prm.nprob = n;
+    int64_t u128 = 0, u64 = 0;
+    for (int i = 0; i < n; ++i) {
+      fill_problem(prm.pr[i], *fs[i0 + i], Bs[i0 + i], Ns[i0 + i], Cs[i0 + i]);
+      u128 += fs[i0 + i]->npanels * ((Ns[i0 + i] + 127) / 128);
+      u64 += fs[i0 + i]->npanels * ((Ns[i0 + i] + 63) / 64);
+    }
+    const int NT = u128 >= 2 * sms ? 128 : 64;
+    const int64_t units = NT == 128 ? u128 : u64;
+    jigsaw_status_t st = launch_params(prm, NT, 1, (int)std::min<int64_t>(units, sms), fs[i0]->device, s);
+    if (st != JIGSAW_SUCCESS) return st;
+  }
+  return JIGSAW_SUCCESS;
 }
 
 }  // namespace jig

@@ -227,3 +227,28 @@ def test_spmm_kernel_variants(force, M, K, v, s, N, monkeypatch):
     C_ref, _ = oracle.spmm(Ai, Bi)
     if np.abs(C_ref).max() <= 2048:
         assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+
+
+def test_grouped_launch_many_mixed_problems():
+    """jigsaw_spmm_batched: one grouped persistent launch per 64 products; 70 mixed
+    shapes / N / sparsities (incl. an all-zero matrix) against the oracle."""
+    rng = np.random.default_rng(5)
+    shapes = [(128, 64), (256, 96), (200, 160), (384, 128), (64, 256)]
+    mats, Bs, hs = [], [], []
+    for i in range(70):
+        M, K = shapes[i % len(shapes)]
+        v = [1, 2, 4, 8][i % 4]
+        M -= M % v
+        s = float(rng.choice([0.5, 0.8, 0.95]))
+        A = synth.vector_sparse(M, K, v, s, 100 + i) if i != 7 else np.zeros((M, K), np.uint16)
+        N = int(rng.choice([64, 136, 256]))
+        mats.append(A)
+        Bs.append(synth.dense_b(K, N, 200 + i))
+        hs.append(jig.reorder(_dev(A), v))
+    dB = [_dev(b) for b in Bs]
+    dC = [torch.full((a.shape[0], b.shape[1]), 3.0, dtype=torch.float16, device="cuda")
+          for a, b in zip(mats, Bs)]
+    jig.spmm_batched(hs, dB, dC)
+    torch.cuda.synchronize()
+    for a, b, c in zip(mats, Bs, dC):
+        spmm_check(_host(c), a, b)

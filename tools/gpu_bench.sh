@@ -10,7 +10,7 @@ timeout 600 python bench.py --workload $WL --detail > $OUT/${TAG}_bench.json 2> 
 tail -3 $OUT/${TAG}_bench.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
    --log-file $OUT/${TAG}_launches.csv python bench.py --workload $WL --steps 2 --warmup 3 --no-cpu --no-cublas > /dev/null 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm -s 108 -c 36 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm -s 72 -c 36 \
    -o $OUT/${TAG}_spmm_full python bench.py --workload $WL --steps 1 --warmup 3 --no-cpu --no-cublas > $OUT/${TAG}_ncu_full.log 2>&1
 tail -5 $OUT/${TAG}_ncu_full.log
 ls -la $OUT
