@@ -166,6 +166,21 @@ JIGSAW_API jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const 
  * accounting in benchmarks); reorder kernels are not counted. */
 JIGSAW_API int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N);
 
+/* ---------------------------------------------------------------- diagnostics */
+
+/* Per-CTA timeline of the most recent k_spmm launch made with the environment
+ * variable JIGSAW_TRACE=1 (otherwise nothing is recorded).  Copies up to
+ * max_ctas records of 16 int64 each into `out` (host): slots 0-11 are SM clock
+ * (clock64) stamps at fixed points of the kernel (entry, setup done, first A/E
+ * copy, first B copies, first full stage, last MMA commit, accumulator ready,
+ * sends done, reduction data ready, stores done, exit), 13 / 15 are
+ * %globaltimer (ns) at exit / entry, 14 is the SM id.  max_ctas < 0 instead
+ * copies the per-k-block timeline of CTAs 0..7 (8 x 4 x 32 int64: A/E copy
+ * issued, B copies issued, stage full seen by the MMA thread, MMAs committed).
+ * Synchronous.  Returns the number of records copied (0 if none, -1 on a CUDA
+ * error). */
+JIGSAW_API int jigsaw_debug_trace(int64_t* out, int max_ctas);
+
 #ifdef __cplusplus
 }
 #endif

@@ -28,7 +28,8 @@ STATUS = {0: "SUCCESS", 1: "INVALID_VALUE", 2: "UNSUPPORTED", 3: "OUT_OF_MEMORY"
 ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_status",
                "jigsaw_last_error_string", "jigsaw_version", "jigsaw_reorder_ex",
                "jigsaw_reorder_host", "jigsaw_get_info", "jigsaw_export_format",
-               "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_launches_per_call"]
+               "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_launches_per_call",
+               "jigsaw_debug_trace"]
 
 
 class JigsawError(RuntimeError):
@@ -91,6 +92,7 @@ def lib(build_if_missing: bool = True):
         "jigsaw_spmm_batched": (ci, [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(i64),
                                      ctypes.POINTER(vp), ci, vp]),
         "jigsaw_spmm_launches_per_call": (ci, [vp, i64]),
+        "jigsaw_debug_trace": (ci, [vp, ci]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -222,6 +224,15 @@ def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: in
     _raise_if(lib().jigsaw_reorder_host(A.ctypes.data_as(ctypes.c_void_p), M, K, v,
                                         ctypes.byref(opt), None, ctypes.byref(out)))
     return Handle(out.value)
+
+
+def debug_trace(max_ctas: int = 1024) -> np.ndarray:
+    """Timeline of the last k_spmm launch made with JIGSAW_TRACE=1: [ctas, 16] int64."""
+    out = np.zeros((max_ctas, 16), np.int64)
+    n = lib().jigsaw_debug_trace(out.ctypes.data_as(ctypes.c_void_p), max_ctas)
+    if n < 0:
+        raise JigsawError(4, "jigsaw_debug_trace failed")
+    return out[:n]
 
 
 def spmm_batched(handles, Bs, Cs, stream=None):

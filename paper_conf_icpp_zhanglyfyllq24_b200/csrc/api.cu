@@ -232,6 +232,11 @@ int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N) {
   return 1;  // jigsaw_spmm: one k_spmm launch; jigsaw_spmm_batched: one per 64 products
 }
 
+int jigsaw_debug_trace(int64_t* out, int max_ctas) {
+  if (!out || max_ctas == 0) return 0;
+  return debug_trace_read(reinterpret_cast<long long*>(out), max_ctas);
+}
+
 void jigsaw_free(jigsaw_handle_t h) {
   if (!h) return;
   int cur = 0;

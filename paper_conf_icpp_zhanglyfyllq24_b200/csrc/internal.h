@@ -27,9 +27,8 @@ struct Format {
   // host copies of per-panel counts / offsets
   std::vector<int32_t> T, D, tile_off, ks_off, kb_off;
   // device per-panel arrays
-  int32_t* d_ksn = nullptr;    // [npanels]   k-steps of the panel = ceil(T_p / 2)
-  int32_t* d_ksoff = nullptr;  // [npanels]   first k-step of the panel
-  int32_t* d_kboff = nullptr;  // [npanels]   first E block of the panel
+  int4* d_pin = nullptr;       // [npanels] {k-steps = ceil(T_p/2), first k-step, first E block, 0}
+  std::vector<int4> pin;       // host copy of d_pin
   // canonical arrays (device)
   int32_t* d_colidx = nullptr;  // [ntiles][16]
   uint8_t* d_perm = nullptr;    // [ntiles][16]
@@ -60,5 +59,6 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
 jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
                                     void* const* Cs, int count, cudaStream_t s);
 int spmm_num_sms();
+int debug_trace_read(long long* host, int max_ctas);
 
 }  // namespace jig

@@ -111,8 +111,11 @@ __global__ void k_compact(const uint4* __restrict__ masks, int64_t K, int32_t* _
 }
 
 // ------------------------------------------------------------------ tile search
+constexpr int kMaxBig = 256;
 struct TileSmem {
   uint32_t bitmap[2048];  // compat[S] for every 4-subset S, indexed by the 16-bit slot mask
+  uint16_t big[kMaxBig];  // compatible 3- and 4-subsets of the real slots (existence test)
+  int nbig;
   uint4 m[16];            // row masks per slot (PAD: 0)
   int32_t cols[16];       // column per slot (kPad = -1)
   int32_t ev[16];         // evicted columns, in eviction order
@@ -164,6 +167,71 @@ __device__ bool complete_cover(const TileSmem& s, uint32_t used, uint32_t& o1, u
   return false;
 }
 
+// Exact existence test for a cover (used to skip exhaustive searches that must
+// fail; it never changes WHICH cover is chosen).  PAD slots are interchangeable
+// zero columns and any group with <= 2 real columns is compatible, so a cover
+// exists iff some k <= 4 disjoint compatible "big" groups (3 or 4 real columns)
+// hold enough real columns that the rest fits 2 per remaining group:
+// sum(|b_i| - 2) >= nreal - 8.  Falls back to "maybe" (true) when the
+// candidate list or the search budget overflows.
+__device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
+  if (lane == 0) s.nbig = 0;
+  __syncwarp();
+  for (int k = lane; k < kNumSubsets; k += 32) {          // 4 real columns
+    const uint32_t sub = g_subs[k];
+    if ((sub & ~realset) == 0 && compat(s, sub)) {
+      const int i = atomicAdd(&s.nbig, 1);
+      if (i < kMaxBig) s.big[i] = (uint16_t)sub;
+    }
+  }
+  if (lane < 16 && ((realset >> lane) & 1u)) {              // 3 real columns, min slot = lane
+    const uint4 ma = s.m[lane];
+    for (uint32_t x = realset & ~((2u << lane) - 1u); x; x &= x - 1) {
+      const int b = __ffs(x) - 1;
+      const uint4 mb = s.m[b];
+      for (uint32_t y = x & (x - 1); y; y &= y - 1) {
+        const int c = __ffs(y) - 1;
+        const uint4 mc = s.m[c];
+        const uint32_t all3 = (ma.x & mb.x & mc.x) | (ma.y & mb.y & mc.y) | (ma.z & mb.z & mc.z) |
+                              (ma.w & mb.w & mc.w);
+        if (!all3) {
+          const int i = atomicAdd(&s.nbig, 1);
+          if (i < kMaxBig) s.big[i] = (uint16_t)((1u << lane) | (1u << b) | (1u << c));
+        }
+      }
+    }
+  }
+  __syncwarp();
+  int found = 0;
+  if (lane == 0) {
+    const int n = s.nbig, need = __popc(realset) - 8;
+    if (n > kMaxBig) {
+      found = 1;
+    } else {
+      // depth-first over disjoint blocks (<= 4 deep), best excess first
+      int idx[4] = {0, 0, 0, 0};
+      uint32_t used[5] = {0, 0, 0, 0, 0};
+      int exc[5] = {0, 0, 0, 0, 0};
+      int d = 0, budget = 1 << 16;
+      while (d >= 0 && !found) {
+        if (--budget < 0) { found = 1; break; }
+        if (idx[d] >= n || d == 4) {          // level exhausted: backtrack
+          --d;
+          if (d >= 0) ++idx[d];
+          continue;
+        }
+        const uint32_t b = s.big[idx[d]];
+        if (b & used[d]) { ++idx[d]; continue; }
+        used[d + 1] = used[d] | b;
+        exc[d + 1] = exc[d] + __popc(b) - 2;
+        if (exc[d + 1] >= need) { found = 1; break; }
+        if (d + 1 < 4) { idx[d + 1] = idx[d] + 1; ++d; } else { ++idx[d]; }
+      }
+    }
+  }
+  return __shfl_sync(kFull, found, 0) != 0;
+}
+
 // Alg. 1 + reorder retry on one tile, executed by one full warp.  On entry
 // s.cols / s.m hold the 16 popped columns; on exit s.cols has evicted slots set
 // to PAD, s.perm the new column order g0||g1||g2||g3, s.ev[0..s.nev) the evictions.
@@ -210,7 +278,8 @@ __device__ void tile_search(TileSmem& s, int lane) {
     __syncwarp();
     // Necessary conditions for a cover (they only skip searches that must fail):
     // every slot lies in some compatible group; 4 groups can hold all real columns.
-    const bool coverable = __all_sync(kFull, lane >= 16 || fr > 0) && hmax * 4 >= __popc(realset);
+    bool coverable = __all_sync(kFull, lane >= 16 || fr > 0) && hmax * 4 >= __popc(realset);
+    if (coverable && __popc(realset) > 8) coverable = cover_exists(s, realset, lane);
     // Alg. 1 lines 9-17: lanes try the candidates for g0 (groups containing slot 0)
     // in lexicographic order, 32 at a time; the lowest successful one wins.
     if (coverable) {
@@ -474,6 +543,7 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   const int64_t qcap = 2 * K + 64;
   uint4* masks = nullptr;
   int32_t *S = nullptr, *Kp = nullptr, *T = nullptr, *queue = nullptr, *tile_off = nullptr;
+  int32_t *d_ksoff = nullptr, *d_kboff = nullptr;
   int* err = nullptr;
   unsigned long long* nnz = nullptr;
   Scratch sc{};
@@ -545,11 +615,11 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   f->nnz = (int64_t)hnnz;
   f->evictions = f->ntiles * 16 - f->kp_total - 0;  // placeholder, replaced below
   {
-    std::vector<int32_t> ksn(npan);
-    for (int p = 0; p < npan; ++p) ksn[p] = (hT[p] + 1) / 2;
-    JIG_TRY(dalloc(&f->d_ksn, sizeof(int32_t) * npan, f->allocs));
-    JIG_TRY(dalloc(&f->d_ksoff, sizeof(int32_t) * (npan + 1), f->allocs));
-    JIG_TRY(dalloc(&f->d_kboff, sizeof(int32_t) * (npan + 1), f->allocs));
+    f->pin.resize(npan);
+    for (int p = 0; p < npan; ++p) f->pin[p] = make_int4((hT[p] + 1) / 2, f->ks_off[p], f->kb_off[p], 0);
+    JIG_TRY(dalloc(&f->d_pin, sizeof(int4) * npan, f->allocs));
+    JIG_TRY(dalloc(&d_ksoff, sizeof(int32_t) * (npan + 1), scratch));
+    JIG_TRY(dalloc(&d_kboff, sizeof(int32_t) * (npan + 1), scratch));
     JIG_TRY(dalloc(&tile_off, sizeof(int32_t) * (npan + 1), scratch));
     JIG_TRY(dalloc(&f->d_colidx, sizeof(int32_t) * 16 * f->ntiles, f->allocs));
     JIG_TRY(dalloc(&f->d_perm, (size_t)16 * f->ntiles, f->allocs));
@@ -558,13 +628,13 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
     JIG_TRY(dalloc(&f->d_Aimg, (size_t)kKStepBytesA * f->nksteps, f->allocs));
     JIG_TRY(dalloc(&f->d_Eimg, (size_t)kEBlockBytes * f->nkblocks, f->allocs));
     JIG_TRY(dalloc(&f->d_G, sizeof(int32_t) * 32 * f->nksteps, f->allocs));
-    JIG_CU(cudaMemcpyAsync(f->d_ksn, ksn.data(), sizeof(int32_t) * npan, cudaMemcpyHostToDevice, stream), "upload");
-    JIG_CU(cudaMemcpyAsync(f->d_ksoff, f->ks_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
-    JIG_CU(cudaMemcpyAsync(f->d_kboff, f->kb_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemcpyAsync(f->d_pin, f->pin.data(), sizeof(int4) * npan, cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemcpyAsync(d_ksoff, f->ks_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
+    JIG_CU(cudaMemcpyAsync(d_kboff, f->kb_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(tile_off, f->tile_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemsetAsync(f->d_Eimg, 0, (size_t)kEBlockBytes * f->nkblocks, stream), "memset E");
     if (maxks > 0)
-      k_emit<<<dim3(maxks, npan), 128, 0, stream>>>(dA, M, K, sc, T, tile_off, f->d_ksoff, f->d_kboff,
+      k_emit<<<dim3(maxks, npan), 128, 0, stream>>>(dA, M, K, sc, T, tile_off, d_ksoff, d_kboff,
                                                   f->d_Aimg, reinterpret_cast<uint32_t*>(f->d_Eimg), f->d_G,
                                                   f->d_colidx, f->d_perm, f->d_kind, f->d_nevict, Kp);
     JIG_CU(cudaGetLastError(), "k_emit launch");

@@ -39,6 +39,7 @@ constexpr int kRowsPerBlock = 32 * kStepsPerBlock;  // B rows per k-block (128)
 constexpr int kChunkB = kRowsPerBlock * 128;        // one 64-column SW128 chunk: 16 KB
 constexpr int kStageA = kStepsPerBlock * kKStepBytesA;  // 16 KB
 constexpr int kStageE = kEBlockBytes;               // 2 KB
+constexpr int kStageG = kRowsPerBlock * 4;          // gather list of a k-block: 512 B
 
 template <int NT, bool kSplit>
 struct Cfg {
@@ -50,7 +51,8 @@ struct Cfg {
   static constexpr uint32_t kTmemCols = 2 * NT + 4 * kStages <= 256 ? 256 : 512;
   static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
   static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
-  static constexpr size_t kSmem = 1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + kRecvBytes + 256;
+  static constexpr size_t kSmem =
+      1024 + (size_t)kStages * (kStageB + kStageA + kStageE + kStageG) + kRecvBytes + 320;
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
@@ -59,40 +61,97 @@ struct Problem {
   const uint8_t* Aimg;
   const uint8_t* Eimg;
   const int32_t* G;
-  const int32_t* ksn;
-  const int32_t* ksoff;
-  const int32_t* kboff;
+  const int4* pin;  // per panel {k-steps, first k-step, first E block, 0} (device)
   const __half* B;
   __half* C;
   int64_t M, N, K;
   int npanels;
   int unit0;  // first global work unit of this problem
+  int pin0;   // offset of this problem's panels in SpmmParams::pin (if use_pin)
 };
 constexpr int kMaxProblems = 64;
+constexpr int kMaxPin = 1536;  // panel table kept in kernel parameter space when it fits
 struct SpmmParams {
   Problem pr[kMaxProblems];
-  int nprob, nunits, S;
+  int4 pin[kMaxPin];
+  int nprob, nunits, S, use_pin;
+  int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
 };
 
+// Opt-in per-CTA timeline (clock64 / %globaltimer), read by jigsaw_debug_trace.
+constexpr int kTraceCTAs = 1024, kTraceSlots = 16;
+__device__ long long g_trace[kTraceCTAs * kTraceSlots];
+constexpr int kTraceKB = 32;
+__device__ long long g_trace_kb[8 * 4 * kTraceKB];  // [cta<8][AE issue, B issue, full seen, mma done][kb]
+#define JIG_TRACE_KB(role, n)                                                        \
+  do {                                                                               \
+    if (prm.trace && blockIdx.x < 8 && (n) < kTraceKB)                               \
+      g_trace_kb[(blockIdx.x * 4 + (role)) * kTraceKB + (n)] = clock64();            \
+  } while (0)
+__device__ __forceinline__ long long gtimer() {
+  long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+#define JIG_TRACE(k)                                                                  \
+  do {                                                                                \
+    if (prm.trace && blockIdx.x < kTraceCTAs) g_trace[blockIdx.x * kTraceSlots + (k)] = clock64(); \
+  } while (0)
+
 // Work unit u -> (problem, panel, first C column, k-block range of this CTA).
+// Fields are copied out of the parameter space by value (LDC); a pointer into the
+// kernel parameters would turn every access into a slow generic load.
 struct Work {
-  const Problem* P;
+  const uint8_t* Aimg;
+  const uint8_t* Eimg;
+  const int32_t* G;
+  const __half* B;
+  __half* C;
+  int64_t M, N, K;
   int p, n0, nks, kb_lo, kb_hi;
+  int64_t ks0, kb0;  // first k-step / E block of the panel
 };
+// `hint` = problem index of this thread's previous unit: units are visited in
+// increasing order, so the scan is amortised O(1) instead of O(problems).
 template <int NT>
-__device__ __forceinline__ Work decode_unit(const SpmmParams& prm, int u, uint32_t rank, int S) {
-  int i = 0;
+__device__ __forceinline__ Work decode_unit(const SpmmParams& prm, int u, uint32_t rank, int S, int& hint) {
+  int i = hint;
+  if (prm.pr[i].unit0 > u) i = 0;
   while (i + 1 < prm.nprob && prm.pr[i + 1].unit0 <= u) ++i;
+  hint = i;
   Work w;
-  w.P = &prm.pr[i];
-  const int lu = u - w.P->unit0;
-  w.p = lu % w.P->npanels;
-  w.n0 = (lu / w.P->npanels) * NT;
-  w.nks = w.P->ksn[w.p];
+  w.Aimg = prm.pr[i].Aimg;
+  w.Eimg = prm.pr[i].Eimg;
+  w.G = prm.pr[i].G;
+  w.B = prm.pr[i].B;
+  w.C = prm.pr[i].C;
+  w.M = prm.pr[i].M;
+  w.N = prm.pr[i].N;
+  w.K = prm.pr[i].K;
+  const int np = prm.pr[i].npanels;
+  const int lu = u - prm.pr[i].unit0;
+  w.p = lu % np;
+  w.n0 = (lu / np) * NT;
+  // panel table from parameter space (no dependent global load at kernel start)
+  const int4 pi = prm.use_pin ? prm.pin[prm.pr[i].pin0 + w.p] : prm.pr[i].pin[w.p];
+  w.nks = pi.x;
+  w.ks0 = pi.y;
+  w.kb0 = pi.z;
   const int nkb = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
   w.kb_lo = (int)(rank * nkb / S);
   w.kb_hi = (int)((rank + 1) * nkb / S);
   return w;
+}
+
+__device__ __forceinline__ float4 ld_shared_f4(uint32_t saddr) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(saddr));
+  return v;
 }
 
 __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
@@ -108,10 +167,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
   uint8_t* sB = smem;                                   // kStages x kStageB (1024-aligned)
   uint8_t* sA = sB + C_::kStages * C_::kStageB;         // kStages x 16 KB
   uint8_t* sE = sA + C_::kStages * kStageA;             // kStages x 2 KB
-  uint8_t* sRecv = sE + C_::kStages * kStageE;          // split-K receive buffer
+  int32_t* sG = reinterpret_cast<int32_t*>(sE + C_::kStages * kStageE);  // kStages x 128 gather rows
+  uint8_t* sRecv = reinterpret_cast<uint8_t*>(sG) + C_::kStages * kStageG;  // split-K receive buffer
   uint64_t* full = reinterpret_cast<uint64_t*>(sRecv + C_::kRecvBytes);
   uint64_t* empty = full + C_::kStages;
-  uint64_t* tfull = empty + C_::kStages;
+  uint64_t* gfull = empty + C_::kStages;  // gather list of the stage has landed
+  uint64_t* tfull = gfull + C_::kStages;
   uint64_t* tempty = tfull + 2;
   uint64_t* recv_full = tempty + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(recv_full + 1);
@@ -120,11 +181,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
   const int S = kSplit ? prm.S : 1;
   const uint32_t rank = kSplit ? cluster_ctarank() : 0;
   const int cluster_id = blockIdx.x / S, nclusters = gridDim.x / S;
+  if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
+    g_trace[blockIdx.x * kTraceSlots + 15] = gtimer();
+    g_trace[blockIdx.x * kTraceSlots + 14] = smid();
+    JIG_TRACE(0);
+  }
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < C_::kStages; ++s) {
       mbar_init(&full[s], 1 + 128);  // A/E expect_tx arrival + 128 B-producer cp.async arrivals
       mbar_init(&empty[s], 1);
+      mbar_init(&gfull[s], 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);
@@ -141,98 +208,85 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
   }
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+  if (threadIdx.x == 0) JIG_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ A / E producer
     if (lane == 0) {
-      int stage = 0;
+      int stage = 0, hint = 0, nkb_issued = 0;
       uint32_t phase = 0;
       for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-        const Work wk = decode_unit<NT>(prm, u, rank, S);
-        const int64_t ks0 = wk.P->ksoff[wk.p], kb0 = wk.P->kboff[wk.p];
+        const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
+        const int64_t ks0 = wk.ks0, kb0 = wk.kb0;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
           const int64_t gks = ks0 + (int64_t)kb * kStepsPerBlock;
           mbar_wait(&empty[stage], phase ^ 1);
+          // gather list first, through the TMA path: the B producers wait only on
+          // it, never on an L1 load queued behind earlier cp.async traffic
+          mbar_arrive_expect_tx(&gfull[stage], (uint32_t)(steps * 128));
+          bulk_g2s(sG + stage * kRowsPerBlock, wk.G + gks * 32, steps * 128, &gfull[stage]);
           mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + kStageE));
-          bulk_g2s(sA + stage * kStageA, wk.P->Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
-          bulk_g2s(sE + stage * kStageE, wk.P->Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
+          bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
+          bulk_g2s(sE + stage * kStageE, wk.Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
+          if (u == cluster_id && kb == wk.kb_lo) JIG_TRACE(2);
+          JIG_TRACE_KB(0, nkb_issued);
+          ++nkb_issued;
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
     }
   } else if (warp >= kBProdWarp0) {
     // ------------------------------------------------------------ B producers
-    // The gather list of the NEXT k-block is loaded while the current one is
-    // issued, so the index load never sits in front of the B copies.
+    // Warp w copies the 32 B rows of k-step w of each k-block; the row indices
+    // come from the stage's gather list in shared memory (TMA-loaded by warp 0).
     const int w = warp - kBProdWarp0;      // k-step within the k-block
     constexpr int LPR = NT / 8;            // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
-    int stage = 0;
+    int stage = 0, hint = 0, traced = 0;
     uint32_t phase = 0;
-    // iterator over the (unit, k-block) pairs of this CTA, skipping empty units
-    auto next_nonempty = [&](int start, int& uo, Work& wo) -> bool {
-      for (int uu = start; uu < prm.nunits; uu += nclusters) {
-        wo = decode_unit<NT>(prm, uu, rank, S);
-        if (wo.kb_hi > wo.kb_lo) { uo = uu; return true; }
-      }
-      return false;
-    };
-    auto gload = [&](const Work& ww, int kk) -> int32_t {
-      const int steps = min(kStepsPerBlock, ww.nks - kk * kStepsPerBlock);
-      const int64_t gks = ww.P->ksoff[ww.p] + (int64_t)kk * kStepsPerBlock;
-      return w < steps ? ww.P->G[(gks + w) * 32 + lane] : 0;
-    };
-    int u = 0;
-    Work wk{};
-    bool have = next_nonempty(cluster_id, u, wk);
-    int kb = have ? wk.kb_lo : 0;
-    int32_t gcur = have ? gload(wk, kb) : 0;
-    while (have) {
-      int un = u, kbn = kb + 1;
-      Work wn = wk;
-      bool hn = true;
-      if (kbn >= wk.kb_hi) {
-        hn = next_nonempty(u + nclusters, un, wn);
-        kbn = wn.kb_lo;
-      }
-      const int32_t gnext = hn ? gload(wn, kbn) : 0;   // prefetch the next gather list
-      const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
+    for (int u = cluster_id; u < prm.nunits; u += nclusters) {
+      const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
       const int col = wk.n0 + 8 * c;
-      const bool colok = col < wk.P->N;
-      mbar_wait(&empty[stage], phase ^ 1);
-      if (w < steps) {
-        uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
-        const __half* Bp = wk.P->B;
-        const int64_t ldb = wk.P->N, K = wk.P->K;
+      const bool colok = col < wk.N;
+      const __half* Bp = wk.B;
+      const int64_t ldb = wk.N, K = wk.K;
+      for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
+        const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
+        mbar_wait(&empty[stage], phase ^ 1);
+        if (w < steps) {
+          mbar_wait(&gfull[stage], phase);
+          const int32_t gl = sG[stage * kRowsPerBlock + 32 * w + lane];
+          uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
 #pragma unroll
-        for (int it = 0; it < 32 / RPI; ++it) {
-          const int j = it * RPI + lane / LPR;
-          const int32_t g = __shfl_sync(kFullMask, gcur, j);
-          const bool ok = colok && g < K;
-          const __half* src = ok ? Bp + (int64_t)g * ldb + col : Bp;
-          cp_async_16(sb + j * 128 + (((c & 7) ^ (j & 7)) << 4), src, ok ? 16u : 0u);
+          for (int it = 0; it < 32 / RPI; ++it) {
+            const int j = it * RPI + lane / LPR;
+            const int32_t g = __shfl_sync(kFullMask, gl, j);
+            const bool ok = colok && g < K;
+            const __half* src = ok ? Bp + (int64_t)g * ldb + col : Bp;
+            cp_async_16(sb + j * 128 + (((c & 7) ^ (j & 7)) << 4), src, ok ? 16u : 0u);
+          }
         }
+        cp_async_mbar_arrive_noinc(&full[stage]);
+        if (lane == 0 && w == 0) {
+          if (traced == 0) JIG_TRACE(3);
+          JIG_TRACE_KB(1, traced);
+          ++traced;
+        }
+        if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
       }
-      cp_async_mbar_arrive_noinc(&full[stage]);
-      if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
-      u = un;
-      wk = wn;
-      kb = kbn;
-      have = hn;
-      gcur = gnext;
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {
       const uint32_t idesc0 = idesc_f16(128, NT, 0, 1, 1, 0);
       const uint32_t idesc1 = idesc_f16(128, NT, 0, 1, 1, 1);
-      int stage = 0;
+      int stage = 0, hint = 0, nkb_mma = 0;
       uint32_t phase = 0;
       int it = 0;
       for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-        const Work wk = decode_unit<NT>(prm, u, rank, S);
+        const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
         const int nks = wk.nks, kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
         const int a = it & 1;
@@ -244,6 +298,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
           const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
           mbar_wait(&full[stage], phase);
           tc_fence_after();
+          if (it == 0 && kb == kb_lo) JIG_TRACE(4);
+          JIG_TRACE_KB(2, nkb_mma);
           const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
           tc_cp_128x128b(e_tmem, smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0));
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
@@ -255,9 +311,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
                           (kb != kb_lo) || (s != 0));
           }
           tc_commit(&empty[stage]);
+          JIG_TRACE_KB(3, nkb_mma);
+          ++nkb_mma;
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
         tc_commit(&tfull[a]);
+        JIG_TRACE(5);
         ++it;
       }
     }
@@ -265,12 +324,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
   } else {
     // ------------------------------------------------------------ epilogue (warps 2-5)
     const int q = warp & 3;  // TMEM lane quarter this warp may access
-    int it = 0;
+    int it = 0, hint = 0;
     for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-      const Work wk = decode_unit<NT>(prm, u, rank, S);
+      const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
       const int p = wk.p, n0 = wk.n0;
-      const int64_t M = wk.P->M, N = wk.P->N;
-      __half* const Cm = wk.P->C;
+      const int64_t M = wk.M, N = wk.N;
+      __half* const Cm = wk.C;
       const bool has_acc = wk.kb_hi > wk.kb_lo;
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it & 1;
@@ -278,6 +337,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
         mbar_wait(&tfull[a], (uint32_t)(it >> 1) & 1);
         tc_fence_after();
       }
+      if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
       if constexpr (!kSplit) {
         const int64_t row = (int64_t)p * 128 + r;
         __half* crow = Cm + row * N + n0;
@@ -328,15 +388,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
             st_async_v4(dst + (c0 + 4 * j) * 4, v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3], dbar);
         }
         // owner: wait for all S partial slices of its rows, sum, convert, store
+        if (warp == 2 && lane == 0) JIG_TRACE(7);
         mbar_wait(recv_full, 0);
+        if (warp == 2 && lane == 0) JIG_TRACE(8);
         const int t = threadIdx.x - 64;                    // 0..127
         constexpr int C8 = NT / 8;                         // 8-column groups per row
         for (int item = t; item < rpo * C8; item += 128) {
           const int i = item / C8, c8 = item % C8;
           float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
           for (int s = 0; s < S; ++s) {
-            const float4* src = reinterpret_cast<const float4*>(sRecv + (s * rpo + i) * C_::kRecvStride + c8 * 32);
-            const float4 x = src[0], y = src[1];
+            const uint32_t src = smem_u32(sRecv + (s * rpo + i) * C_::kRecvStride + c8 * 32);
+            const float4 x = ld_shared_f4(src), y = ld_shared_f4(src + 16);
             acc[0] += x.x; acc[1] += x.y; acc[2] += x.z; acc[3] += x.w;
             acc[4] += y.x; acc[5] += y.y; acc[6] += y.z; acc[7] += y.w;
           }
@@ -352,6 +414,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
           }
         }
       }
+      if (warp == 2 && lane == 0) JIG_TRACE(9);
       if (has_acc) {
         tc_fence_before();
         __syncwarp();
@@ -360,6 +423,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
       }
     }
   }
+  if (threadIdx.x == 0) JIG_TRACE(10);
   tc_fence_before();
   if constexpr (kSplit) {
     cluster_sync_all();  // no CTA leaves while peers may still target its shared memory
@@ -367,6 +431,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
     __syncthreads();
   }
   if (warp == 1) tmem_dealloc<C_::kTmemCols>(tbase);
+  if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
+    JIG_TRACE(11);
+    g_trace[blockIdx.x * kTraceSlots + 13] = gtimer();
+  }
 }
 
 int g_num_sms[64] = {0};
@@ -428,19 +496,24 @@ void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* gr
   for (int64_t p = 0; p < f.npanels; ++p) kb_total += (f.T[p] + 7) / 8;
   const double kb_avg = f.npanels ? (double)kb_total / f.npanels : 0.0;
   int s = 1;
-  while (s < 8 && u64 * (2 * s) <= sms && kb_avg >= 2.0 * s) s *= 2;
+  // clusters of 8 do not all fit in one wave of 148 SMs (GPC granularity): S <= 4
+  while (s < 4 && u64 * (2 * s) <= sms && kb_avg >= 2.0 * s) s *= 2;
   *NT = 64;
   *S = s;
   *grid = s > 1 ? (int)(u64 * s) : (int)std::min<int64_t>(u64, sms);
 }
 
-static void fill_problem(Problem& P, const Format& f, const void* dB, int64_t N, void* dC) {
+static void fill_problem(SpmmParams& prm, int i, const Format& f, const void* dB, int64_t N, void* dC) {
+  Problem& P = prm.pr[i];
+  P.pin0 = i == 0 ? 0 : prm.pr[i - 1].pin0 + prm.pr[i - 1].npanels;
+  if (P.pin0 + f.npanels <= kMaxPin)
+    std::copy(f.pin.begin(), f.pin.end(), prm.pin + P.pin0);
+  else
+    prm.use_pin = 0;
   P.Aimg = f.d_Aimg;
   P.Eimg = f.d_Eimg;
   P.G = f.d_G;
-  P.ksn = f.d_ksn;
-  P.ksoff = f.d_ksoff;
-  P.kboff = f.d_kboff;
+  P.pin = f.d_pin;
   P.B = reinterpret_cast<const __half*>(dB);
   P.C = reinterpret_cast<__half*>(dC);
   P.M = f.M;
@@ -449,8 +522,13 @@ static void fill_problem(Problem& P, const Format& f, const void* dB, int64_t N,
   P.npanels = (int)f.npanels;
 }
 
+int g_trace_ctas = 0;
+
 static jigsaw_status_t launch_params(SpmmParams& prm, int NT, int S, int grid, int dev, cudaStream_t s) {
   prm.S = S;
+  const char* tr = getenv("JIGSAW_TRACE");
+  prm.trace = (tr && tr[0] == '1') ? 1 : 0;
+  if (prm.trace) g_trace_ctas = std::min(grid, kTraceCTAs);
   int u = 0;
   for (int i = 0; i < prm.nprob; ++i) {
     prm.pr[i].unit0 = u;
@@ -465,7 +543,8 @@ static jigsaw_status_t launch_params(SpmmParams& prm, int NT, int S, int grid, i
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
   thread_local SpmmParams prm;  // large (param space); host-side scratch
   prm.nprob = 1;
-  fill_problem(prm.pr[0], f, dB, N, dC);
+  prm.use_pin = 1;
+  fill_problem(prm, 0, f, dB, N, dC);
   int NT = 128, S = 1, grid = 1;
   choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
   if (const char* e = getenv("JIGSAW_FORCE_SPLIT")) {  // test hook: force NT = 64 with split S
@@ -489,9 +568,10 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
   for (int i0 = 0; i0 < count; i0 += kMaxProblems) {
     const int n = std::min(kMaxProblems, count - i0);
     prm.nprob = n;
+    prm.use_pin = 1;
     int64_t u128 = 0, u64 = 0;
     for (int i = 0; i < n; ++i) {
-      fill_problem(prm.pr[i], *fs[i0 + i], Bs[i0 + i], Ns[i0 + i], Cs[i0 + i]);
+      fill_problem(prm, i, *fs[i0 + i], Bs[i0 + i], Ns[i0 + i], Cs[i0 + i]);
       u128 += fs[i0 + i]->npanels * ((Ns[i0 + i] + 127) / 128);
       u64 += fs[i0 + i]->npanels * ((Ns[i0 + i] + 63) / 64);
     }
@@ -501,6 +581,20 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
     if (st != JIGSAW_SUCCESS) return st;
   }
   return JIGSAW_SUCCESS;
+}
+
+// Copies the timeline of the last traced launch (JIGSAW_TRACE=1): per CTA 16
+// int64 slots (clock64 at the trace points 0-11, 13 = %globaltimer at exit,
+// 14 = SM id, 15 = %globaltimer at entry).  Returns the CTA count.
+int debug_trace_read(long long* host, int max_ctas) {
+  if (max_ctas < 0) {  // per-k-block timeline of CTAs 0..7: 8*4*32 int64
+    if (cudaMemcpyFromSymbol(host, g_trace_kb, sizeof(long long) * 8 * 4 * kTraceKB) != cudaSuccess) return -1;
+    return 8;
+  }
+  const int n = std::min(max_ctas, g_trace_ctas);
+  if (n <= 0) return 0;
+  if (cudaMemcpyFromSymbol(host, g_trace, sizeof(long long) * kTraceSlots * n) != cudaSuccess) return -1;
+  return n;
 }
 
 }  // namespace jig

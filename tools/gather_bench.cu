@@ -1,0 +1,147 @@
+// tools/gather_bench.cu -- developer microbenchmark (not product): throughput of
+// gathering random 256-byte B-row segments into a 4-stage shared-memory ring,
+// all 148 SMs busy, B resident in L2.  Decides how k_spmm stages B.
+//   mode 0: cp.async 16 B (LDGSTS), 4 warps      mode 1: same, 8 warps
+//   mode 2: TMA tile::gather4 (box {64,1}, SW128), 1 issuing thread
+//   mode 3: TMA gather4 issued by 4 warps (one elected lane each)
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o gb tools/gather_bench.cu
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+
+#include "../paper_conf_icpp_zhanglyfyllq24_b200/csrc/ptx.cuh"
+
+using namespace jig;
+
+constexpr int kRows = 128, kStages = 4, kRowBytes = 256, kStageBytes = kRows * kRowBytes;
+constexpr int KB = 64;  // k-blocks per CTA
+
+__global__ void __launch_bounds__(320, 1) gather_kernel(const __grid_constant__ CUtensorMap tm, const uint16_t* B,
+                                                        int ldb, int K, const int* idx, int mode, long long* out) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t full[kStages], empty[kStages];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int nprod = (mode == 1) ? 8 : 4;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&full[s], mode <= 1 ? nprod * 32 : 1 + (mode == 3 ? 3 : 0));
+      mbar_init(&empty[s], 1);
+    }
+    fence_barrier_init();
+  }
+  __syncthreads();
+  const int* myidx = idx + (size_t)blockIdx.x * KB * kRows;
+  long long t0 = clock64();
+  if (warp == 0) {  // consumer
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t ph = 0;
+      for (int kb = 0; kb < KB; ++kb) {
+        mbar_wait(&full[stage], ph);
+        mbar_arrive(&empty[stage]);
+        if (++stage == kStages) { stage = 0; ph ^= 1; }
+      }
+      out[blockIdx.x] = clock64() - t0;
+    }
+  } else if (warp - 1 < nprod) {
+    const int w = warp - 1;
+    int stage = 0;
+    uint32_t ph = 0;
+    for (int kb = 0; kb < KB; ++kb) {
+      const int* ri = myidx + kb * kRows;
+      mbar_wait(&empty[stage], ph ^ 1);
+      uint8_t* st = sm + stage * kStageBytes;
+      if (mode <= 1) {
+        // rows per warp: 128 / nprod; 16 lanes per row (256 B), 2 rows per instruction
+        const int rpw = kRows / nprod;
+        const int c = lane & 15;
+        const int g0 = ri[w * rpw + (lane % rpw)];
+        for (int it = 0; it < rpw / 2; ++it) {
+          const int j = 2 * it + (lane >> 4);
+          const int g = __shfl_sync(0xffffffffu, g0, j % rpw);
+          const int row = w * rpw + j;
+          cp_async_16(st + (c >> 3) * (kRows * 128) + row * 128 + (((c & 7) ^ (row & 7)) << 4),
+                      B + (size_t)g * ldb + 8 * c, 16);
+        }
+        cp_async_mbar_arrive_noinc(&full[stage]);
+      } else if (mode == 2) {
+        if (w == 0 && lane == 0) {
+          mbar_arrive_expect_tx(&full[stage], kStageBytes);
+          for (int q = 0; q < kRows / 4; ++q)
+            for (int ch = 0; ch < 2; ++ch)
+              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, ri[4 * q], ri[4 * q + 1], ri[4 * q + 2],
+                          ri[4 * q + 3], &full[stage]);
+        }
+      } else {
+        if (lane == 0) {
+          if (w == 0) mbar_arrive_expect_tx(&full[stage], kStageBytes);
+          else mbar_arrive(&full[stage]);
+          for (int q = w * 8; q < w * 8 + 8; ++q)
+            for (int ch = 0; ch < 2; ++ch)
+              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, ri[4 * q], ri[4 * q + 1], ri[4 * q + 2],
+                          ri[4 * q + 3], &full[stage]);
+        }
+      }
+      if (++stage == kStages) { stage = 0; ph ^= 1; }
+    }
+  }
+  __syncthreads();
+}
+
+typedef CUresult (*EncodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+int main() {
+  const int K = 4096, N = 256, grid = 148;
+  uint16_t* dB;
+  int* didx;
+  long long* dout;
+  cudaMalloc(&dB, (size_t)K * N * 2);
+  cudaMemset(dB, 0, (size_t)K * N * 2);
+  std::vector<int> h((size_t)grid * KB * kRows);
+  srand(3);
+  for (auto& x : h) x = rand() % K;
+  cudaMalloc(&didx, h.size() * 4);
+  cudaMemcpy(didx, h.data(), h.size() * 4, cudaMemcpyHostToDevice);
+  cudaMalloc(&dout, grid * 8);
+  EncodeTiled enc;
+  cudaDriverEntryPointQueryResult q;
+  cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&enc, cudaEnableDefault, &q);
+  CUtensorMap tm;
+  cuuint64_t gdim[2] = {(cuuint64_t)N, (cuuint64_t)K};
+  cuuint64_t gstr[1] = {(cuuint64_t)N * 2};
+  cuuint32_t box[2] = {64, 1}, es[2] = {1, 1};
+  enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, dB, gdim, gstr, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+      CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  const int smem = kStages * kStageBytes + 1024;
+  cudaFuncSetAttribute(gather_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  const char* names[] = {"LDGSTS 4 warps", "LDGSTS 8 warps", "TMA gather4, 1 issuer", "TMA gather4, 4 issuers"};
+  for (int mode = 0; mode < 4; ++mode) {
+    for (int rep = 0; rep < 3; ++rep) {
+      cudaEvent_t a, b;
+      cudaEventCreate(&a);
+      cudaEventCreate(&b);
+      cudaEventRecord(a);
+      gather_kernel<<<grid, 320, smem>>>(tm, dB, N, K, didx, mode, dout);
+      cudaEventRecord(b);
+      cudaError_t e = cudaDeviceSynchronize();
+      if (e != cudaSuccess) { printf("mode %d error %s\n", mode, cudaGetErrorString(e)); return 1; }
+      float ms;
+      cudaEventElapsedTime(&ms, a, b);
+      std::vector<long long> cyc(grid);
+      cudaMemcpy(cyc.data(), dout, grid * 8, cudaMemcpyDeviceToHost);
+      long long mx = 0;
+      for (auto c : cyc) mx = c > mx ? c : mx;
+      const double bytes = (double)grid * KB * kStageBytes;
+      if (rep == 2)
+        printf("%-24s %8.1f us  %7.1f GB/s total  %5.1f B/clk/SM (max CTA %lld cyc, %.0f cyc per k-block)\n",
+               names[mode], ms * 1e3, bytes / ms / 1e6, (double)KB * kStageBytes / mx, mx, (double)mx / KB);
+    }
+  }
+  return 0;
+}
