@@ -85,9 +85,7 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
     if (opt->panel_rows != kPanelRows)
       return set_status(opt->panel_rows == 64 ? JIGSAW_ERROR_UNSUPPORTED : JIGSAW_ERROR_INVALID_VALUE,
                         "panel_rows must be 128 (64 is not built in this version)");
-    if (opt->residual_mode == JIGSAW_RESIDUAL_DENSE)
-      return set_status(JIGSAW_ERROR_UNSUPPORTED, "DENSE residual mode is not built in this version");
-    if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC)
+    if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC && opt->residual_mode != JIGSAW_RESIDUAL_DENSE)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
     for (int i = 0; i < 6; ++i)
       if (opt->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved options must be zero");
@@ -131,8 +129,9 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
   jigsaw_handle_s* h = new (std::nothrow) jigsaw_handle_s();
   if (!h) return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "host allocation failed");
   set_status(JIGSAW_SUCCESS);
-  s = build_format(static_cast<const uint16_t*>(A), M, K, v, kPanelRows, JIGSAW_RESIDUAL_SPTC,
-                   reinterpret_cast<cudaStream_t>(stream), &h->f);
+  s = build_format(static_cast<const uint16_t*>(A), M, K, v, kPanelRows,
+                   opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC, reinterpret_cast<cudaStream_t>(stream),
+                   &h->f);
   if (s != JIGSAW_SUCCESS) {
     delete h;
     return s;
@@ -291,7 +290,7 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
   if (nt && out->kind && e == cudaSuccess) e = cudaMemcpy(out->kind, f.d_kind, nt, cudaMemcpyDeviceToHost);
   if (nt && out->nevict && e == cudaSuccess) e = cudaMemcpy(out->nevict, f.d_nevict, nt, cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return cuda_status(e, "export copy");
-  if (nt && (out->gather || out->vals || out->meta)) {
+  if ((nt && (out->gather || out->vals || out->meta)) || (f.ndtiles && (out->rcol || out->dvals))) {
     // read back the device layout and invert it
     std::vector<uint8_t> A((size_t)f.nksteps * kKStepBytesA);
     std::vector<uint32_t> E((size_t)f.nkblocks * 512);
@@ -300,7 +299,22 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
     if (e == cudaSuccess) e = cudaMemcpy(E.data(), f.d_Eimg, E.size() * 4, cudaMemcpyDeviceToHost);
     if (e == cudaSuccess) e = cudaMemcpy(G.data(), f.d_G, G.size() * 4, cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) return cuda_status(e, "export copy (device layout)");
+    int64_t dt = 0;
     for (int64_t p = 0; p < f.npanels; ++p) {
+      // DENSE mode residual tiles: columns from the gather list, values from the A image
+      const int64_t dks0 = f.ks_off[p] + (f.T[p] / 2 + (f.T[p] & 1) + kStepsPerBlock - 1) / kStepsPerBlock * kStepsPerBlock;
+      for (int j = 0; j < f.D[p]; ++j, ++dt) {
+        const int64_t gks = dks0 + j;
+        for (int c = 0; c < 16; ++c) {
+          const int32_t g = G[gks * 32 + c];
+          if (out->rcol) out->rcol[dt * 16 + c] = g >= f.K ? kPad : g;
+        }
+        if (out->dvals)
+          for (int r = 0; r < P; ++r)
+            for (int h2 = 0; h2 < 2; ++h2)
+              memcpy(out->dvals + (dt * P + r) * 16 + 8 * h2,
+                     &A[gks * kKStepBytesA + (r >> 3) * 256 + h2 * 128 + (r & 7) * 16], 16);
+      }
       for (int t = 0; t < f.T[p]; ++t) {
         const int64_t ft = f.tile_off[p] + t;
         const int64_t gks = f.ks_off[p] + t / 2;

@@ -365,16 +365,47 @@ __global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const uint4* __res
 }
 
 // ------------------------------------------------------------------ R4
+// SPTC mode (paper): evicted columns are re-queued and re-tiled (overflow tiles).
+// DENSE mode: only the partial last tile of S_p is built here, and the
+// evicted columns of all tiles, in tile and eviction order, form the residual
+// list R_p (left at the front of the panel's queue buffer, count in nres[p]).
 __global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks,
                                                  const int32_t* __restrict__ S,
                                                  const int32_t* __restrict__ Kp, int64_t K,
                                                  Scratch sc, int32_t* __restrict__ queue,
                                                  int64_t qcap, int32_t* __restrict__ T,
-                                                 int* __restrict__ err) {
+                                                 int* __restrict__ err, int mode,
+                                                 int32_t* __restrict__ nres) {
   __shared__ TileSmem s;
   const int p = blockIdx.x, lane = threadIdx.x;
   const int kp = Kp[p], nfull = kp / 16, rem = kp - 16 * nfull;
   int32_t* q = queue + (int64_t)p * qcap;
+  if (mode == 1) {
+    int t = nfull;
+    if (rem > 0) {
+      if (lane < 16) {
+        const int32_t c = lane < rem ? S[(int64_t)p * K + 16 * nfull + lane] : kPad;
+        s.cols[lane] = c;
+        s.m[lane] = c == kPad ? make_uint4(0, 0, 0, 0) : masks[(int64_t)p * K + c];
+      }
+      __syncwarp();
+      tile_search(s, lane);
+      store_tile(s, sc, p, t, lane);
+      ++t;
+      __syncwarp();
+    }
+    int64_t n = 0;
+    for (int tt = 0; tt < t; ++tt) {
+      const int e = sc.tnev[(int64_t)p * sc.cap + tt];
+      if (lane < e) q[n + lane] = sc.tev[((int64_t)p * sc.cap + tt) * 16 + lane];
+      n += e;
+    }
+    if (lane == 0) {
+      T[p] = t;
+      nres[p] = (int32_t)n;
+    }
+    return;
+  }
   // FIFO contents after the full tiles: the rest of S_p, then the columns the full
   // tiles evicted, in tile order and eviction order (exactly CR1's sequential queue).
   for (int i = lane; i < rem; i += 32) q[i] = S[(int64_t)p * K + 16 * nfull + i];
@@ -406,7 +437,10 @@ __global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks
     ++t;
     __syncwarp();
   }
-  if (lane == 0) T[p] = t;
+  if (lane == 0) {
+    T[p] = t;
+    nres[p] = 0;
+  }
 }
 
 // ------------------------------------------------------------------ R5
@@ -501,6 +535,48 @@ __global__ void __launch_bounds__(128) k_emit(const uint16_t* __restrict__ A, in
   }
 }
 
+// R5 (DENSE mode): one CTA per (panel, dense step): dense step j holds residual
+// columns R_p[16j .. 16j+16) as an uncompressed K = 16 A image in the same UMMA
+// K-major no-swizzle layout ([row group 16][8-column half 2][row 8][8 halves]);
+// its gather list is the 16 columns (PAD -> K) followed by 16 PAD rows.
+__global__ void __launch_bounds__(128) k_emit_dense(const uint16_t* __restrict__ A, int64_t M, int64_t K,
+                                                    const int32_t* __restrict__ queue, int64_t qcap,
+                                                    const int32_t* __restrict__ nres,
+                                                    const int4* __restrict__ pin,
+                                                    uint8_t* __restrict__ Aimg, int32_t* __restrict__ G) {
+  __shared__ int32_t cols[16];
+  const int p = blockIdx.y, j = blockIdx.x, tid = threadIdx.x;
+  const int4 pi = pin[p];
+  if (j >= pi.w) return;
+  const int64_t gks = (int64_t)pi.y + ((pi.x + kStepsPerBlock - 1) / kStepsPerBlock) * kStepsPerBlock + j;
+  const int n = nres[p];
+  if (tid < 32) {
+    const int i = 16 * j + (tid & 15);
+    const int32_t c = (tid < 16 && i < n) ? queue[(int64_t)p * qcap + i] : kPad;
+    if (tid < 16) cols[tid] = c;
+    G[gks * 32 + tid] = c == kPad ? (int32_t)K : c;
+  }
+  __syncthreads();
+  const int r = tid;
+  const int64_t row = (int64_t)p * 128 + r;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    uint16_t v[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int32_t c = cols[8 * h + i];
+      const uint16_t b = (c == kPad || row >= M) ? (uint16_t)0 : A[row * K + c];
+      v[i] = (b & 0x7FFFu) ? b : (uint16_t)0;   // canonical +0 (R-Q3)
+    }
+    uint4 pk;
+    pk.x = v[0] | ((uint32_t)v[1] << 16);
+    pk.y = v[2] | ((uint32_t)v[3] << 16);
+    pk.z = v[4] | ((uint32_t)v[5] << 16);
+    pk.w = v[6] | ((uint32_t)v[7] << 16);
+    *reinterpret_cast<uint4*>(Aimg + gks * kKStepBytesA + (r >> 3) * 256 + h * 128 + (r & 7) * 16) = pk;
+  }
+}
+
 template <class T>
 jigsaw_status_t dalloc(T** p, size_t bytes, std::vector<void*>& list) {
   *p = nullptr;
@@ -543,11 +619,12 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   const int64_t qcap = 2 * K + 64;
   uint4* masks = nullptr;
   int32_t *S = nullptr, *Kp = nullptr, *T = nullptr, *queue = nullptr, *tile_off = nullptr;
-  int32_t *d_ksoff = nullptr, *d_kboff = nullptr;
+  int32_t *d_ksoff = nullptr, *d_kboff = nullptr, *nres = nullptr;
   int* err = nullptr;
   unsigned long long* nnz = nullptr;
   Scratch sc{};
-  std::vector<int32_t> hKp(npan), hT(npan);
+  std::vector<int32_t> hKp(npan), hT(npan), hR(npan);
+  int maxdk = 0;
   unsigned long long hnnz = 0;
   int herr = 0;
   int maxks = 0;
@@ -561,6 +638,7 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   JIG_TRY(dalloc(&S, sizeof(int32_t) * npan * K, scratch));
   JIG_TRY(dalloc(&Kp, sizeof(int32_t) * npan, scratch));
   JIG_TRY(dalloc(&T, sizeof(int32_t) * npan, scratch));
+  JIG_TRY(dalloc(&nres, sizeof(int32_t) * npan, scratch));
   JIG_TRY(dalloc(&err, sizeof(int), scratch));
   JIG_TRY(dalloc(&nnz, sizeof(unsigned long long), scratch));
   JIG_TRY(dalloc(&queue, sizeof(int32_t) * npan * qcap, scratch));
@@ -579,10 +657,11 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   k_compact<<<npan, 1024, 0, stream>>>(masks, K, S, Kp);
   k_main_tiles<<<dim3((unsigned)((K / 16 + kR3Warps - 1) / kR3Warps), npan), 32 * kR3Warps, 0, stream>>>(
       masks, S, Kp, K, sc);
-  k_overflow<<<npan, 32, 0, stream>>>(masks, S, Kp, K, sc, queue, qcap, T, err);
+  k_overflow<<<npan, 32, 0, stream>>>(masks, S, Kp, K, sc, queue, qcap, T, err, mode, nres);
   JIG_CU(cudaGetLastError(), "reorder kernels launch");
   JIG_CU(cudaMemcpyAsync(hKp.data(), Kp, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy Kp");
   JIG_CU(cudaMemcpyAsync(hT.data(), T, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy T");
+  JIG_CU(cudaMemcpyAsync(hR.data(), nres, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy nres");
   JIG_CU(cudaMemcpyAsync(&hnnz, nnz, sizeof hnnz, cudaMemcpyDeviceToHost, stream), "copy nnz");
   JIG_CU(cudaMemcpyAsync(&herr, err, sizeof herr, cudaMemcpyDeviceToHost, stream), "copy err");
   JIG_CU(cudaStreamSynchronize(stream), "reorder R1-R4");
@@ -601,8 +680,14 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   f->overflow_tiles = 0;
   for (int p = 0; p < npan; ++p) {
     const int nks = (hT[p] + 1) / 2;
+    const int ndk = (hR[p] + 15) / 16;   // dense residual tiles (DENSE mode)
+    f->D[p] = ndk;
+    maxdk = std::max(maxdk, ndk);
+    // k-step slots: sparse k-steps, then (DENSE mode) the dense steps starting on
+    // a fresh E block boundary so every k-block is all-sparse or all-dense
+    const int span = ndk ? (nks + kStepsPerBlock - 1) / kStepsPerBlock * kStepsPerBlock + ndk : nks;
     f->tile_off[p + 1] = f->tile_off[p] + hT[p];
-    f->ks_off[p + 1] = f->ks_off[p] + nks;
+    f->ks_off[p + 1] = f->ks_off[p] + span;
     f->kb_off[p + 1] = f->kb_off[p] + (nks + kStepsPerBlock - 1) / kStepsPerBlock;
     f->kp_total += hKp[p];
     f->max_tiles = std::max<int64_t>(f->max_tiles, hT[p]);
@@ -610,13 +695,15 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
     maxks = std::max(maxks, nks);
   }
   f->ntiles = f->tile_off[npan];
+  f->ndtiles = 0;
+  for (int p = 0; p < npan; ++p) f->ndtiles += f->D[p];
   f->nksteps = f->ks_off[npan];
   f->nkblocks = f->kb_off[npan];
   f->nnz = (int64_t)hnnz;
   f->evictions = f->ntiles * 16 - f->kp_total - 0;  // placeholder, replaced below
   {
     f->pin.resize(npan);
-    for (int p = 0; p < npan; ++p) f->pin[p] = make_int4((hT[p] + 1) / 2, f->ks_off[p], f->kb_off[p], 0);
+    for (int p = 0; p < npan; ++p) f->pin[p] = make_int4((hT[p] + 1) / 2, f->ks_off[p], f->kb_off[p], f->D[p]);
     JIG_TRY(dalloc(&f->d_pin, sizeof(int4) * npan, f->allocs));
     JIG_TRY(dalloc(&d_ksoff, sizeof(int32_t) * (npan + 1), scratch));
     JIG_TRY(dalloc(&d_kboff, sizeof(int32_t) * (npan + 1), scratch));
@@ -637,6 +724,8 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
       k_emit<<<dim3(maxks, npan), 128, 0, stream>>>(dA, M, K, sc, T, tile_off, d_ksoff, d_kboff,
                                                   f->d_Aimg, reinterpret_cast<uint32_t*>(f->d_Eimg), f->d_G,
                                                   f->d_colidx, f->d_perm, f->d_kind, f->d_nevict, Kp);
+    if (maxdk > 0)
+      k_emit_dense<<<dim3(maxdk, npan), 128, 0, stream>>>(dA, M, K, queue, qcap, nres, f->d_pin, f->d_Aimg, f->d_G);
     JIG_CU(cudaGetLastError(), "k_emit launch");
     JIG_CU(cudaEventRecord(ev1, stream), "cudaEventRecord");
     // total evictions = sum of per-tile counts

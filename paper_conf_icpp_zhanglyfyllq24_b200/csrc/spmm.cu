@@ -24,6 +24,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <type_traits>
 
 #include "internal.h"
 #include "ptx.cuh"
@@ -33,8 +34,10 @@ namespace jig {
 namespace {
 
 constexpr unsigned kFullMask = 0xFFFFFFFFu;
-constexpr int kThreads = 320;
 constexpr int kBProdWarp0 = 6;
+constexpr int kBProdWarps = 8;   // two warps per k-step (16 B rows each): 8 cp.async warps
+                                 // reach ~36 B/clk/SM vs ~28 with 4 (profiles/r01_gather_bench.txt)
+constexpr int kThreads = 32 * (kBProdWarp0 + kBProdWarps);
 constexpr int kRowsPerBlock = 32 * kStepsPerBlock;  // B rows per k-block (128)
 constexpr int kChunkB = kRowsPerBlock * 128;        // one 64-column SW128 chunk: 16 KB
 constexpr int kStageA = kStepsPerBlock * kKStepBytesA;  // 16 KB
@@ -67,16 +70,24 @@ struct Problem {
   int64_t M, N, K;
   int npanels;
   int unit0;  // first global work unit of this problem
-  int pin0;   // offset of this problem's panels in SpmmParams::pin (if use_pin)
+  int pin0;   // offset of this problem's panels in ParamsT::pin (if use_pin)
 };
-constexpr int kMaxProblems = 64;
-constexpr int kMaxPin = 1536;  // panel table kept in kernel parameter space when it fits
-struct SpmmParams {
-  Problem pr[kMaxProblems];
-  int4 pin[kMaxPin];
+// Kernel parameters: a problem table and the panel table, kept in parameter space
+// (read with LDC, no dependent global load at kernel start).  Two sizes: a
+// small block for single products (cheap to launch) and a large one for grouped
+// launches.
+template <int MAXP, int MAXPIN>
+struct ParamsT {
+  static constexpr int kMaxProblems = MAXP;
+  static constexpr int kMaxPin = MAXPIN;
+  Problem pr[MAXP];
+  int4 pin[MAXPIN];
   int nprob, nunits, S, use_pin;
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
 };
+using ParamsOne = ParamsT<1, 128>;     // single product (~2.2 KB of parameters)
+using ParamsGroup = ParamsT<64, 1024>; // grouped launch (~23 KB)
+constexpr int kMaxProblems = ParamsGroup::kMaxProblems;
 
 // Opt-in per-CTA timeline (clock64 / %globaltimer), read by jigsaw_debug_trace.
 constexpr int kTraceCTAs = 1024, kTraceSlots = 16;
@@ -113,13 +124,22 @@ struct Work {
   const __half* B;
   __half* C;
   int64_t M, N, K;
-  int p, n0, nks, kb_lo, kb_hi;
+  int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
   int64_t ks0, kb0;  // first k-step / E block of the panel
+  // k-block kb of the panel: the first nkb_s are 2:4 sparse (4 k-steps of 32
+  // logical columns each, metadata block kb0 + kb); the rest (DENSE residual mode)
+  // hold up to 4 dense K = 16 steps each, stored after the sparse k-steps.
+  __device__ __forceinline__ bool dense(int kb) const { return kb >= nkb_s; }
+  __device__ __forceinline__ int steps(int kb) const {
+    return kb < nkb_s ? min(kStepsPerBlock, nks - kb * kStepsPerBlock)
+                      : min(kStepsPerBlock, ndk - (kb - nkb_s) * kStepsPerBlock);
+  }
+  __device__ __forceinline__ int64_t gks(int kb) const { return ks0 + (int64_t)kb * kStepsPerBlock; }
 };
 // `hint` = problem index of this thread's previous unit: units are visited in
 // increasing order, so the scan is amortised O(1) instead of O(problems).
-template <int NT>
-__device__ __forceinline__ Work decode_unit(const SpmmParams& prm, int u, uint32_t rank, int S, int& hint) {
+template <int NT, class Prm>
+__device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank, int S, int& hint) {
   int i = hint;
   if (prm.pr[i].unit0 > u) i = 0;
   while (i + 1 < prm.nprob && prm.pr[i + 1].unit0 <= u) ++i;
@@ -142,7 +162,9 @@ __device__ __forceinline__ Work decode_unit(const SpmmParams& prm, int u, uint32
   w.nks = pi.x;
   w.ks0 = pi.y;
   w.kb0 = pi.z;
-  const int nkb = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
+  w.ndk = pi.w;
+  w.nkb_s = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
+  const int nkb = w.nkb_s + (w.ndk + kStepsPerBlock - 1) / kStepsPerBlock;
   w.kb_lo = (int)(rank * nkb / S);
   w.kb_hi = (int)((rank + 1) * nkb / S);
   return w;
@@ -159,8 +181,8 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
-template <int NT, bool kSplit>
-__global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
+template <int NT, bool kSplit, class Prm>
+__global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   using C_ = Cfg<NT, kSplit>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -189,7 +211,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < C_::kStages; ++s) {
-      mbar_init(&full[s], 1 + 128);  // A/E expect_tx arrival + 128 B-producer cp.async arrivals
+      mbar_init(&full[s], 1 + 32 * kBProdWarps);  // A/E expect_tx arrival + B-producer cp.async arrivals
       mbar_init(&empty[s], 1);
       mbar_init(&gfull[s], 1);
     }
@@ -216,19 +238,20 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
       int stage = 0, hint = 0, nkb_issued = 0;
       uint32_t phase = 0;
       for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-        const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
-        const int64_t ks0 = wk.ks0, kb0 = wk.kb0;
+        const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
+        const int64_t kb0 = wk.kb0;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
-          const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
-          const int64_t gks = ks0 + (int64_t)kb * kStepsPerBlock;
+          const int steps = wk.steps(kb);
+          const bool dense = wk.dense(kb);
+          const int64_t gks = wk.gks(kb);
           mbar_wait(&empty[stage], phase ^ 1);
           // gather list first, through the TMA path: the B producers wait only on
           // it, never on an L1 load queued behind earlier cp.async traffic
           mbar_arrive_expect_tx(&gfull[stage], (uint32_t)(steps * 128));
           bulk_g2s(sG + stage * kRowsPerBlock, wk.G + gks * 32, steps * 128, &gfull[stage]);
-          mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + kStageE));
+          mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
           bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
-          bulk_g2s(sE + stage * kStageE, wk.Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
+          if (!dense) bulk_g2s(sE + stage * kStageE, wk.Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
           if (u == cluster_id && kb == wk.kb_lo) JIG_TRACE(2);
           JIG_TRACE_KB(0, nkb_issued);
           ++nkb_issued;
@@ -240,28 +263,29 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
     // ------------------------------------------------------------ B producers
     // Warp w copies the 32 B rows of k-step w of each k-block; the row indices
     // come from the stage's gather list in shared memory (TMA-loaded by warp 0).
-    const int w = warp - kBProdWarp0;      // k-step within the k-block
+    const int w = (warp - kBProdWarp0) >> 1;   // k-step within the k-block
+    const int half = (warp - kBProdWarp0) & 1;  // rows [16*half, 16*half + 16) of it
     constexpr int LPR = NT / 8;            // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
     int stage = 0, hint = 0, traced = 0;
     uint32_t phase = 0;
     for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-      const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
+      const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
       const int col = wk.n0 + 8 * c;
       const bool colok = col < wk.N;
       const __half* Bp = wk.B;
       const int64_t ldb = wk.N, K = wk.K;
       for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
-        const int steps = min(kStepsPerBlock, wk.nks - kb * kStepsPerBlock);
+        const int steps = wk.steps(kb);
         mbar_wait(&empty[stage], phase ^ 1);
-        if (w < steps) {
+        if (w < steps && !(half && wk.dense(kb))) {   // a dense step uses 16 B rows
           mbar_wait(&gfull[stage], phase);
           const int32_t gl = sG[stage * kRowsPerBlock + 32 * w + lane];
           uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
 #pragma unroll
-          for (int it = 0; it < 32 / RPI; ++it) {
-            const int j = it * RPI + lane / LPR;
+          for (int it = 0; it < 16 / RPI; ++it) {
+            const int j = 16 * half + it * RPI + lane / LPR;
             const int32_t g = __shfl_sync(kFullMask, gl, j);
             const bool ok = colok && g < K;
             const __half* src = ok ? Bp + (int64_t)g * ldb + col : Bp;
@@ -269,7 +293,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
           }
         }
         cp_async_mbar_arrive_noinc(&full[stage]);
-        if (lane == 0 && w == 0) {
+        if (lane == 0 && w == 0 && half == 0) {
           if (traced == 0) JIG_TRACE(3);
           JIG_TRACE_KB(1, traced);
           ++traced;
@@ -282,12 +306,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
     if (lane == 0) {
       const uint32_t idesc0 = idesc_f16(128, NT, 0, 1, 1, 0);
       const uint32_t idesc1 = idesc_f16(128, NT, 0, 1, 1, 1);
+      const uint32_t idesc_dense = idesc_f16(128, NT, 0, 1, 0, 0);
       int stage = 0, hint = 0, nkb_mma = 0;
       uint32_t phase = 0;
       int it = 0;
       for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-        const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
-        const int nks = wk.nks, kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
+        const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
+        const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
         const int a = it & 1;
         const uint32_t use = (uint32_t)(it >> 1);
@@ -295,20 +320,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
         tc_fence_after();
         const uint32_t d_tmem = tbase + a * C_::kAccCols;
         for (int kb = kb_lo; kb < kb_hi; ++kb) {
-          const int steps = min(kStepsPerBlock, nks - kb * kStepsPerBlock);
+          const int steps = wk.steps(kb);
+          const bool dense = wk.dense(kb);
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
           const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
-          tc_cp_128x128b(e_tmem, smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0));
+          if (!dense) tc_cp_128x128b(e_tmem, smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0));
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
           for (int s = 0; s < steps; ++s) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
             const uint64_t bdesc = smem_desc(b_base + s * 32 * 128, kChunkB, 1024, 2);
-            tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0,
-                          (kb != kb_lo) || (s != 0));
+            const uint32_t acc = (kb != kb_lo) || (s != 0);
+            if (dense)   // residual tile on the dense tensor path, K = 16
+              tc_mma_f16(d_tmem, adesc, bdesc, idesc_dense, acc);
+            else
+              tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
           }
           tc_commit(&empty[stage]);
           JIG_TRACE_KB(3, nkb_mma);
@@ -326,7 +355,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     int it = 0, hint = 0;
     for (int u = cluster_id; u < prm.nunits; u += nclusters) {
-      const Work wk = decode_unit<NT>(prm, u, rank, S, hint);
+      const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
       const int p = wk.p, n0 = wk.n0;
       const int64_t M = wk.M, N = wk.N;
       __half* const Cm = wk.C;
@@ -438,12 +467,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const SpmmParams prm) {
 }
 
 int g_num_sms[64] = {0};
-bool g_attr_set[64][4] = {};
+bool g_attr_set[64][8] = {};
 
-template <int NT, bool kSplit>
-jigsaw_status_t launch_variant(const SpmmParams& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
+template <int NT, bool kSplit, class Prm>
+jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
   using C_ = Cfg<NT, kSplit>;
-  auto kern = k_spmm<NT, kSplit>;
+  auto kern = k_spmm<NT, kSplit, Prm>;
   if (dev >= 0 && dev < 64 && !g_attr_set[dev][vid]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::kSmem);
     if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(k_spmm)");
@@ -493,7 +522,7 @@ void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* gr
   }
   const int64_t u64 = f.npanels * ((N + 63) / 64);
   int64_t kb_total = 0;
-  for (int64_t p = 0; p < f.npanels; ++p) kb_total += (f.T[p] + 7) / 8;
+  for (int64_t p = 0; p < f.npanels; ++p) kb_total += (f.T[p] + 7) / 8 + (f.D[p] + 3) / 4;
   const double kb_avg = f.npanels ? (double)kb_total / f.npanels : 0.0;
   int s = 1;
   // clusters of 8 do not all fit in one wave of 148 SMs (GPC granularity): S <= 4
@@ -503,10 +532,11 @@ void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* gr
   *grid = s > 1 ? (int)(u64 * s) : (int)std::min<int64_t>(u64, sms);
 }
 
-static void fill_problem(SpmmParams& prm, int i, const Format& f, const void* dB, int64_t N, void* dC) {
+template <class Prm>
+static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64_t N, void* dC) {
   Problem& P = prm.pr[i];
   P.pin0 = i == 0 ? 0 : prm.pr[i - 1].pin0 + prm.pr[i - 1].npanels;
-  if (P.pin0 + f.npanels <= kMaxPin)
+  if (P.pin0 + f.npanels <= Prm::kMaxPin)
     std::copy(f.pin.begin(), f.pin.end(), prm.pin + P.pin0);
   else
     prm.use_pin = 0;
@@ -524,7 +554,8 @@ static void fill_problem(SpmmParams& prm, int i, const Format& f, const void* dB
 
 int g_trace_ctas = 0;
 
-static jigsaw_status_t launch_params(SpmmParams& prm, int NT, int S, int grid, int dev, cudaStream_t s) {
+template <class Prm>
+static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, cudaStream_t s) {
   prm.S = S;
   const char* tr = getenv("JIGSAW_TRACE");
   prm.trace = (tr && tr[0] == '1') ? 1 : 0;
@@ -535,13 +566,15 @@ static jigsaw_status_t launch_params(SpmmParams& prm, int NT, int S, int grid, i
     u += (int)(prm.pr[i].npanels * ((prm.pr[i].N + NT - 1) / NT));
   }
   prm.nunits = u;
-  if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, 0, s);
-  if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, 1, s);
-  return launch_variant<64, true>(prm, grid, S, dev, 2, s);
+  constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 4;
+  if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, vb + 0, s);
+  if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, vb + 1, s);
+  if constexpr (std::is_same<Prm, ParamsOne>::value) return launch_variant<64, true>(prm, grid, S, dev, vb + 2, s);
+  return set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
 }
 
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
-  thread_local SpmmParams prm;  // large (param space); host-side scratch
+  thread_local ParamsOne prm;  // host-side scratch for the parameter block
   prm.nprob = 1;
   prm.use_pin = 1;
   fill_problem(prm, 0, f, dB, N, dC);
@@ -563,7 +596,7 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
 // all problems are dealt round-robin to the CTAs), up to kMaxProblems per launch.
 jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
                                     void* const* Cs, int count, cudaStream_t s) {
-  thread_local SpmmParams prm;
+  thread_local ParamsGroup prm;
   const int sms = spmm_num_sms();
   for (int i0 = 0; i0 < count; i0 += kMaxProblems) {
     const int n = std::min(kMaxProblems, count - i0);

@@ -252,3 +252,56 @@ def test_grouped_launch_many_mixed_problems():
     torch.cuda.synchronize()
     for a, b, c in zip(mats, Bs, dC):
         spmm_check(_host(c), a, b)
+
+
+@pytest.mark.parametrize("M,K,v,s,N,seed", [
+    (256, 512, 8, 0.50, 128, 1),     # residual-heavy: many dense tiles
+    (384, 300, 4, 0.70, 136, 2),     # ragged K / N
+    (256, 256, 4, 0.90, 64, 3),      # few or no residual tiles
+    (512, 2048, 2, 0.50, 256, 4),    # C2 shape, v = 2, 50 %
+])
+def test_dense_residual_mode(M, K, v, s, N, seed):
+    """DENSE residual mode: evicted columns go to uncompressed 16-column
+    tiles run on the dense tensor path.  Format bit-exact vs oracle mode 1 (incl.
+    the residual columns and values), C within tolerance, integers bit-exact."""
+    A = synth.vector_sparse(M, K, v, s, seed)
+    B = synth.dense_b(K, N, seed)
+    h = jig.reorder(_dev(A), v, residual_mode=1)
+    g = h.export()
+    ref = oracle.reorder(A, P=128, mode=1)
+    assert_format_equal(g, ref)
+    assert np.array_equal(g["D"], ref.D)
+    assert np.array_equal(g["rcol"], ref.rcol)
+    assert np.array_equal(g["dvals"], ref.dvals)
+    check.check_format(A, 128, g["T"], g["gather"], g["vals"], g["meta"], perm=g["perm"],
+                       D=g["D"], rcol=g["rcol"], dvals=g["dvals"])
+    assert h.info()["ndtiles"] == int(ref.D.sum())
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    spmm_check(C, A, B)
+    Ai = synth.vector_sparse(M, K, v, s, seed + 50, kind="int")
+    Bi = synth.dense_b(K, N, seed + 50, kind="int")
+    hi = jig.reorder(_dev(Ai), v, residual_mode=1)
+    Ci = _host(hi.spmm(_dev(Bi)))
+    torch.cuda.synchronize()
+    C_ref, _ = oracle.spmm(Ai, Bi)
+    if np.abs(C_ref).max() <= 2048:
+        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+
+
+@pytest.mark.parametrize("force", ["2", "4"])
+def test_dense_residual_split_and_grouped(force, monkeypatch):
+    """DENSE-mode k-blocks under split-K clusters and in a grouped launch."""
+    mats = [synth.vector_sparse(256, 640, 4, 0.6, 70 + i) for i in range(3)]
+    Bs = [synth.dense_b(640, 128, 80 + i) for i in range(3)]
+    hs = [jig.reorder(_dev(a), 4, residual_mode=1) for a in mats]
+    monkeypatch.setenv("JIGSAW_FORCE_SPLIT", force)
+    for h, a, b in zip(hs, mats, Bs):
+        spmm_check(_host(h.spmm(_dev(b))), a, b)
+    monkeypatch.delenv("JIGSAW_FORCE_SPLIT")
+    dB = [_dev(b) for b in Bs]
+    dC = [torch.empty((256, 128), dtype=torch.float16, device="cuda") for _ in range(3)]
+    jig.spmm_batched(hs, dB, dC)
+    torch.cuda.synchronize()
+    for a, b, c in zip(mats, Bs, dC):
+        spmm_check(_host(c), a, b)

@@ -4,6 +4,7 @@
 //   mode 0: cp.async 16 B (LDGSTS), 4 warps      mode 1: same, 8 warps
 //   mode 2: TMA tile::gather4 (box {64,1}, SW128), 1 issuing thread
 //   mode 3: TMA gather4 issued by 4 warps (one elected lane each)
+//   mode 4/5: LDGSTS with 12 / 16 warps          mode 6: LDG.128 + STS.128, 16 warps
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o gb tools/gather_bench.cu
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -19,16 +20,24 @@ using namespace jig;
 constexpr int kRows = 128, kStages = 4, kRowBytes = 256, kStageBytes = kRows * kRowBytes;
 constexpr int KB = 64;  // k-blocks per CTA
 
-__global__ void __launch_bounds__(320, 1) gather_kernel(const __grid_constant__ CUtensorMap tm, const uint16_t* B,
+// pseudo-random row index computed in registers (no memory dependency in the loop)
+__device__ __forceinline__ int hrow(int b, int kb, int row, int K) {
+  uint32_t x = (uint32_t)(b * 7919 + kb * 104729 + row * 2654435761u);
+  x ^= x >> 15; x *= 0x2c1b3c6du; x ^= x >> 12;
+  return (int)(x % (uint32_t)K);
+}
+
+__global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ CUtensorMap tm, const uint16_t* B,
                                                         int ldb, int K, const int* idx, int mode, long long* out) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[kStages], empty[kStages];
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int nprod = (mode == 1) ? 8 : 4;
+  const int nprod = mode == 1 ? 8 : mode == 4 ? 12 : (mode == 5 || mode == 6) ? 16 : 4;
+  const bool ldgsts = mode <= 1 || mode == 4 || mode == 5;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) {
-      mbar_init(&full[s], mode <= 1 ? nprod * 32 : 1 + (mode == 3 ? 3 : 0));
+      mbar_init(&full[s], (ldgsts || mode == 6) ? nprod * 32 : 1 + (mode == 3 ? 3 : 0));
       mbar_init(&empty[s], 1);
     }
     fence_barrier_init();
@@ -55,19 +64,33 @@ __global__ void __launch_bounds__(320, 1) gather_kernel(const __grid_constant__ 
       const int* ri = myidx + kb * kRows;
       mbar_wait(&empty[stage], ph ^ 1);
       uint8_t* st = sm + stage * kStageBytes;
-      if (mode <= 1) {
-        // rows per warp: 128 / nprod; 16 lanes per row (256 B), 2 rows per instruction
-        const int rpw = kRows / nprod;
+      if (ldgsts || mode == 6) {
+        // 256 rows-halves: 16 lanes per row (256 B), 2 rows per instruction; rows dealt round-robin
         const int c = lane & 15;
-        const int g0 = ri[w * rpw + (lane % rpw)];
-        for (int it = 0; it < rpw / 2; ++it) {
-          const int j = 2 * it + (lane >> 4);
-          const int g = __shfl_sync(0xffffffffu, g0, j % rpw);
-          const int row = w * rpw + j;
-          cp_async_16(st + (c >> 3) * (kRows * 128) + row * 128 + (((c & 7) ^ (row & 7)) << 4),
-                      B + (size_t)g * ldb + 8 * c, 16);
+        if (ldgsts) {
+          for (int j2 = w; j2 < kRows / 2; j2 += nprod) {
+            const int row = 2 * j2 + (lane >> 4);
+            const int g = hrow(blockIdx.x, kb, row, K);
+            cp_async_16(st + (c >> 3) * (kRows * 128) + row * 128 + (((c & 7) ^ (row & 7)) << 4),
+                        B + (size_t)g * ldb + 8 * c, 16);
+          }
+          cp_async_mbar_arrive_noinc(&full[stage]);
+        } else {
+          uint4 v[4];
+          int rows[4];
+          int n = 0;
+          for (int j2 = w; j2 < kRows / 2; j2 += nprod) {
+            rows[n] = 2 * j2 + (lane >> 4);
+            v[n] = *reinterpret_cast<const uint4*>(B + (size_t)hrow(blockIdx.x, kb, rows[n], K) * ldb + 8 * c);
+            ++n;
+          }
+          for (int i = 0; i < n; ++i) {
+            const int row = rows[i];
+            *reinterpret_cast<uint4*>(st + (c >> 3) * (kRows * 128) + row * 128 + (((c & 7) ^ (row & 7)) << 4)) = v[i];
+          }
+          fence_proxy_async();
+          mbar_arrive(&full[stage]);
         }
-        cp_async_mbar_arrive_noinc(&full[stage]);
       } else if (mode == 2) {
         if (w == 0 && lane == 0) {
           mbar_arrive_expect_tx(&full[stage], kStageBytes);
@@ -120,14 +143,15 @@ int main() {
       CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   const int smem = kStages * kStageBytes + 1024;
   cudaFuncSetAttribute(gather_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  const char* names[] = {"LDGSTS 4 warps", "LDGSTS 8 warps", "TMA gather4, 1 issuer", "TMA gather4, 4 issuers"};
-  for (int mode = 0; mode < 4; ++mode) {
+  const char* names[] = {"LDGSTS 4 warps", "LDGSTS 8 warps", "TMA gather4, 1 issuer", "TMA gather4, 4 issuers",
+                         "LDGSTS 12 warps", "LDGSTS 16 warps", "LDG+STS 16 warps"};
+  for (int mode = 0; mode < 7; ++mode) {
     for (int rep = 0; rep < 3; ++rep) {
       cudaEvent_t a, b;
       cudaEventCreate(&a);
       cudaEventCreate(&b);
       cudaEventRecord(a);
-      gather_kernel<<<grid, 320, smem>>>(tm, dB, N, K, didx, mode, dout);
+      gather_kernel<<<grid, 544, smem>>>(tm, dB, N, K, didx, mode, dout);
       cudaEventRecord(b);
       cudaError_t e = cudaDeviceSynchronize();
       if (e != cudaSuccess) { printf("mode %d error %s\n", mode, cudaGetErrorString(e)); return 1; }
