@@ -43,19 +43,48 @@ FLUSH_BYTES = 256 << 20
 
 # ------------------------------------------------------------------ workloads
 def workload(name: str):
-    """(points, description).  A point is (M, K, v, s, N)."""
+    """(points, description, scaling).  A point is (M, K, v, s, N)."""
     if name == "c2":
         return synth.c2_points(), ("C2: DLMC-transformer A 512x2048 and 2048x512, v=2/4/8, "
-                                   "s=.50/.70/.80/.90/.95/.98, N=256 (36 matrices)")
+                                   "s=.50/.70/.80/.90/.95/.98, N=256 (36 matrices)"), "weak"
     if name == "c1":
         c = synth.C1
-        return [(c["M"], c["K"], c["v"], c["s"], c["N"])], "C1: 256x256 v=4 s=.80 N=64"
+        return [(c["M"], c["K"], c["v"], c["s"], c["N"])], "C1: 256x256 v=4 s=.80 N=64", "weak"
+    if name == "c3":
+        pts = [(M, K, v, s, N) for (M, K) in synth.C3_SHAPES for v in synth.C3_V for s in synth.C3_S
+               for N in synth.C3_N]
+        return pts, ("C3: ResNet-50 conv-as-GEMM layers (19 shapes) x v=4/8 x s=.70/.80/.90/.95 x "
+                     "N=256/1024 (304 matrices)"), "weak"
     if name == "c4":
         return synth.c4_points(), ("C4: pruned Llama linear 4096x4096 and 11008x4096, v=8, "
-                                   "s=.50/.70/.80/.90, N=2048 (8 matrices)")
+                                   "s=.50/.70/.80/.90, N=2048 (8 matrices)"), "weak"
+    if name == "c5a":
+        L = synth.C2_SHAPES + synth.C3_SHAPES
+        pts = [(L[i % len(L)][0], L[i % len(L)][1], (4, 8)[i % 2], (0.7, 0.8, 0.9, 0.95)[(i // 2) % 4], 256)
+               for i in range(64)]
+        return pts, ("C5a: batch of 64 DLMC-shaped matrices (C2 + C3 shapes), v=4/8, s=.7-.95, N=256, "
+                     "sharded by matrix (LPT) across the GPUs"), "strong"
     if name == "c5b":
-        return [(4096, 4096, 8, 0.90, 16384)], "C5b: 4096x4096 v=8 s=.90 N=16384 (per GPU)"
+        return [(4096, 4096, 8, 0.90, 16384)], ("C5b: 4096x4096 v=8 s=.90 N=16384, B/C column-sharded "
+                                                "across the GPUs"), "strong"
     raise SystemExit(f"unknown workload {name}")
+
+
+def local_jobs(name, points, rank, world):
+    """This rank's share of the workload: list of (M, K, v, s, N, seed, n0, n1).
+    Weak workloads: every point, seeds offset by rank.  c5a: matrices assigned by
+    LPT on the dense-equivalent work.  c5b: the same A on every rank, columns
+    [n0, n1) of one B (paper_conf_icpp_zhanglyfyllq24_b200.shard)."""
+    from paper_conf_icpp_zhanglyfyllq24_b200 import shard
+    if name == "c5a":
+        costs = [2.0 * M * K * N * (1 - s) for (M, K, v, s, N) in points]
+        mine = shard.lpt_assign(costs, world)[rank]
+        return [(*points[i], point_seed(i, 0), 0, points[i][4]) for i in mine]
+    if name == "c5b":
+        (M, K, v, s, N), = points
+        n0, n1 = shard.column_shards(N, world)[rank]
+        return [(M, K, v, s, N, point_seed(0, 0), n0, n1)] if n1 > n0 else []
+    return [(M, K, v, s, N, point_seed(i, rank), 0, N) for i, (M, K, v, s, N) in enumerate(points)]
 
 
 def point_seed(i: int, rank: int) -> int:
@@ -137,7 +166,7 @@ def run_reference(args):
     if rank != 0:
         return 0
     import oracle
-    points, desc = workload(args.workload)
+    points, desc, scaling = workload(args.workload)
     cores = 1
     try:
         os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
@@ -169,7 +198,7 @@ def run_reference(args):
     sample = f"first {rows_per_point} rows of each of the {len(points)} matrices, full N"
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "TFLOP/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+            "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": desc, "l2": "n/a (CPU)"},
             "cpu_baseline": {"value": val, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
@@ -235,13 +264,19 @@ def main():
     stream = torch.cuda.current_stream()
     hbm, bf16, peak_src = load_peaks()
 
-    points, desc = workload(args.workload)
+    all_points, desc, scaling = workload(args.workload)
+    jobs = local_jobs(args.workload, all_points, rank, world)
+    points = [(M, K, v, s, n1 - n0) for (M, K, v, s, N, seed, n0, n1) in jobs]
+    total_eff = sum(2 * M * K * N for (M, K, v, s, N) in all_points) * (world if scaling == "weak" else 1)
     mats, hs, dB, dC, dA = [], [], [], [], []
     reorder_ms = 0.0
     alg_bytes = exec_flops = eff_flops = 0
-    for i, (M, K, v, s, N) in enumerate(points):
-        A = synth.vector_sparse(M, K, v, s, point_seed(i, rank))
-        B = synth.dense_b(K, N, point_seed(i, rank))
+    for (M, K, v, s, N, seed, n0, n1) in jobs:
+        A = synth.vector_sparse(M, K, v, s, seed)
+        B = synth.dense_b(K, N, seed)
+        if (n0, n1) != (0, N):
+            B = np.ascontiguousarray(B[:, n0:n1])
+        N = n1 - n0
         mats.append((A, B))
         a_t = torch.from_numpy(A.view(np.int16)).to(dev).view(torch.float16)
         h = jig.reorder(a_t, v)
@@ -311,7 +346,7 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms = float(t.item())
     ms_per_step = total_ms / args.steps
-    value = eff_flops * world / (ms_per_step * 1e-3) / 1e12
+    value = total_eff / (ms_per_step * 1e-3) / 1e12   # whole job, all ranks
 
     # roofline of the dominant (only) kernel, k_spmm: algorithmic bytes / flops per
     # launch over the average launch duration of the timed region
@@ -329,10 +364,10 @@ def main():
     roof["per_launch_us"] = ms_per_step * 1e3 / launches
     roof["t_roof_us_per_step"] = max(t_hbm, t_tc) * 1e6
     try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        if prof.get("workload") == args.workload:
-            roof["traffic"] = prof["bytes_per_step"] / launches
-            roof["traffic_source"] = prof.get("source")
+        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))[args.workload]
+        roof["traffic"] = prof["bytes_per_step"] / launches
+        roof["traffic_unit"] = "bytes per launch"
+        roof["traffic_source"] = prof.get("source")
     except Exception:
         pass
 
@@ -435,15 +470,15 @@ def main():
     line = {
         "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f16",
+        "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f16",
         "data": "synthetic",
-        "config": {"workload": desc, "matrices_per_gpu": len(points),
+        "config": {"workload": desc, "matrices_on_rank0": len(points),
                    "flops": "dense-equivalent 2*M*N*K per matrix",
                    "l2": "flushed (256 MB write) before every timed step", "launch": "step = jigsaw_spmm_batched over the batch (one grouped k_spmm launch per 64 matrices), captured in a CUDA graph",
                    "seeds": f"synth.SEED_BASE + 1000*rank + index", "format": "P=128, SPTC residual"},
         "roofline": roof,
         "cpu_baseline": cpu,
-        "e2e": {"value": eff_flops * world / e2e_s / 1e12, "unit": "TFLOP/s",
+        "e2e": {"value": total_eff / e2e_s / 1e12, "unit": "TFLOP/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h},
         "e2e_full": {"value": eff_flops / full_s / 1e12, "unit": "TFLOP/s",
                      "note": "rank 0: jigsaw_reorder_host + jigsaw_spmm_host per matrix, one pass"},

@@ -76,17 +76,19 @@ struct Problem {
 // (read with LDC, no dependent global load at kernel start).  Two sizes: a
 // small block for single products (cheap to launch) and a large one for grouped
 // launches.
-template <int MAXP, int MAXPIN>
+template <int MAXP, int MAXPIN, int MAXU>
 struct ParamsT {
   static constexpr int kMaxProblems = MAXP;
   static constexpr int kMaxPin = MAXPIN;
+  static constexpr int kMaxUnits = MAXU;
   Problem pr[MAXP];
   int4 pin[MAXPIN];
-  int nprob, nunits, S, use_pin;
+  uint32_t ulist[MAXU];  // grouped launches: schedule slot -> (problem << 26) | local unit
+  int nprob, nunits, S, use_pin, use_ulist;
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
 };
-using ParamsOne = ParamsT<1, 128>;     // single product (~2.2 KB of parameters)
-using ParamsGroup = ParamsT<64, 1024>; // grouped launch (~23 KB)
+using ParamsOne = ParamsT<1, 128, 1>;        // single product (~2.2 KB of parameters)
+using ParamsGroup = ParamsT<64, 1024, 2048>; // grouped launch (~31 KB)
 constexpr int kMaxProblems = ParamsGroup::kMaxProblems;
 
 // Opt-in per-CTA timeline (clock64 / %globaltimer), read by jigsaw_debug_trace.
@@ -140,10 +142,18 @@ struct Work {
 // increasing order, so the scan is amortised O(1) instead of O(problems).
 template <int NT, class Prm>
 __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank, int S, int& hint) {
-  int i = hint;
-  if (prm.pr[i].unit0 > u) i = 0;
-  while (i + 1 < prm.nprob && prm.pr[i + 1].unit0 <= u) ++i;
-  hint = i;
+  int i, lu;
+  if (Prm::kMaxUnits > 1 && prm.use_ulist) {  // host-ordered schedule (longest units first, snake)
+    const uint32_t code = prm.ulist[u];
+    i = (int)(code >> 26);
+    lu = (int)(code & ((1u << 26) - 1));
+  } else {
+    i = hint;
+    if (prm.pr[i].unit0 > u) i = 0;
+    while (i + 1 < prm.nprob && prm.pr[i + 1].unit0 <= u) ++i;
+    hint = i;
+    lu = u - prm.pr[i].unit0;
+  }
   Work w;
   w.Aimg = prm.pr[i].Aimg;
   w.Eimg = prm.pr[i].Eimg;
@@ -154,7 +164,6 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.N = prm.pr[i].N;
   w.K = prm.pr[i].K;
   const int np = prm.pr[i].npanels;
-  const int lu = u - prm.pr[i].unit0;
   w.p = lu % np;
   w.n0 = (lu / np) * NT;
   // panel table from parameter space (no dependent global load at kernel start)
@@ -577,6 +586,7 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   thread_local ParamsOne prm;  // host-side scratch for the parameter block
   prm.nprob = 1;
   prm.use_pin = 1;
+  prm.use_ulist = 0;
   fill_problem(prm, 0, f, dB, N, dC);
   int NT = 128, S = 1, grid = 1;
   choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
@@ -610,7 +620,34 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
     }
     const int NT = u128 >= 2 * sms ? 128 : 64;
     const int64_t units = NT == 128 ? u128 : u64;
-    jigsaw_status_t st = launch_params(prm, NT, 1, (int)std::min<int64_t>(units, sms), fs[i0]->device, s);
+    const int grid = (int)std::min<int64_t>(units, sms);
+    // Static schedule: units sorted by cost (k-blocks of their panel), longest
+    // first, dealt to the persistent CTAs in snake order (CTA c takes slots
+    // c, c + grid, ...), so the per-CTA loads even out (LPT-like).
+    prm.use_ulist = 0;
+    if (units <= ParamsGroup::kMaxUnits) {
+      thread_local std::vector<std::pair<int, uint32_t>> order;
+      order.clear();
+      for (int i = 0; i < n; ++i) {
+        const Format& f = *fs[i0 + i];
+        const int ntn = (int)((Ns[i0 + i] + NT - 1) / NT);
+        for (int t = 0; t < ntn; ++t)
+          for (int p = 0; p < f.npanels; ++p) {
+            const int cost = (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4 + 1;
+            order.push_back({-cost, ((uint32_t)i << 26) | (uint32_t)(t * f.npanels + p)});
+          }
+      }
+      std::stable_sort(order.begin(), order.end(),
+                       [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
+      for (size_t k = 0; k < order.size(); ++k) {
+        const int r = (int)(k / grid), c = (int)(k % grid);
+        const int mr = (int)std::min<int64_t>(grid, (int64_t)order.size() - (int64_t)r * grid);
+        const int slot = r * grid + ((r & 1) ? mr - 1 - c : c);
+        prm.ulist[slot] = order[k].second;
+      }
+      prm.use_ulist = 1;
+    }
+    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, s);
     if (st != JIGSAW_SUCCESS) return st;
   }
   return JIGSAW_SUCCESS;

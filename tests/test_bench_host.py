@@ -1,0 +1,35 @@
+"""Host logic of bench.py: workloads match BASELINE.json's configs and the
+multi-GPU job split covers every matrix / column exactly once (no GPU)."""
+import numpy as np
+
+import bench
+
+
+def test_workloads():
+    pts, desc, sc = bench.workload("c2")
+    assert len(pts) == 36 and sc == "weak" and all(N == 256 for *_, N in pts)
+    assert {(M, K) for (M, K, *_) in pts} == {(512, 2048), (2048, 512)}
+    assert len(bench.workload("c3")[0]) == 19 * 2 * 4 * 2
+    assert len(bench.workload("c4")[0]) == 8
+    assert len(bench.workload("c5a")[0]) == 64 and bench.workload("c5a")[2] == "strong"
+    assert bench.workload("c5b")[0] == [(4096, 4096, 8, 0.90, 16384)]
+
+
+def test_strong_scaling_jobs_partition_the_work():
+    for name in ("c5a", "c5b"):
+        pts, _, _ = bench.workload(name)
+        for world in (1, 2, 4, 8):
+            jobs = [bench.local_jobs(name, pts, r, world) for r in range(world)]
+            if name == "c5a":
+                seeds = sorted(j[5] for js in jobs for j in js)
+                assert seeds == sorted(bench.point_seed(i, 0) for i in range(64))
+            else:
+                cols = np.concatenate([np.arange(j[6], j[7]) for js in jobs for j in js])
+                assert np.array_equal(cols, np.arange(16384))
+                assert len({j[5] for js in jobs for j in js}) == 1     # same A on every rank
+
+
+def test_weak_scaling_jobs_differ_by_rank():
+    pts, _, _ = bench.workload("c2")
+    a, b = bench.local_jobs("c2", pts, 0, 2), bench.local_jobs("c2", pts, 1, 2)
+    assert len(a) == len(b) == 36 and {j[5] for j in a}.isdisjoint({j[5] for j in b})
