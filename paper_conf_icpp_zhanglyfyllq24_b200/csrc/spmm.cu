@@ -55,7 +55,7 @@ struct Cfg {
   static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
   static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
   static constexpr size_t kSmem =
-      1024 + (size_t)kStages * (kStageB + kStageA + kStageE + kStageG) + kRecvBytes + 320;
+      1024 + (size_t)kStages * (kStageB + kStageA + kStageE + kStageG) + kRecvBytes + 512;
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
@@ -85,6 +85,7 @@ struct ParamsT {
   int4 pin[MAXPIN];
   uint32_t ulist[MAXU];  // grouped launches: schedule slot -> (problem << 26) | local unit
   int nprob, nunits, S, use_pin, use_ulist;
+  int sched;  // >= 0: dynamic tile scheduler on counter slot `sched`; -1: static round-robin
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
 };
 using ParamsOne = ParamsT<1, 128, 1>;        // single product (~2.2 KB of parameters)
@@ -179,6 +180,25 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   return w;
 }
 
+// Dynamic tile scheduler (persistent launches): CTA b starts with unit b, then
+// takes gridDim.x + atomicAdd(counter); the counter slot is reset by the last CTA
+// to finish, so launches (and CUDA-graph replays) need no host-side memset.
+constexpr int kSchedSlots = 64, kSD = 4;  // counter slots per device, unit-ring depth
+__device__ int g_sched[kSchedSlots][2];   // [next unit, CTAs done]
+
+// Unit-ring consumer: the A/E producer publishes each unit id (or -1 = done)
+// into a kSD-deep ring in shared memory; every consumer warp reads the same
+// sequence and releases the slot (one arrival per warp).
+__device__ __forceinline__ int ring_take(const volatile int* ring, uint64_t* rfull, uint64_t* rempty, int& slot,
+                                         uint32_t& ph, bool full_warp, int lane) {
+  mbar_wait(&rfull[slot], ph);
+  const int u = ring[slot];
+  if (full_warp) __syncwarp();
+  if (lane == 0) mbar_arrive(&rempty[slot]);
+  if (++slot == kSD) { slot = 0; ph ^= 1; }
+  return u;
+}
+
 __device__ __forceinline__ float4 ld_shared_f4(uint32_t saddr) {
   float4 v;
   asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(saddr));
@@ -206,12 +226,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint64_t* tfull = gfull + C_::kStages;
   uint64_t* tempty = tfull + 2;
   uint64_t* recv_full = tempty + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(recv_full + 1);
+  uint64_t* rfull = recv_full + 1;   // unit ring (dynamic scheduler)
+  uint64_t* rempty = rfull + kSD;
+  volatile int* ring = reinterpret_cast<volatile int*>(rempty + kSD);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rempty + kSD) + kSD;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = kSplit ? prm.S : 1;
   const uint32_t rank = kSplit ? cluster_ctarank() : 0;
   const int cluster_id = blockIdx.x / S, nclusters = gridDim.x / S;
+  const bool dyn = !kSplit && prm.sched >= 0;
   if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
     g_trace[blockIdx.x * kTraceSlots + 15] = gtimer();
     g_trace[blockIdx.x * kTraceSlots + 14] = smid();
@@ -229,6 +253,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       mbar_init(&tempty[a], 4);
     }
     mbar_init(recv_full, 1);
+    for (int i = 0; i < kSD; ++i) {
+      mbar_init(&rfull[i], 1);
+      mbar_init(&rempty[i], kBProdWarps + 1 + 4);  // B-producer warps + MMA + epilogue warps
+    }
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc<C_::kTmemCols>(tmem_slot);
@@ -244,9 +272,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   if (warp == 0) {
     // ------------------------------------------------------------ A / E producer
     if (lane == 0) {
-      int stage = 0, hint = 0, nkb_issued = 0;
-      uint32_t phase = 0;
-      for (int u = cluster_id; u < prm.nunits; u += nclusters) {
+      int stage = 0, hint = 0, nkb_issued = 0, rslot = 0;
+      uint32_t phase = 0, rph = 0;
+      int* ctr = dyn ? &g_sched[prm.sched][0] : nullptr;
+      for (int un = cluster_id;;) {
+        const int u = un < prm.nunits ? un : -1;
+        if (dyn) {  // publish the unit to the other warp roles
+          mbar_wait(&rempty[rslot], rph ^ 1);
+          ring[rslot] = u;
+          mbar_arrive(&rfull[rslot]);
+          if (++rslot == kSD) { rslot = 0; rph ^= 1; }
+        }
+        if (u < 0) break;
+        un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : u + nclusters;  // latency hidden by the loads below
         const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
         const int64_t kb0 = wk.kb0;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
@@ -267,6 +305,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
+      if (dyn) {  // the last CTA to finish fetching resets the counter slot
+        __threadfence();
+        if (atomicAdd(&g_sched[prm.sched][1], 1) == (int)gridDim.x - 1) {
+          atomicExch(&g_sched[prm.sched][0], 0);
+          atomicExch(&g_sched[prm.sched][1], 0);
+        }
+      }
     }
   } else if (warp >= kBProdWarp0) {
     // ------------------------------------------------------------ B producers
@@ -277,9 +322,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     constexpr int LPR = NT / 8;            // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
-    int stage = 0, hint = 0, traced = 0;
-    uint32_t phase = 0;
-    for (int u = cluster_id; u < prm.nunits; u += nclusters) {
+    int stage = 0, hint = 0, traced = 0, rslot = 0;
+    uint32_t phase = 0, rph = 0;
+    for (int us = cluster_id;; us += nclusters) {
+      const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
+      if (u < 0) break;
       const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
       const int col = wk.n0 + 8 * c;
       const bool colok = col < wk.N;
@@ -316,10 +363,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const uint32_t idesc0 = idesc_f16(128, NT, 0, 1, 1, 0);
       const uint32_t idesc1 = idesc_f16(128, NT, 0, 1, 1, 1);
       const uint32_t idesc_dense = idesc_f16(128, NT, 0, 1, 0, 0);
-      int stage = 0, hint = 0, nkb_mma = 0;
-      uint32_t phase = 0;
+      int stage = 0, hint = 0, nkb_mma = 0, rslot = 0;
+      uint32_t phase = 0, rph = 0;
       int it = 0;
-      for (int u = cluster_id; u < prm.nunits; u += nclusters) {
+      for (int us = cluster_id;; us += nclusters) {
+        const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, false, 0) : (us < prm.nunits ? us : -1);
+        if (u < 0) break;
         const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
@@ -362,8 +411,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   } else {
     // ------------------------------------------------------------ epilogue (warps 2-5)
     const int q = warp & 3;  // TMEM lane quarter this warp may access
-    int it = 0, hint = 0;
-    for (int u = cluster_id; u < prm.nunits; u += nclusters) {
+    int it = 0, hint = 0, rslot = 0;
+    uint32_t rph = 0;
+    for (int us = cluster_id;; us += nclusters) {
+      const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
+      if (u < 0) break;
       const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
       const int p = wk.p, n0 = wk.n0;
       const int64_t M = wk.M, N = wk.N;
@@ -563,9 +615,15 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
 
 int g_trace_ctas = 0;
 
+int g_sched_next[64] = {0};
+
 template <class Prm>
 static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, cudaStream_t s) {
   prm.S = S;
+  // persistent launches use the dynamic scheduler on a rotating counter slot
+  prm.sched = -1;
+  if (S == 1 && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
+    prm.sched = (g_sched_next[dev]++) % kSchedSlots;
   const char* tr = getenv("JIGSAW_TRACE");
   prm.trace = (tr && tr[0] == '1') ? 1 : 0;
   if (prm.trace) g_trace_ctas = std::min(grid, kTraceCTAs);

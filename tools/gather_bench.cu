@@ -5,6 +5,8 @@
 //   mode 2: TMA tile::gather4 (box {64,1}, SW128), 1 issuing thread
 //   mode 3: TMA gather4 issued by 4 warps (one elected lane each)
 //   mode 4/5: LDGSTS with 12 / 16 warps          mode 6: LDG.128 + STS.128, 16 warps
+//   mode 7/8: TMA gather4 from 8 / 16 issuing warps
+//   mode 9: half the rows by 8 LDGSTS warps, half by 8 TMA gather4 warps
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o gb tools/gather_bench.cu
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -33,11 +35,14 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[kStages], empty[kStages];
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int nprod = mode == 1 ? 8 : mode == 4 ? 12 : (mode == 5 || mode == 6) ? 16 : 4;
+  const int nprod = mode == 1 ? 8 : mode == 4 ? 12 : (mode == 5 || mode == 6 || mode == 8 || mode == 9) ? 16
+                    : mode == 7 ? 8 : 4;
   const bool ldgsts = mode <= 1 || mode == 4 || mode == 5;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) {
-      mbar_init(&full[s], (ldgsts || mode == 6) ? nprod * 32 : 1 + (mode == 3 ? 3 : 0));
+      mbar_init(&full[s], (ldgsts || mode == 6) ? nprod * 32
+                          : mode == 9 ? 8 * 32 + 8
+                          : (mode == 7 || mode == 8) ? nprod : 1 + (mode == 3 ? 3 : 0));
       mbar_init(&empty[s], 1);
     }
     fence_barrier_init();
@@ -91,6 +96,31 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
           fence_proxy_async();
           mbar_arrive(&full[stage]);
         }
+      } else if (mode == 7 || mode == 8 || (mode == 9 && w >= 8)) {
+        // TMA gather4: each issuing warp takes a share of the 32 row-quads x 2 chunks
+        const int nt = mode == 9 ? 8 : nprod, wt = mode == 9 ? w - 8 : w;
+        const int q0 = mode == 9 ? 16 : 0;                      // mode 9: rows 64..127
+        const int nq = mode == 9 ? 16 : 32;
+        if (lane == 0) {
+          uint32_t bytes = 0;
+          for (int q = q0 + wt; q < q0 + nq; q += nt) bytes += 2 * 512;
+          mbar_arrive_expect_tx(&full[stage], bytes);
+          for (int q = q0 + wt; q < q0 + nq; q += nt)
+            for (int ch = 0; ch < 2; ++ch)
+              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, hrow(blockIdx.x, kb, 4 * q, K),
+                          hrow(blockIdx.x, kb, 4 * q + 1, K), hrow(blockIdx.x, kb, 4 * q + 2, K),
+                          hrow(blockIdx.x, kb, 4 * q + 3, K), &full[stage]);
+        }
+      } else if (mode == 9) {
+        // LDGSTS warps 0..7: rows 0..63
+        const int c = lane & 15;
+        for (int j2 = w; j2 < 32; j2 += 8) {
+          const int row = 2 * j2 + (lane >> 4);
+          const int g = hrow(blockIdx.x, kb, row, K);
+          cp_async_16(st + (c >> 3) * (kRows * 128) + row * 128 + (((c & 7) ^ (row & 7)) << 4),
+                      B + (size_t)g * ldb + 8 * c, 16);
+        }
+        cp_async_mbar_arrive_noinc(&full[stage]);
       } else if (mode == 2) {
         if (w == 0 && lane == 0) {
           mbar_arrive_expect_tx(&full[stage], kStageBytes);
@@ -144,8 +174,9 @@ int main() {
   const int smem = kStages * kStageBytes + 1024;
   cudaFuncSetAttribute(gather_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   const char* names[] = {"LDGSTS 4 warps", "LDGSTS 8 warps", "TMA gather4, 1 issuer", "TMA gather4, 4 issuers",
-                         "LDGSTS 12 warps", "LDGSTS 16 warps", "LDG+STS 16 warps"};
-  for (int mode = 0; mode < 7; ++mode) {
+                         "LDGSTS 12 warps", "LDGSTS 16 warps", "LDG+STS 16 warps", "TMA gather4, 8 issuers",
+                         "TMA gather4, 16 issuers", "LDGSTS 8w + gather4 8w"};
+  for (int mode = 0; mode < 10; ++mode) {
     for (int rep = 0; rep < 3; ++rep) {
       cudaEvent_t a, b;
       cudaEventCreate(&a);
