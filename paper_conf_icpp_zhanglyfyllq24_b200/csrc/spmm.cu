@@ -48,10 +48,11 @@ template <int NT, bool kSplit>
 struct Cfg {
   static constexpr int kChunks = NT / 64;
   static constexpr int kStageB = kChunks * kChunkB;
-  static constexpr int kStages = NT == 128 ? 4 : 5;
+  static constexpr int kStages = NT == 256 ? 2 : NT == 128 ? 4 : 5;
   static constexpr int kAccCols = NT;
-  static constexpr int kEColBase = 2 * NT;
-  static constexpr uint32_t kTmemCols = 2 * NT + 4 * kStages <= 256 ? 256 : 512;
+  static constexpr int kAccBufs = NT == 256 ? 1 : 2;   // TMEM: 512 columns total
+  static constexpr int kEColBase = kAccBufs * NT;
+  static constexpr uint32_t kTmemCols = kAccBufs * NT + 4 * kStages <= 256 ? 256 : 512;
   static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
   static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
   static constexpr size_t kSmem =
@@ -372,8 +373,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
-        const int a = it & 1;
-        const uint32_t use = (uint32_t)(it >> 1);
+        const int a = it % C_::kAccBufs;
+        const uint32_t use = (uint32_t)(it / C_::kAccBufs);
         mbar_wait(&tempty[a], (use & 1) ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tbase + a * C_::kAccCols;
@@ -422,9 +423,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       __half* const Cm = wk.C;
       const bool has_acc = wk.kb_hi > wk.kb_lo;
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
-      const int a = it & 1;
+      const int a = it % C_::kAccBufs;
       if (has_acc) {
-        mbar_wait(&tfull[a], (uint32_t)(it >> 1) & 1);
+        mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
         tc_fence_after();
       }
       if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
@@ -528,7 +529,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 }
 
 int g_num_sms[64] = {0};
-bool g_attr_set[64][8] = {};
+bool g_attr_set[64][8] = {};  // [device][variant]
 
 template <int NT, bool kSplit, class Prm>
 jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
@@ -574,8 +575,18 @@ int spmm_num_sms() {
 // persistent; otherwise NT = 64 and, when the panels carry enough k-blocks,
 // split-K over a cluster of S = 2/4/8 CTAs.
 void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* grid) {
-  const int64_t u128 = f.npanels * ((N + 127) / 128);
-  if (u128 >= sms) {
+  const int64_t u256 = f.npanels * ((N + 255) / 256), u128 = f.npanels * ((N + 127) / 128);
+  const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
+  int64_t kbs = 0;
+  for (int64_t p = 0; p < f.npanels; ++p) kbs += (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
+  const bool long_units = kbs >= 24 * f.npanels;  // NT = 256 runs a 2-stage ring: needs long units
+  if ((u256 >= sms && long_units && force == 0) || force == 256) {   // large: A read once per 256 columns
+    *NT = 256;
+    *S = 1;
+    *grid = (int)std::min<int64_t>(u256, sms);
+    return;
+  }
+  if (u128 >= sms || force == 128) {
     *NT = 128;
     *S = 1;
     *grid = (int)std::min<int64_t>(u128, sms);
@@ -634,6 +645,7 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   }
   prm.nunits = u;
   constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 4;
+  if (NT == 256) return launch_variant<256, false>(prm, grid, 1, dev, vb + 3, s);
   if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, vb + 0, s);
   if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, vb + 1, s);
   if constexpr (std::is_same<Prm, ParamsOne>::value) return launch_variant<64, true>(prm, grid, S, dev, vb + 2, s);
@@ -676,8 +688,18 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
       u128 += fs[i0 + i]->npanels * ((Ns[i0 + i] + 127) / 128);
       u64 += fs[i0 + i]->npanels * ((Ns[i0 + i] + 63) / 64);
     }
-    const int NT = u128 >= 2 * sms ? 128 : 64;
-    const int64_t units = NT == 128 ? u128 : u64;
+    int64_t u256 = 0, kbs = 0, npan = 0;
+    for (int i = 0; i < n; ++i) {
+      const Format& f = *fs[i0 + i];
+      u256 += f.npanels * ((Ns[i0 + i] + 255) / 256);
+      for (int64_t p = 0; p < f.npanels; ++p) kbs += (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
+      npan += f.npanels;
+    }
+    const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
+    int NT = u128 >= 2 * sms ? 128 : 64;
+    if ((u256 >= sms && kbs >= 24 * npan && force == 0) || force == 256) NT = 256;
+    if (force == 128 || force == 64) NT = force;
+    const int64_t units = NT == 256 ? u256 : NT == 128 ? u128 : u64;
     const int grid = (int)std::min<int64_t>(units, sms);
     // Static schedule: units sorted by cost (k-blocks of their panel), longest
     // first, dealt to the persistent CTAs in snake order (CTA c takes slots

@@ -305,3 +305,21 @@ def test_dense_residual_split_and_grouped(force, monkeypatch):
     torch.cuda.synchronize()
     for a, b, c in zip(mats, Bs, dC):
         spmm_check(_host(c), a, b)
+
+
+@pytest.mark.parametrize("nt", ["64", "128", "256"])
+def test_tile_width_variants(nt, monkeypatch):
+    """k_spmm with N tiles of 64 / 128 / 256 columns (single and grouped launches,
+    SPTC and DENSE residual), N not a multiple of the tile width."""
+    monkeypatch.setenv("JIGSAW_FORCE_NT", nt)
+    mats = [synth.vector_sparse(384, 700, 8, 0.85, 90 + i) for i in range(2)]
+    Bs = [synth.dense_b(700, 328, 91 + i) for i in range(2)]
+    hs = [jig.reorder(_dev(mats[0]), 8), jig.reorder(_dev(mats[1]), 8, residual_mode=1)]
+    for h, a, b in zip(hs, mats, Bs):
+        spmm_check(_host(h.spmm(_dev(b))), a, b)
+    dB = [_dev(b) for b in Bs]
+    dC = [torch.empty((384, 328), dtype=torch.float16, device="cuda") for _ in range(2)]
+    jig.spmm_batched(hs, dB, dC)
+    torch.cuda.synchronize()
+    for a, b, c in zip(mats, Bs, dC):
+        spmm_check(_host(c), a, b)
