@@ -130,8 +130,11 @@ __device__ __forceinline__ bool compat(const TileSmem& s, uint32_t sub) {
 // Lexicographically first completion of the cover given g0 (R-Q8): g1 holds the
 // smallest uncovered slot, candidates tried in lexicographic order; then g2; g3
 // is the rest.
+// Pruning (exact, never changes the result): no compatible group holds more than
+// `hmax` real columns, so the real columns still uncovered must fit hmax per
+// remaining group.
 __device__ bool complete_cover(const TileSmem& s, uint32_t used, uint32_t& o1, uint32_t& o2,
-                               uint32_t& o3) {
+                               uint32_t& o3, uint32_t realset, int hmax) {
   const int lo1 = __ffs(~used & 0xFFFFu) - 1;
   const uint32_t av1 = ~used & 0xFFFFu & ~(1u << lo1);
   for (uint32_t x = av1; x; x &= x - 1) {
@@ -143,6 +146,7 @@ __device__ bool complete_cover(const TileSmem& s, uint32_t used, uint32_t& o1, u
         const uint32_t s1 = (1u << lo1) | (1u << b) | (1u << c) | (1u << d);
         if (!compat(s, s1)) continue;
         const uint32_t u2 = used | s1;
+        if (__popc(realset & ~u2) > 2 * hmax) continue;
         const int lo2 = __ffs(~u2 & 0xFFFFu) - 1;
         const uint32_t av2 = ~u2 & 0xFFFFu & ~(1u << lo2);
         for (uint32_t x2 = av2; x2; x2 &= x2 - 1) {
@@ -279,7 +283,30 @@ __device__ void tile_search(TileSmem& s, int lane) {
     // Necessary conditions for a cover (they only skip searches that must fail):
     // every slot lies in some compatible group; 4 groups can hold all real columns.
     bool coverable = __all_sync(kFull, lane >= 16 || fr > 0) && hmax * 4 >= __popc(realset);
-    if (coverable && __popc(realset) > 8) coverable = cover_exists(s, realset, lane);
+    const int nreal = __popc(realset);
+    if (nreal > 8) {
+      const bool ex = cover_exists(s, realset, lane);
+      if (s.nbig == 0) {
+        // No compatible group holds 3+ real columns, and none will after more
+        // evictions: every real column is in the same number of compatible groups
+        // (C(pad,3) + (real-1)*C(pad,2)), so the retry evicts the smallest real
+        // slots one by one until 8 remain -- done here in one step (identical result).
+        if (lane == 0) {
+          int need = nreal - 8;
+          for (int j = 0; j < 16 && need > 0; ++j) {
+            if (!((realset >> j) & 1u)) continue;
+            s.ev[s.nev++] = s.cols[j];
+            s.cols[j] = kPad;
+            s.m[j] = make_uint4(0, 0, 0, 0);
+            --need;
+          }
+        }
+        __syncwarp();
+        realset = __ballot_sync(kFull, lane < 16 && s.cols[lane] != kPad) & 0xFFFFu;
+        continue;
+      }
+      coverable = coverable && ex;
+    }
     // Alg. 1 lines 9-17: lanes try the candidates for g0 (groups containing slot 0)
     // in lexicographic order, 32 at a time; the lowest successful one wins.
     if (coverable) {
@@ -289,7 +316,8 @@ __device__ void tile_search(TileSmem& s, int lane) {
         bool ok = false;
         if (k < kNumG0) {
           g0 = g_subs[k];
-          ok = compat(s, g0) && complete_cover(s, g0, a1, a2, a3);
+          ok = compat(s, g0) && __popc(realset & ~g0) <= 3 * hmax &&
+               complete_cover(s, g0, a1, a2, a3, realset, hmax);
         }
         const unsigned b = __ballot_sync(kFull, ok);
         if (b) {

@@ -29,9 +29,10 @@ def report(tag, ev_us, tr, ghz):
           f"start spread {(start.max() - start.min()) / 1e3:.2f} us")
     for k, name in NAMES.items():
         d = (tr[:, k] - tr[:, 0]) / ghz / 1e3
-        d = d[tr[:, k] != 0]
+        d = d[(tr[:, k] != 0) & (d > -1) & (d < 1e4)]
         if len(d):
-            print(f"   {name:16s} median {np.median(d):7.2f} us   max {d.max():7.2f} us")
+            print(f"   {name:16s} min {d.min():7.2f}  p10 {np.percentile(d, 10):7.2f}  median {np.median(d):7.2f}"
+                  f"  p90 {np.percentile(d, 90):7.2f}  max {d.max():7.2f} us")
 
 
 def main():
