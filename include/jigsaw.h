@@ -175,8 +175,9 @@ JIGSAW_API int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N);
  * copy, first B copies, first full stage, last MMA commit, accumulator ready,
  * sends done, reduction data ready, stores done, exit), 13 / 15 are
  * %globaltimer (ns) at exit / entry, 14 is the SM id.  max_ctas < 0 instead
- * copies the per-k-block timeline of CTAs 0..7 (8 x 4 x 32 int64: A/E copy
- * issued, B copies issued, stage full seen by the MMA thread, MMAs committed).
+ * copies the per-k-block timeline of CTAs 0..7 (8 x 6 x 32 int64: A/E copy
+ * issued, B copies issued, stage full seen by the MMA thread, commit issued,
+ * metadata copy issued, MMAs issued).
  * Synchronous.  Returns the number of records copied (0 if none, -1 on a CUDA
  * error). */
 JIGSAW_API int jigsaw_debug_trace(int64_t* out, int max_ctas);

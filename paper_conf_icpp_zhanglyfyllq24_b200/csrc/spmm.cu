@@ -97,11 +97,11 @@ constexpr int kMaxProblems = ParamsGroup::kMaxProblems;
 constexpr int kTraceCTAs = 1024, kTraceSlots = 16;
 __device__ long long g_trace[kTraceCTAs * kTraceSlots];
 constexpr int kTraceKB = 32;
-__device__ long long g_trace_kb[8 * 4 * kTraceKB];  // [cta<8][AE issue, B issue, full seen, mma done][kb]
+__device__ long long g_trace_kb[8 * 6 * kTraceKB];  // [cta<8][AE issue, B issue, full seen, commit, after cp, after mma][kb]
 #define JIG_TRACE_KB(role, n)                                                        \
   do {                                                                               \
     if (prm.trace && blockIdx.x < 8 && (n) < kTraceKB)                               \
-      g_trace_kb[(blockIdx.x * 4 + (role)) * kTraceKB + (n)] = clock64();            \
+      g_trace_kb[(blockIdx.x * 6 + (role)) * kTraceKB + (n)] = clock64();            \
   } while (0)
 __device__ __forceinline__ long long gtimer() {
   long long t;
@@ -387,6 +387,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           JIG_TRACE_KB(2, nkb_mma);
           const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
           if (!dense) tc_cp_128x128b(e_tmem, smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0));
+          JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
           for (int s = 0; s < steps; ++s) {
@@ -398,6 +399,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             else
               tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
           }
+          JIG_TRACE_KB(5, nkb_mma);
           tc_commit(&empty[stage]);
           JIG_TRACE_KB(3, nkb_mma);
           ++nkb_mma;
@@ -737,8 +739,8 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
 // int64 slots (clock64 at the trace points 0-11, 13 = %globaltimer at exit,
 // 14 = SM id, 15 = %globaltimer at entry).  Returns the CTA count.
 int debug_trace_read(long long* host, int max_ctas) {
-  if (max_ctas < 0) {  // per-k-block timeline of CTAs 0..7: 8*4*32 int64
-    if (cudaMemcpyFromSymbol(host, g_trace_kb, sizeof(long long) * 8 * 4 * kTraceKB) != cudaSuccess) return -1;
+  if (max_ctas < 0) {  // per-k-block timeline of CTAs 0..7: 8*6*32 int64
+    if (cudaMemcpyFromSymbol(host, g_trace_kb, sizeof(long long) * 8 * 6 * kTraceKB) != cudaSuccess) return -1;
     return 8;
   }
   const int n = std::min(max_ctas, g_trace_ctas);

@@ -101,7 +101,8 @@ __global__ void probe_kernel(const uint8_t* A_img, const uint8_t* E_img, const _
 }
 
 // throughput: loop of MMAs on garbage smem data
-__global__ void tput_kernel(int iters, int sparse, long long* cycles) {
+//   alay: A smem layout 0 = no swizzle (LBO 128, SBO 256), 6 = SW32 K-major, 2 = SW128 K-major
+__global__ void tput_kernel(int iters, int sparse, int N, int alay, long long* cycles) {
   extern __shared__ __align__(1024) uint8_t sm[];
   __shared__ uint64_t bar;
   __shared__ uint32_t tmem_base;
@@ -112,9 +113,11 @@ __global__ void tput_kernel(int iters, int sparse, long long* cycles) {
   tc_fence_after();
   uint32_t tb = tmem_base;
   if (tid == 0) {
-    uint64_t adesc = smem_desc(smem_u32(sm), 128, 256, 0);
-    uint64_t bdesc = smem_desc(smem_u32(sm + 8192), 4096 * 2, 1024, 2);
-    uint32_t idesc = idesc_f16(128, 256, 0, 1, sparse, 0);
+    uint64_t adesc = alay == 0 ? smem_desc(smem_u32(sm), 128, 256, 0)
+                   : alay == 6 ? smem_desc(smem_u32(sm), 16, 256, 6)
+                               : smem_desc(smem_u32(sm), 16, 1024, 2);
+    uint64_t bdesc = smem_desc(smem_u32(sm + 32768), 4096 * 2, 1024, 2);
+    uint32_t idesc = idesc_f16(128, N, 0, 1, sparse, 0);
     long long t0 = clock64();
     for (int i = 0; i < iters; ++i) {
       if (sparse) tc_mma_sp_f16(tb, adesc, bdesc, tb + 256, idesc, 1);
@@ -276,25 +279,30 @@ int main() {
   // throughput
   long long* dcyc;
   CK(cudaMalloc(&dcyc, 148 * 8));
-  CK(cudaFuncSetAttribute(tput_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 80 * 1024));
-  for (int sp = 0; sp <= 1; ++sp) {
+  struct TV { int sp, N, alay; const char* name; };
+  TV tvs[] = {{0, 256, 0, "dense  N256 A noswz"}, {1, 256, 0, "sparse N256 A noswz"},
+              {1, 128, 0, "sparse N128 A noswz"}, {1, 64, 0, "sparse N64  A noswz"},
+              {1, 128, 6, "sparse N128 A SW32 "}, {1, 128, 2, "sparse N128 A SW128"},
+              {0, 128, 0, "dense  N128 A noswz"}, {0, 128, 2, "dense  N128 A SW128"}};
+  CK(cudaFuncSetAttribute(tput_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 100 * 1024));
+  for (auto& tv : tvs) {
     int iters = 4096;
-    tput_kernel<<<148, 128, 80 * 1024>>>(iters, sp, dcyc);
+    tput_kernel<<<148, 128, 100 * 1024>>>(iters, tv.sp, tv.N, tv.alay, dcyc);
     CK(cudaDeviceSynchronize());
     cudaEvent_t a, b;
     cudaEventCreate(&a);
     cudaEventCreate(&b);
     cudaEventRecord(a);
-    tput_kernel<<<148, 128, 80 * 1024>>>(iters, sp, dcyc);
+    tput_kernel<<<148, 128, 100 * 1024>>>(iters, tv.sp, tv.N, tv.alay, dcyc);
     cudaEventRecord(b);
     CK(cudaDeviceSynchronize());
     float ms;
     cudaEventElapsedTime(&ms, a, b);
     long long cyc;
     CK(cudaMemcpy(&cyc, dcyc, 8, cudaMemcpyDeviceToHost));
-    double flops = 2.0 * 128 * 256 * (sp ? 32 : 16) * (double)iters * 148;  // logical
-    printf("%s MMA M128 N256: %.1f cycles/mma (SM0), %.1f TFLOP/s logical (event %.3f ms)\n",
-           sp ? "sparse" : "dense ", (double)cyc / iters, flops / ms / 1e9, ms);
+    double flops = 2.0 * 128 * tv.N * (tv.sp ? 32 : 16) * (double)iters * 148;  // logical
+    printf("%s: %.1f cycles/mma (SM0), %.1f TFLOP/s logical (event %.3f ms)\n", tv.name,
+           (double)cyc / iters, flops / ms / 1e9, ms);
   }
   return 0;
 }

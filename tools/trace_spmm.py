@@ -71,15 +71,15 @@ def main():
         torch.cuda.synchronize()
     tr = jig.debug_trace()
     report("grouped C2 batch (36)", e0.elapsed_time(e1) * 1e3, tr, ghz)
-    kb = np.zeros(8 * 4 * 32, np.int64)
+    kb = np.zeros(8 * 6 * 32, np.int64)
     import ctypes
     jig.lib().jigsaw_debug_trace(kb.ctypes.data_as(ctypes.c_void_p), -1)
-    kb = kb.reshape(8, 4, 32)
+    kb = kb.reshape(8, 6, 32)
     for cta in range(2):
         t0 = tr[cta, 0]
-        print(f"  CTA {cta} per k-block (us after entry): AE-issue / B-issue / full-seen / mma-commit")
+        print(f"  CTA {cta} per k-block (us after entry): AE-issue / B-issue / full-seen / after-cp / after-mma / commit")
         for k in range(32):
-            row = [(kb[cta, r, k] - t0) / ghz / 1e3 if kb[cta, r, k] > t0 else float('nan') for r in range(4)]
+            row = [(kb[cta, r, k] - t0) / ghz / 1e3 if kb[cta, r, k] > t0 else float('nan') for r in (0, 1, 2, 4, 5, 3)]
             print("   kb %2d  " % k + "  ".join(f"{x:7.2f}" for x in row))
 
 
