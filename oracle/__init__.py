@@ -102,13 +102,13 @@ def spmm(A, B, rows=None):
 def tile_reorder(masks, cols, W=16, G=4, Z=2):
     """Alg. 1 + reorder retry on one tile.
 
-    masks: W python ints (row bitmasks, row r = bit r, P <= 128 rows)
+    masks: W python ints (row bitmasks, row r = bit r, P <= 256 rows)
     cols : W column ids (PAD = -1)
     Returns (perm, cols_after, evicted)."""
-    m = np.zeros(2 * W, dtype=np.uint64)
+    m = np.zeros(4 * W, dtype=np.uint64)
     for j, x in enumerate(masks):
-        m[2 * j] = np.uint64(int(x) & ((1 << 64) - 1))
-        m[2 * j + 1] = np.uint64(int(x) >> 64)
+        for w in range(4):
+            m[4 * j + w] = np.uint64((int(x) >> (64 * w)) & ((1 << 64) - 1))
     c = np.ascontiguousarray(np.asarray(cols, dtype=np.int32))
     perm = np.zeros(W, dtype=np.uint8)
     ev = np.zeros(16, dtype=np.int32)

@@ -96,12 +96,13 @@ int orc_spmm(const uint16_t *A, int64_t M, int64_t K,
 }
 
 /* ------------------------------------------------------------------------- */
-/* Row masks: one P-bit mask per column of a panel (P <= 128, two 64-bit words)*/
+/* Row masks: one P-bit mask per column of a panel (P <= 256, four 64-bit words)*/
 /* ------------------------------------------------------------------------- */
 
-typedef struct { uint64_t w[2]; } mask128;
+#define MASK_WORDS 4
+typedef struct { uint64_t w[MASK_WORDS]; } mask256;
 
-static int mask_is_zero(mask128 m) { return (m.w[0] | m.w[1]) == 0; }
+static int mask_is_zero(mask256 m) { return (m.w[0] | m.w[1] | m.w[2] | m.w[3]) == 0; }
 
 /* ------------------------------------------------------------------------- */
 /* Alg. 1 + reorder retry on one tile                    */
@@ -109,7 +110,7 @@ static int mask_is_zero(mask128 m) { return (m.w[0] | m.w[1]) == 0; }
 
 typedef struct {
     int W, G, Z;                /* tile width, group size, max nonzeros per group and row */
-    mask128 m[16];              /* per-slot row masks; PAD slots have mask 0 */
+    mask256 m[16];              /* per-slot row masks; PAD slots have mask 0 */
     int real[16];               /* 1 if the slot holds a real (non-PAD) column */
     unsigned char compat[1 << 16];   /* compat[S] for every G-subset S (bitmask of slots) */
     int nsub;                   /* number of G-subsets of W slots */
@@ -151,7 +152,7 @@ static void enum_subsets(tile_ctx *t)
  * plane c[j] has a row bit set once that row has seen > j nonzeros. */
 static int group_compatible(const tile_ctx *t, uint32_t s)
 {
-    for (int w = 0; w < 2; ++w) {
+    for (int w = 0; w < MASK_WORDS; ++w) {
         uint64_t c[17] = {0};
         for (uint32_t rest = s; rest; rest &= rest - 1) {
             int j = __builtin_ctz(rest);
@@ -186,7 +187,7 @@ static int dfs(tile_ctx *t, uint32_t used, int depth)
 }
 
 /* TileReorder on one tile (R-Q8, R-Q11).
- *  masks  : W row masks (2 words each, row r of the panel is bit r%64 of word r/64)
+ *  masks  : W row masks (4 words each, row r of the panel is bit r%64 of word r/64)
  *  cols   : in/out, W column ids (ORC_PAD = -1); evicted slots become ORC_PAD
  *  perm   : out, W slot indices: the new column order g0 || g1 || ... (groups sorted)
  *  evicted: out, evicted column ids in eviction order; *nev their count
@@ -204,8 +205,8 @@ int orc_tile_reorder(const uint64_t *masks, int W, int G, int Z,
     enum_subsets(t);
     for (int j = 0; j < W; ++j) {
         t->real[j] = cols[j] != ORC_PAD;
-        t->m[j].w[0] = t->real[j] ? masks[2 * j] : 0;
-        t->m[j].w[1] = t->real[j] ? masks[2 * j + 1] : 0;
+        for (int w = 0; w < MASK_WORDS; ++w)
+            t->m[j].w[w] = t->real[j] ? masks[MASK_WORDS * j + w] : 0;
     }
     *nev = 0;
     for (;;) {
@@ -254,7 +255,7 @@ int orc_tile_reorder(const uint64_t *masks, int W, int G, int Z,
         evicted[(*nev)++] = cols[best];
         cols[best] = ORC_PAD;
         t->real[best] = 0;
-        t->m[best].w[0] = t->m[best].w[1] = 0;
+        for (int w = 0; w < MASK_WORDS; ++w) t->m[best].w[w] = 0;
     }
 }
 
@@ -346,14 +347,14 @@ static void compress_tile(orc_format *f, const uint16_t *A, int64_t row0, int64_
 }
 
 /* CR1 over panels [p0, p1) of A (M x K fp16 bits, row-major).
- *   P    : panel rows (1..128)                         (R-Q5, R-Q6)
+ *   P    : panel rows (1..256)                         (R-Q5, R-Q6)
  *   mode : 0 = SPTC (paper: evicted columns re-queued)
  *          1 = DENSE (evicted columns -> dense residual tail; R-Q12)
  * Returns an opaque format or NULL. */
 void *orc_reorder_range(const uint16_t *A, int64_t M, int64_t K, int P, int mode,
                         int p0, int p1)
 {
-    if (!A || M <= 0 || K <= 0 || P < 1 || P > 128 || (mode != 0 && mode != 1)) return NULL;
+    if (!A || M <= 0 || K <= 0 || P < 1 || P > 256 || (mode != 0 && mode != 1)) return NULL;
     int npan = (int)((M + P - 1) / P);
     if (p0 < 0 || p1 > npan || p0 > p1) return NULL;
     orc_format *f = calloc(1, sizeof(orc_format));
@@ -361,7 +362,7 @@ void *orc_reorder_range(const uint16_t *A, int64_t M, int64_t K, int P, int mode
     f->M = M; f->K = K; f->P = P; f->mode = mode; f->npanels = p1 - p0;
     f->T = calloc((size_t)(p1 - p0) + 1, sizeof(int64_t));
     f->D = calloc((size_t)(p1 - p0) + 1, sizeof(int64_t));
-    mask128 *cm = malloc((size_t)K * sizeof(mask128));
+    mask256 *cm = malloc((size_t)K * sizeof(mask256));
     int32_t *queue = malloc((size_t)(K + 16) * 2 * sizeof(int32_t) + 64);
     int32_t *resid = malloc((size_t)(K + 16) * sizeof(int32_t) + 64);
     if (!f->T || !f->D || !cm || !queue || !resid) { free(cm); free(queue); free(resid); return NULL; }
@@ -372,7 +373,7 @@ void *orc_reorder_range(const uint16_t *A, int64_t M, int64_t K, int P, int mode
          * the columns with any nonzero, in ascending order (R-Q4, Fig. 6). */
         int64_t head = 0, tail = 0;
         for (int64_t c = 0; c < K; ++c) {
-            mask128 m = {{0, 0}};
+            mask256 m = {{0, 0, 0, 0}};
             for (int r = 0; r < P; ++r)
                 if (nz16(a_at(A, M, K, row0 + r, (int32_t)c))) m.w[r / 64] |= 1ull << (r % 64);
             cm[c] = m;
@@ -383,11 +384,11 @@ void *orc_reorder_range(const uint16_t *A, int64_t M, int64_t K, int P, int mode
         /* MMA_TILE granularity: pop up to 16 columns per tile. */
         while (head < tail) {
             int32_t cols[16];
-            uint64_t mk[32];
+            uint64_t mk[16 * MASK_WORDS];
             for (int j = 0; j < 16; ++j) {
                 cols[j] = head < tail ? queue[head++] : ORC_PAD;
-                mask128 m = cols[j] == ORC_PAD ? (mask128){{0, 0}} : cm[cols[j]];
-                mk[2 * j] = m.w[0]; mk[2 * j + 1] = m.w[1];
+                mask256 m = cols[j] == ORC_PAD ? (mask256){{0, 0, 0, 0}} : cm[cols[j]];
+                for (int w = 0; w < MASK_WORDS; ++w) mk[MASK_WORDS * j + w] = m.w[w];
             }
             uint8_t perm[16]; int32_t ev[16]; int nev = 0;
             if (orc_tile_reorder(mk, 16, 4, 2, cols, perm, ev, &nev)) return NULL;

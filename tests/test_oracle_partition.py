@@ -56,7 +56,7 @@ def test_partition_matches_exhaustive_enumeration(partitions):
     rng = np.random.default_rng(2024)
     n_ok = n_fail = 0
     for trial in range(40):
-        P = int(rng.choice([1, 3, 8, 16, 40, 64, 128]))
+        P = int(rng.choice([1, 3, 8, 16, 40, 64, 128, 200, 256]))
         dens = float(rng.uniform(0.1, 0.6))
         m = [int(sum(1 << r for r in range(P) if rng.random() < dens)) for _ in range(16)]
         m = [x if x else 1 << int(rng.integers(P)) for x in m]      # real columns are nonzero

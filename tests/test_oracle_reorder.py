@@ -90,6 +90,8 @@ def test_already_24_needs_no_reorder(seed):
     (128, 192, 8, 0.50, 128, "uniform", 1),
     (96, 100, 4, 0.95, 32, "uniform", 0),        # K not a multiple of 16
     (64, 64, 1, 0.0, 64, "uniform", 0),          # fully dense
+    (512, 384, 8, 0.90, 256, "uniform", 0),      # 256-row panels (CTA-pair option, R-Q6)
+    (600, 256, 4, 0.80, 256, "uniform", 1),      # 256-row panels, ragged, DENSE mode
 ])
 def test_format_valid_and_bounded(M, K, v, s, P, kind, mode):
     A = synth.vector_sparse(M, K, v, s, 17, kind=kind)
