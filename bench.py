@@ -238,6 +238,8 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--workload", default="c2")
+    ap.add_argument("--panel-rows", type=int, default=128, choices=[128, 256],
+                    help="reorder panel height: 128 (one CTA per panel) or 256 (CTA pairs)")
     ap.add_argument("--impl", default="jigsaw", choices=["jigsaw", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-cublas", action="store_true")
@@ -279,7 +281,7 @@ def main():
         N = n1 - n0
         mats.append((A, B))
         a_t = torch.from_numpy(A.view(np.int16)).to(dev).view(torch.float16)
-        h = jig.reorder(a_t, v)
+        h = jig.reorder(a_t, v, panel_rows=args.panel_rows)
         info = h.info()
         reorder_ms += info["reorder_ms"]
         hs.append(h)
@@ -458,7 +460,7 @@ def main():
     # e2e_full: host A -> reorder -> host B -> SpMM -> host C (all §8(a) rows)
     t0 = time.perf_counter()
     for (A, B), (M, K, v, s, N) in zip(mats, points):
-        hh = jig.reorder_host(A, v)
+        hh = jig.reorder_host(A, v, panel_rows=args.panel_rows)
         hh.spmm_host(B)
         hh.free()
     full_s = time.perf_counter() - t0
@@ -475,7 +477,7 @@ def main():
         "config": {"workload": desc, "matrices_on_rank0": len(points),
                    "flops": "dense-equivalent 2*M*N*K per matrix",
                    "l2": "flushed (256 MB write) before every timed step", "launch": "step = jigsaw_spmm_batched over the batch (one grouped k_spmm launch per 64 matrices), captured in a CUDA graph",
-                   "seeds": f"synth.SEED_BASE + 1000*rank + index", "format": "P=128, SPTC residual"},
+                   "seeds": f"synth.SEED_BASE + 1000*rank + index", "format": f"P={args.panel_rows}, SPTC residual"},
         "roofline": roof,
         "cpu_baseline": cpu,
         "e2e": {"value": total_eff / e2e_s / 1e12, "unit": "TFLOP/s",

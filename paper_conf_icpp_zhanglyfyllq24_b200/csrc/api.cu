@@ -82,9 +82,9 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
   if (!(v == 1 || v == 2 || v == 4 || v == 8)) return set_status(JIGSAW_ERROR_INVALID_VALUE, "v must be 1, 2, 4 or 8");
   if (M % v) return set_status(JIGSAW_ERROR_INVALID_VALUE, "M must be a multiple of v");
   if (opt) {
-    if (opt->panel_rows != kPanelRows)
+    if (opt->panel_rows != kPanelRows && opt->panel_rows != kPairPanelRows)
       return set_status(opt->panel_rows == 64 ? JIGSAW_ERROR_UNSUPPORTED : JIGSAW_ERROR_INVALID_VALUE,
-                        "panel_rows must be 128 (64 is not built in this version)");
+                        "panel_rows must be 128 or 256 (64 is not built in this version)");
     if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC && opt->residual_mode != JIGSAW_RESIDUAL_DENSE)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
     for (int i = 0; i < 6; ++i)
@@ -129,7 +129,7 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
   jigsaw_handle_s* h = new (std::nothrow) jigsaw_handle_s();
   if (!h) return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "host allocation failed");
   set_status(JIGSAW_SUCCESS);
-  s = build_format(static_cast<const uint16_t*>(A), M, K, v, kPanelRows,
+  s = build_format(static_cast<const uint16_t*>(A), M, K, v, opt ? opt->panel_rows : kPanelRows,
                    opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC, reinterpret_cast<cudaStream_t>(stream),
                    &h->f);
   if (s != JIGSAW_SUCCESS) {
@@ -292,8 +292,8 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
   if (e != cudaSuccess) return cuda_status(e, "export copy");
   if ((nt && (out->gather || out->vals || out->meta)) || (f.ndtiles && (out->rcol || out->dvals))) {
     // read back the device layout and invert it
-    std::vector<uint8_t> A((size_t)f.nksteps * kKStepBytesA);
-    std::vector<uint32_t> E((size_t)f.nkblocks * 512);
+    std::vector<uint8_t> A((size_t)f.planeA() * f.halves());
+    std::vector<uint32_t> E((size_t)f.planeE() / 4 * f.halves());
     std::vector<int32_t> G((size_t)f.nksteps * 32);
     e = cudaMemcpy(A.data(), f.d_Aimg, A.size(), cudaMemcpyDeviceToHost);
     if (e == cudaSuccess) e = cudaMemcpy(E.data(), f.d_Eimg, E.size() * 4, cudaMemcpyDeviceToHost);
@@ -313,7 +313,9 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
           for (int r = 0; r < P; ++r)
             for (int h2 = 0; h2 < 2; ++h2)
               memcpy(out->dvals + (dt * P + r) * 16 + 8 * h2,
-                     &A[gks * kKStepBytesA + (r >> 3) * 256 + h2 * 128 + (r & 7) * 16], 16);
+                     &A[(r >> 7) * f.planeA() + gks * kKStepBytesA + ((r & 127) >> 3) * 256 + h2 * 128 +
+                        (r & 7) * 16],
+                     16);
       }
       for (int t = 0; t < f.T[p]; ++t) {
         const int64_t ft = f.tile_off[p] + t;
@@ -327,12 +329,14 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
             out->gather[ft * 16 + j] = g >= f.K ? kPad : g;
           }
         for (int r = 0; r < P; ++r) {
+          const int half = r >> 7, rr = r & 127;
           if (out->vals)
-            memcpy(out->vals + (ft * P + r) * 8, &A[gks * kKStepBytesA + (r >> 3) * 256 + h2 * 128 + (r & 7) * 16], 16);
+            memcpy(out->vals + (ft * P + r) * 8,
+                   &A[half * f.planeA() + gks * kKStepBytesA + (rr >> 3) * 256 + h2 * 128 + (rr & 7) * 16], 16);
           if (out->meta) {
-            const int m2 = r >> 4, m0 = r & 7, hi = (r >> 3) & 1;
+            const int m2 = rr >> 4, m0 = rr & 7, hi = (rr >> 3) & 1;
             const int L = m0 + 8 * h2 + 16 * m2;
-            const uint32_t w = E[(kb * 128 + L) * 4 + col];
+            const uint32_t w = E[half * (f.planeE() / 4) + (kb * 128 + L) * 4 + col];
             out->meta[ft * P + r] = (uint16_t)(hi ? (w >> 16) : (w & 0xFFFF));
           }
         }

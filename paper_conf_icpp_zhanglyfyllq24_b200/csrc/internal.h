@@ -13,8 +13,9 @@
 namespace jig {
 
 constexpr int kTileCols = 16;     // logical columns per tile (the paper's MMA_TILE width)
-constexpr int kPanelRows = 128;   // P = tcgen05 M (R-Q5)
-constexpr int kKStepBytesA = 4096;  // 128 rows x 16 halves (compressed 32 logical) per k-step
+constexpr int kPanelRows = 128;   // P = tcgen05 M of one CTA (R-Q5); the default panel height
+constexpr int kPairPanelRows = 256;  // P = tcgen05 M of a CTA pair (cta_group::2, R-Q6)
+constexpr int kKStepBytesA = 4096;  // 128 rows x 16 halves (compressed 32 logical) per k-step and half
 constexpr int kStepsPerBlock = 4;   // k-steps per E block (tcgen05.cp 128x128b = 4 TMEM columns)
 constexpr int kEBlockBytes = 2048;  // 128 lanes x 16 B
 constexpr int kPad = -1;
@@ -35,9 +36,14 @@ struct Format {
   uint8_t* d_kind = nullptr;    // [ntiles]
   uint8_t* d_nevict = nullptr;  // [ntiles]
   // device layout consumed by the SpMM kernel
-  uint8_t* d_Aimg = nullptr;  // [nksteps][4096]: UMMA K-major no-swizzle core matrices
-  uint8_t* d_Eimg = nullptr;  // [nkblocks][128][4] u32: TMEM metadata lanes
+  // A and E are stored as P/128 planes, one per 128-row half of every panel (the
+  // CTA of a pair that owns those rows), each plane contiguous per k-block.
+  uint8_t* d_Aimg = nullptr;  // [halves][nksteps][4096]: UMMA K-major no-swizzle core matrices
+  uint8_t* d_Eimg = nullptr;  // [halves][nkblocks][128][4] u32: TMEM metadata lanes
   int32_t* d_G = nullptr;     // [nksteps][32]: B row per logical column (PAD -> K, TMA zero fill)
+  int halves() const { return P / kPanelRows; }
+  int64_t planeA() const { return nksteps * (int64_t)kKStepBytesA; }
+  int64_t planeE() const { return nkblocks * (int64_t)kEBlockBytes; }
   // stats
   int64_t nnz = 0, kp_total = 0, evictions = 0, overflow_tiles = 0, max_tiles = 0;
   int64_t device_bytes = 0;

@@ -49,12 +49,34 @@ jigsaw_status_t init_tables(int dev) {
   return JIGSAW_SUCCESS;
 }
 
+// Row mask of one column inside a panel of up to 256 rows (row r = bit r%32 of word r/32).
+struct RowMask {
+  uint4 lo, hi;
+};
+__device__ __forceinline__ RowMask zero_mask() { return RowMask{make_uint4(0, 0, 0, 0), make_uint4(0, 0, 0, 0)}; }
+// bits set where >= 3 of the 4 masks are set (the Alg. 1 compatibility test)
+__device__ __forceinline__ uint32_t three_of_four(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  return (a & b & (c | d)) | (c & d & (a | b));
+}
+__device__ __forceinline__ uint32_t any_three_of_four(const RowMask& a, const RowMask& b, const RowMask& c,
+                                                      const RowMask& d) {
+  return three_of_four(a.lo.x, b.lo.x, c.lo.x, d.lo.x) | three_of_four(a.lo.y, b.lo.y, c.lo.y, d.lo.y) |
+         three_of_four(a.lo.z, b.lo.z, c.lo.z, d.lo.z) | three_of_four(a.lo.w, b.lo.w, c.lo.w, d.lo.w) |
+         three_of_four(a.hi.x, b.hi.x, c.hi.x, d.hi.x) | three_of_four(a.hi.y, b.hi.y, c.hi.y, d.hi.y) |
+         three_of_four(a.hi.z, b.hi.z, c.hi.z, d.hi.z) | three_of_four(a.hi.w, b.hi.w, c.hi.w, d.hi.w);
+}
+__device__ __forceinline__ uint32_t all_three(const RowMask& a, const RowMask& b, const RowMask& c) {
+  return (a.lo.x & b.lo.x & c.lo.x) | (a.lo.y & b.lo.y & c.lo.y) | (a.lo.z & b.lo.z & c.lo.z) |
+         (a.lo.w & b.lo.w & c.lo.w) | (a.hi.x & b.hi.x & c.hi.x) | (a.hi.y & b.hi.y & c.hi.y) |
+         (a.hi.z & b.hi.z & c.hi.z) | (a.hi.w & b.hi.w & c.hi.w);
+}
+
 // ------------------------------------------------------------------ R1
 __global__ void k_colmask(const uint16_t* __restrict__ A, int64_t M, int64_t K, int P,
-                          uint4* __restrict__ masks, unsigned long long* __restrict__ nnz) {
+                          RowMask* __restrict__ masks, unsigned long long* __restrict__ nnz) {
   const int p = blockIdx.y;
   const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  uint32_t w[4] = {0, 0, 0, 0};
+  uint32_t w[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   int cnt = 0;
   if (c < K) {
     const int64_t row0 = (int64_t)p * P;
@@ -67,14 +89,14 @@ __global__ void k_colmask(const uint16_t* __restrict__ A, int64_t M, int64_t K, 
         ++cnt;
       }
     }
-    masks[(int64_t)p * K + c] = make_uint4(w[0], w[1], w[2], w[3]);
+    masks[(int64_t)p * K + c] = RowMask{make_uint4(w[0], w[1], w[2], w[3]), make_uint4(w[4], w[5], w[6], w[7])};
   }
   for (int o = 16; o; o >>= 1) cnt += __shfl_xor_sync(kFull, cnt, o);
   if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(nnz, (unsigned long long)cnt);
 }
 
 // ------------------------------------------------------------------ R2
-__global__ void k_compact(const uint4* __restrict__ masks, int64_t K, int32_t* __restrict__ S,
+__global__ void k_compact(const RowMask* __restrict__ masks, int64_t K, int32_t* __restrict__ S,
                           int32_t* __restrict__ Kp) {
   __shared__ int wsum[32];
   __shared__ int total;
@@ -85,8 +107,8 @@ __global__ void k_compact(const uint4* __restrict__ masks, int64_t K, int32_t* _
     const int64_t c = c0 + tid;
     bool flag = false;
     if (c < K) {
-      const uint4 m = masks[(int64_t)p * K + c];
-      flag = (m.x | m.y | m.z | m.w) != 0;
+      const RowMask m = masks[(int64_t)p * K + c];
+      flag = (m.lo.x | m.lo.y | m.lo.z | m.lo.w | m.hi.x | m.hi.y | m.hi.z | m.hi.w) != 0;
     }
     const unsigned b = __ballot_sync(kFull, flag);
     const int lpre = __popc(b & ((1u << lane) - 1u));
@@ -116,7 +138,7 @@ struct TileSmem {
   uint32_t bitmap[2048];  // compat[S] for every 4-subset S, indexed by the 16-bit slot mask
   uint16_t big[kMaxBig];  // compatible 3- and 4-subsets of the real slots (existence test)
   int nbig;
-  uint4 m[16];            // row masks per slot (PAD: 0)
+  RowMask m[16];          // row masks per slot (PAD: 0)
   int32_t cols[16];       // column per slot (kPad = -1)
   int32_t ev[16];         // evicted columns, in eviction order
   uint8_t perm[16];
@@ -189,15 +211,14 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
     }
   }
   if (lane < 16 && ((realset >> lane) & 1u)) {              // 3 real columns, min slot = lane
-    const uint4 ma = s.m[lane];
+    const RowMask ma = s.m[lane];
     for (uint32_t x = realset & ~((2u << lane) - 1u); x; x &= x - 1) {
       const int b = __ffs(x) - 1;
-      const uint4 mb = s.m[b];
+      const RowMask mb = s.m[b];
       for (uint32_t y = x & (x - 1); y; y &= y - 1) {
         const int c = __ffs(y) - 1;
-        const uint4 mc = s.m[c];
-        const uint32_t all3 = (ma.x & mb.x & mc.x) | (ma.y & mb.y & mc.y) | (ma.z & mb.z & mc.z) |
-                              (ma.w & mb.w & mc.w);
+        const RowMask mc = s.m[c];
+        const uint32_t all3 = all_three(ma, mb, mc);
         if (!all3) {
           const int i = atomicAdd(&s.nbig, 1);
           if (i < kMaxBig) s.big[i] = (uint16_t)((1u << lane) | (1u << b) | (1u << c));
@@ -260,11 +281,7 @@ __device__ void tile_search(TileSmem& s, int lane) {
         const int b = __ffs(r) - 1; r &= r - 1;
         const int c = __ffs(r) - 1; r &= r - 1;
         const int d = __ffs(r) - 1;
-        const uint4 ma = s.m[a], mb = s.m[b], mc = s.m[c], md = s.m[d];
-        const uint32_t bad = ((ma.x & mb.x & (mc.x | md.x)) | (mc.x & md.x & (ma.x | mb.x))) |
-                             ((ma.y & mb.y & (mc.y | md.y)) | (mc.y & md.y & (ma.y | mb.y))) |
-                             ((ma.z & mb.z & (mc.z | md.z)) | (mc.z & md.z & (ma.z | mb.z))) |
-                             ((ma.w & mb.w & (mc.w | md.w)) | (mc.w & md.w & (ma.w | mb.w)));
+        const uint32_t bad = any_three_of_four(s.m[a], s.m[b], s.m[c], s.m[d]);
         ok = bad == 0;
         if (ok) {
           atomicOr(&s.bitmap[sub >> 5], 1u << (sub & 31));
@@ -297,7 +314,7 @@ __device__ void tile_search(TileSmem& s, int lane) {
             if (!((realset >> j) & 1u)) continue;
             s.ev[s.nev++] = s.cols[j];
             s.cols[j] = kPad;
-            s.m[j] = make_uint4(0, 0, 0, 0);
+            s.m[j] = zero_mask();
             --need;
           }
         }
@@ -345,7 +362,7 @@ __device__ void tile_search(TileSmem& s, int lane) {
     if (lane == 0) {
       s.ev[s.nev++] = s.cols[e];
       s.cols[e] = kPad;
-      s.m[e] = make_uint4(0, 0, 0, 0);
+      s.m[e] = zero_mask();
     }
     realset &= ~(1u << e);
     __syncwarp();
@@ -372,7 +389,7 @@ __device__ void store_tile(const TileSmem& s, const Scratch& sc, int p, int t, i
 
 // ------------------------------------------------------------------ R3
 constexpr int kR3Warps = 4;
-__global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const uint4* __restrict__ masks,
+__global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const RowMask* __restrict__ masks,
                                                               const int32_t* __restrict__ S,
                                                               const int32_t* __restrict__ Kp,
                                                               int64_t K, Scratch sc) {
@@ -397,7 +414,7 @@ __global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const uint4* __res
 // DENSE mode: only the partial last tile of S_p is built here, and the
 // evicted columns of all tiles, in tile and eviction order, form the residual
 // list R_p (left at the front of the panel's queue buffer, count in nres[p]).
-__global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks,
+__global__ void __launch_bounds__(32) k_overflow(const RowMask* __restrict__ masks,
                                                  const int32_t* __restrict__ S,
                                                  const int32_t* __restrict__ Kp, int64_t K,
                                                  Scratch sc, int32_t* __restrict__ queue,
@@ -414,7 +431,7 @@ __global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks
       if (lane < 16) {
         const int32_t c = lane < rem ? S[(int64_t)p * K + 16 * nfull + lane] : kPad;
         s.cols[lane] = c;
-        s.m[lane] = c == kPad ? make_uint4(0, 0, 0, 0) : masks[(int64_t)p * K + c];
+        s.m[lane] = c == kPad ? zero_mask() : masks[(int64_t)p * K + c];
       }
       __syncwarp();
       tile_search(s, lane);
@@ -454,7 +471,7 @@ __global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks
     if (lane < 16) {
       const int32_t c = head + lane < tail ? q[head + lane] : kPad;
       s.cols[lane] = c;
-      s.m[lane] = c == kPad ? make_uint4(0, 0, 0, 0) : masks[(int64_t)p * K + c];
+      s.m[lane] = c == kPad ? zero_mask() : masks[(int64_t)p * K + c];
     }
     head = min(head + 16, tail);
     __syncwarp();
@@ -472,24 +489,26 @@ __global__ void __launch_bounds__(32) k_overflow(const uint4* __restrict__ masks
 }
 
 // ------------------------------------------------------------------ R5
-// One CTA (128 threads = rows) per (panel, k-step): compresses the two tiles of
-// the k-step (R-Q15, R-Q16) and writes
+// One CTA (P threads = rows) per (panel, k-step): compresses the two tiles of
+// the k-step (R-Q15, R-Q16) and writes, per 128-row half of the
+// panel (P = 256 -> two halves, one per CTA of the pair), into that half's plane
 //   A image : 4096 B = [row group 16][tile 2][row 8][8 halves]  (UMMA K-major,
 //             no swizzle: LBO = 128 B between the two tiles, SBO = 256 B)
 //   E lanes : TMEM metadata layout of tcgen05.mma.sp kind::f16 -- lane
 //             L = m0 + 8*h + 16*m2 holds rows r = 16*m2 + m0 and r + 8 of tile half h
-//   G rows  : B row per logical column, PAD -> K (TMA zero fill)
-__global__ void __launch_bounds__(128) k_emit(const uint16_t* __restrict__ A, int64_t M, int64_t K,
+//   G rows  : B row per logical column, PAD -> K (TMA zero fill); one list per k-step
+__global__ void __launch_bounds__(256) k_emit(const uint16_t* __restrict__ A, int64_t M, int64_t K, int P,
                                               Scratch sc, const int32_t* __restrict__ T,
                                               const int32_t* __restrict__ tile_off,
                                               const int32_t* __restrict__ ksoff,
                                               const int32_t* __restrict__ kboff,
-                                              uint8_t* __restrict__ Aimg, uint32_t* __restrict__ Eimg,
+                                              uint8_t* __restrict__ Aimg, int64_t planeA,
+                                              uint32_t* __restrict__ Eimg, int64_t planeE,
                                               int32_t* __restrict__ G, int32_t* __restrict__ colidx,
                                               uint8_t* __restrict__ perm, uint8_t* __restrict__ kind,
                                               uint8_t* __restrict__ nevict, const int32_t* __restrict__ Kp) {
   __shared__ int32_t gat[2][16];
-  __shared__ uint16_t smeta[2][128];
+  __shared__ uint16_t smeta[2][256];
   const int p = blockIdx.y, ks = blockIdx.x, tid = threadIdx.x;
   const int Tp = T[p];
   const int nks = (Tp + 1) / 2;
@@ -513,8 +532,9 @@ __global__ void __launch_bounds__(128) k_emit(const uint16_t* __restrict__ A, in
     G[gks * 32 + tid] = g == kPad ? (int32_t)K : g;
   }
   __syncthreads();
-  const int r = tid;
-  const int64_t row = (int64_t)p * 128 + r;
+  const int r = tid, half = r >> 7, rr = r & 127;
+  const int64_t row = (int64_t)p * P + r;
+  uint8_t* Ah = Aimg + half * planeA + gks * kKStepBytesA;
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
     uint16_t v[8];
@@ -551,15 +571,15 @@ __global__ void __launch_bounds__(128) k_emit(const uint16_t* __restrict__ A, in
     pk.y = v[2] | ((uint32_t)v[3] << 16);
     pk.z = v[4] | ((uint32_t)v[5] << 16);
     pk.w = v[6] | ((uint32_t)v[7] << 16);
-    *reinterpret_cast<uint4*>(Aimg + gks * kKStepBytesA + (r >> 3) * 256 + h * 128 + (r & 7) * 16) = pk;
+    *reinterpret_cast<uint4*>(Ah + (rr >> 3) * 256 + h * 128 + (rr & 7) * 16) = pk;
     smeta[h][r] = meta;
   }
   __syncthreads();
   {
-    const int L = tid, m0 = L & 7, h = (L >> 3) & 1, m2 = L >> 4;
-    const int rr = 16 * m2 + m0;
-    const uint32_t w = (uint32_t)smeta[h][rr] | ((uint32_t)smeta[h][rr + 8] << 16);
-    Eimg[((int64_t)(kboff[p] + ks / kStepsPerBlock) * 128 + L) * 4 + (ks % kStepsPerBlock)] = w;
+    const int L = tid & 127, m0 = L & 7, h = (L >> 3) & 1, m2 = L >> 4;
+    const int r0 = half * 128 + 16 * m2 + m0;
+    const uint32_t w = (uint32_t)smeta[h][r0] | ((uint32_t)smeta[h][r0 + 8] << 16);
+    Eimg[half * planeE + ((int64_t)(kboff[p] + ks / kStepsPerBlock) * 128 + L) * 4 + (ks % kStepsPerBlock)] = w;
   }
 }
 
@@ -567,11 +587,12 @@ __global__ void __launch_bounds__(128) k_emit(const uint16_t* __restrict__ A, in
 // columns R_p[16j .. 16j+16) as an uncompressed K = 16 A image in the same UMMA
 // K-major no-swizzle layout ([row group 16][8-column half 2][row 8][8 halves]);
 // its gather list is the 16 columns (PAD -> K) followed by 16 PAD rows.
-__global__ void __launch_bounds__(128) k_emit_dense(const uint16_t* __restrict__ A, int64_t M, int64_t K,
+__global__ void __launch_bounds__(256) k_emit_dense(const uint16_t* __restrict__ A, int64_t M, int64_t K, int P,
                                                     const int32_t* __restrict__ queue, int64_t qcap,
                                                     const int32_t* __restrict__ nres,
                                                     const int4* __restrict__ pin,
-                                                    uint8_t* __restrict__ Aimg, int32_t* __restrict__ G) {
+                                                    uint8_t* __restrict__ Aimg, int64_t planeA,
+                                                    int32_t* __restrict__ G) {
   __shared__ int32_t cols[16];
   const int p = blockIdx.y, j = blockIdx.x, tid = threadIdx.x;
   const int4 pi = pin[p];
@@ -585,8 +606,9 @@ __global__ void __launch_bounds__(128) k_emit_dense(const uint16_t* __restrict__
     G[gks * 32 + tid] = c == kPad ? (int32_t)K : c;
   }
   __syncthreads();
-  const int r = tid;
-  const int64_t row = (int64_t)p * 128 + r;
+  const int r = tid, rr = r & 127;
+  const int64_t row = (int64_t)p * P + r;
+  uint8_t* Ah = Aimg + (r >> 7) * planeA + gks * kKStepBytesA;
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
     uint16_t v[8];
@@ -601,7 +623,7 @@ __global__ void __launch_bounds__(128) k_emit_dense(const uint16_t* __restrict__
     pk.y = v[2] | ((uint32_t)v[3] << 16);
     pk.z = v[4] | ((uint32_t)v[5] << 16);
     pk.w = v[6] | ((uint32_t)v[7] << 16);
-    *reinterpret_cast<uint4*>(Aimg + gks * kKStepBytesA + (r >> 3) * 256 + h * 128 + (r & 7) * 16) = pk;
+    *reinterpret_cast<uint4*>(Ah + (rr >> 3) * 256 + h * 128 + (rr & 7) * 16) = pk;
   }
 }
 
@@ -645,7 +667,7 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   const int npan = (int)((M + P - 1) / P);
   const int cap = (int)(K / 8 + 2);
   const int64_t qcap = 2 * K + 64;
-  uint4* masks = nullptr;
+  RowMask* masks = nullptr;
   int32_t *S = nullptr, *Kp = nullptr, *T = nullptr, *queue = nullptr, *tile_off = nullptr;
   int32_t *d_ksoff = nullptr, *d_kboff = nullptr, *nres = nullptr;
   int* err = nullptr;
@@ -662,7 +684,7 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   f->npanels = npan;
   if ((st = init_tables(dev)) != JIGSAW_SUCCESS) return st;
 
-  JIG_TRY(dalloc(&masks, sizeof(uint4) * npan * K, scratch));
+  JIG_TRY(dalloc(&masks, sizeof(RowMask) * npan * K, scratch));
   JIG_TRY(dalloc(&S, sizeof(int32_t) * npan * K, scratch));
   JIG_TRY(dalloc(&Kp, sizeof(int32_t) * npan, scratch));
   JIG_TRY(dalloc(&T, sizeof(int32_t) * npan, scratch));
@@ -740,20 +762,22 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
     JIG_TRY(dalloc(&f->d_perm, (size_t)16 * f->ntiles, f->allocs));
     JIG_TRY(dalloc(&f->d_kind, (size_t)f->ntiles, f->allocs));
     JIG_TRY(dalloc(&f->d_nevict, (size_t)f->ntiles, f->allocs));
-    JIG_TRY(dalloc(&f->d_Aimg, (size_t)kKStepBytesA * f->nksteps, f->allocs));
-    JIG_TRY(dalloc(&f->d_Eimg, (size_t)kEBlockBytes * f->nkblocks, f->allocs));
+    JIG_TRY(dalloc(&f->d_Aimg, (size_t)kKStepBytesA * f->nksteps * f->halves(), f->allocs));
+    JIG_TRY(dalloc(&f->d_Eimg, (size_t)kEBlockBytes * f->nkblocks * f->halves(), f->allocs));
     JIG_TRY(dalloc(&f->d_G, sizeof(int32_t) * 32 * f->nksteps, f->allocs));
     JIG_CU(cudaMemcpyAsync(f->d_pin, f->pin.data(), sizeof(int4) * npan, cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(d_ksoff, f->ks_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(d_kboff, f->kb_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(tile_off, f->tile_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
-    JIG_CU(cudaMemsetAsync(f->d_Eimg, 0, (size_t)kEBlockBytes * f->nkblocks, stream), "memset E");
+    JIG_CU(cudaMemsetAsync(f->d_Eimg, 0, (size_t)kEBlockBytes * f->nkblocks * f->halves(), stream), "memset E");
     if (maxks > 0)
-      k_emit<<<dim3(maxks, npan), 128, 0, stream>>>(dA, M, K, sc, T, tile_off, d_ksoff, d_kboff,
-                                                  f->d_Aimg, reinterpret_cast<uint32_t*>(f->d_Eimg), f->d_G,
-                                                  f->d_colidx, f->d_perm, f->d_kind, f->d_nevict, Kp);
+      k_emit<<<dim3(maxks, npan), P, 0, stream>>>(dA, M, K, P, sc, T, tile_off, d_ksoff, d_kboff, f->d_Aimg,
+                                                f->planeA(), reinterpret_cast<uint32_t*>(f->d_Eimg),
+                                                f->planeE() / 4, f->d_G, f->d_colidx, f->d_perm, f->d_kind,
+                                                f->d_nevict, Kp);
     if (maxdk > 0)
-      k_emit_dense<<<dim3(maxdk, npan), 128, 0, stream>>>(dA, M, K, queue, qcap, nres, f->d_pin, f->d_Aimg, f->d_G);
+      k_emit_dense<<<dim3(maxdk, npan), P, 0, stream>>>(dA, M, K, P, queue, qcap, nres, f->d_pin, f->d_Aimg,
+                                                      f->planeA(), f->d_G);
     JIG_CU(cudaGetLastError(), "k_emit launch");
     JIG_CU(cudaEventRecord(ev1, stream), "cudaEventRecord");
     // total evictions = sum of per-tile counts
@@ -770,7 +794,8 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
     f->reorder_ms = ms;
   }
   f->device_bytes = 0;
-  f->device_bytes += (int64_t)f->nksteps * (kKStepBytesA + 128) + (int64_t)f->nkblocks * kEBlockBytes +
+  f->device_bytes += (int64_t)f->nksteps * (kKStepBytesA * f->halves() + 128) +
+                     (int64_t)f->nkblocks * kEBlockBytes * f->halves() +
                      (int64_t)f->ntiles * (16 * 4 + 16 + 2) + (int64_t)npan * 12;
   for (void* p : scratch) cudaFree(p);
   cudaEventDestroy(ev0);

@@ -44,11 +44,15 @@ constexpr int kStageA = kStepsPerBlock * kKStepBytesA;  // 16 KB
 constexpr int kStageE = kEBlockBytes;               // 2 KB
 constexpr int kStageG = kRowsPerBlock * 4;          // gather list of a k-block: 512 B
 
-template <int NT, bool kSplit>
+// NT = the MMA's N (C columns per work unit).  kPair: a cluster of two CTAs runs
+// one 256-row panel with tcgen05 cta_group::2 (M = 256); each CTA stages NT/2 of
+// the B columns and holds its 128 rows x NT accumulator.
+template <int NT, bool kSplit, bool kPair = false>
 struct Cfg {
-  static constexpr int kChunks = NT / 64;
+  static constexpr int kNTL = kPair ? NT / 2 : NT;  // B columns staged by this CTA
+  static constexpr int kChunks = kNTL / 64;
   static constexpr int kStageB = kChunks * kChunkB;
-  static constexpr int kStages = NT == 256 ? 2 : NT == 128 ? 4 : 5;
+  static constexpr int kStages = kPair ? (NT == 256 ? 4 : 6) : NT == 256 ? 2 : NT == 128 ? 4 : 5;
   static constexpr int kAccCols = NT;
   static constexpr int kAccBufs = NT == 256 ? 1 : 2;   // TMEM: 512 columns total
   static constexpr int kEColBase = kAccBufs * NT;
@@ -69,6 +73,7 @@ struct Problem {
   const __half* B;
   __half* C;
   int64_t M, N, K;
+  int64_t planeA, planeE;  // bytes between the A / E planes of the two 128-row halves (P = 256)
   int npanels;
   int unit0;  // first global work unit of this problem
   int pin0;   // offset of this problem's panels in ParamsT::pin (if use_pin)
@@ -130,6 +135,7 @@ struct Work {
   int64_t M, N, K;
   int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
   int64_t ks0, kb0;  // first k-step / E block of the panel
+  int64_t row0;      // first C row written by this CTA
   // k-block kb of the panel: the first nkb_s are 2:4 sparse (4 k-steps of 32
   // logical columns each, metadata block kb0 + kb); the rest (DENSE residual mode)
   // hold up to 4 dense K = 16 steps each, stored after the sparse k-steps.
@@ -142,7 +148,9 @@ struct Work {
 };
 // `hint` = problem index of this thread's previous unit: units are visited in
 // increasing order, so the scan is amortised O(1) instead of O(problems).
-template <int NT, class Prm>
+// kPair: `rank` selects this CTA's 128-row half of the 256-row panel (its A / E
+// plane); otherwise it selects the CTA's k-block share of a split-K cluster of S.
+template <int NT, bool kPair, class Prm>
 __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank, int S, int& hint) {
   int i, lu;
   if (Prm::kMaxUnits > 1 && prm.use_ulist) {  // host-ordered schedule (longest units first, snake)
@@ -176,8 +184,17 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.ndk = pi.w;
   w.nkb_s = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
   const int nkb = w.nkb_s + (w.ndk + kStepsPerBlock - 1) / kStepsPerBlock;
-  w.kb_lo = (int)(rank * nkb / S);
-  w.kb_hi = (int)((rank + 1) * nkb / S);
+  if constexpr (kPair) {
+    w.Aimg += rank * prm.pr[i].planeA;
+    w.Eimg += rank * prm.pr[i].planeE;
+    w.row0 = (int64_t)w.p * kPairPanelRows + rank * kPanelRows;
+    w.kb_lo = 0;
+    w.kb_hi = nkb;
+  } else {
+    w.row0 = (int64_t)w.p * kPanelRows;
+    w.kb_lo = (int)(rank * nkb / S);
+    w.kb_hi = (int)((rank + 1) * nkb / S);
+  }
   return w;
 }
 
@@ -211,9 +228,10 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
-template <int NT, bool kSplit, class Prm>
+template <int NT, bool kSplit, bool kPair, class Prm>
 __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
-  using C_ = Cfg<NT, kSplit>;
+  static_assert(!(kSplit && kPair), "split-K and CTA pairs are separate variants");
+  using C_ = Cfg<NT, kSplit, kPair>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sB = smem;                                   // kStages x kStageB (1024-aligned)
@@ -229,14 +247,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint64_t* recv_full = tempty + 2;
   uint64_t* rfull = recv_full + 1;   // unit ring (dynamic scheduler)
   uint64_t* rempty = rfull + kSD;
-  volatile int* ring = reinterpret_cast<volatile int*>(rempty + kSD);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rempty + kSD) + kSD;
+  uint64_t* pfull = rempty + kSD;    // kPair, even CTA: the odd CTA's stage has landed
+  volatile int* ring = reinterpret_cast<volatile int*>(pfull + C_::kStages);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pfull + C_::kStages) + kSD;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = kSplit ? prm.S : 1;
-  const uint32_t rank = kSplit ? cluster_ctarank() : 0;
-  const int cluster_id = blockIdx.x / S, nclusters = gridDim.x / S;
-  const bool dyn = !kSplit && prm.sched >= 0;
+  const int CS = kPair ? 2 : S;  // CTAs per cluster
+  const uint32_t rank = (kSplit || kPair) ? cluster_ctarank() : 0;
+  const int cluster_id = blockIdx.x / CS, nclusters = gridDim.x / CS;
+  const bool dyn = !kSplit && !kPair && prm.sched >= 0;
   if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
     g_trace[blockIdx.x * kTraceSlots + 15] = gtimer();
     g_trace[blockIdx.x * kTraceSlots + 14] = smid();
@@ -248,10 +268,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       mbar_init(&full[s], 1 + 32 * kBProdWarps);  // A/E expect_tx arrival + B-producer cp.async arrivals
       mbar_init(&empty[s], 1);
       mbar_init(&gfull[s], 1);
+      mbar_init(&pfull[s], 1);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&tfull[a], 1);
-      mbar_init(&tempty[a], 4);
+      mbar_init(&tempty[a], kPair ? 8 : 4);  // epilogue warps (of both CTAs of a pair)
     }
     mbar_init(recv_full, 1);
     for (int i = 0; i < kSD; ++i) {
@@ -260,8 +281,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     }
     fence_barrier_init();
   }
-  if (warp == 1) tmem_alloc<C_::kTmemCols>(tmem_slot);
-  if constexpr (kSplit) {
+  if (warp == 1) {
+    if constexpr (kPair)
+      tmem_alloc_pair<C_::kTmemCols>(tmem_slot);
+    else
+      tmem_alloc<C_::kTmemCols>(tmem_slot);
+  }
+  if constexpr (kSplit || kPair) {
     cluster_sync_all();  // peers' barriers are initialised before any st.async targets them
   } else {
     __syncthreads();
@@ -286,7 +312,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         }
         if (u < 0) break;
         un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : u + nclusters;  // latency hidden by the loads below
-        const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
         const int64_t kb0 = wk.kb0;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           const int steps = wk.steps(kb);
@@ -320,7 +346,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     // come from the stage's gather list in shared memory (TMA-loaded by warp 0).
     const int w = (warp - kBProdWarp0) >> 1;   // k-step within the k-block
     const int half = (warp - kBProdWarp0) & 1;  // rows [16*half, 16*half + 16) of it
-    constexpr int LPR = NT / 8;            // lanes per B row (16-byte chunks per row)
+    constexpr int LPR = C_::kNTL / 8;      // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
     int stage = 0, hint = 0, traced = 0, rslot = 0;
@@ -328,8 +354,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     for (int us = cluster_id;; us += nclusters) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
-      const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
-      const int col = wk.n0 + 8 * c;
+      const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+      const int col = wk.n0 + (kPair ? (int)rank * C_::kNTL : 0) + 8 * c;
       const bool colok = col < wk.N;
       const __half* Bp = wk.B;
       const int64_t ldb = wk.N, K = wk.K;
@@ -358,35 +384,65 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
       }
     }
+  } else if (warp == 1 && kPair && rank != 0) {
+    // ------------------------------------------------------------ pair relay (odd CTA)
+    // The even CTA issues the pair's MMAs; it may read this CTA's stage only once
+    // this CTA's A/E bulk copies and B cp.async have landed: relay full -> pfull.
+    if (lane == 0) {
+      int stage = 0, hint = 0;
+      uint32_t phase = 0;
+      const uint32_t rpfull = mapa_shared(smem_u32(pfull), 0);
+      for (int us = cluster_id; us < prm.nunits; us += nclusters) {
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
+        for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
+          mbar_wait(&full[stage], phase);
+          fence_proxy_async();
+          mbar_arrive_cluster(rpfull + 8 * stage);
+          if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+    __syncwarp();
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {
-      const uint32_t idesc0 = idesc_f16(128, NT, 0, 1, 1, 0);
-      const uint32_t idesc1 = idesc_f16(128, NT, 0, 1, 1, 1);
-      const uint32_t idesc_dense = idesc_f16(128, NT, 0, 1, 0, 0);
+      constexpr int MM = kPair ? 256 : 128;
+      const uint32_t idesc0 = idesc_f16(MM, NT, 0, 1, 1, 0);
+      const uint32_t idesc1 = idesc_f16(MM, NT, 0, 1, 1, 1);
+      const uint32_t idesc_dense = idesc_f16(MM, NT, 0, 1, 0, 0);
       int stage = 0, hint = 0, nkb_mma = 0, rslot = 0;
       uint32_t phase = 0, rph = 0;
       int it = 0;
       for (int us = cluster_id;; us += nclusters) {
         const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, false, 0) : (us < prm.nunits ? us : -1);
         if (u < 0) break;
-        const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
         const int a = it % C_::kAccBufs;
         const uint32_t use = (uint32_t)(it / C_::kAccBufs);
-        mbar_wait(&tempty[a], (use & 1) ^ 1);
+        if (kPair)
+          mbar_wait_cluster(&tempty[a], (use & 1) ^ 1);
+        else
+          mbar_wait(&tempty[a], (use & 1) ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tbase + a * C_::kAccCols;
         for (int kb = kb_lo; kb < kb_hi; ++kb) {
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
           mbar_wait(&full[stage], phase);
+          if (kPair) mbar_wait_cluster(&pfull[stage], phase);
           tc_fence_after();
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
           const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
-          if (!dense) tc_cp_128x128b(e_tmem, smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0));
+          if (!dense) {
+            const uint64_t edesc = smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0);
+            if constexpr (kPair)
+              tc_cp_128x128b_pair(e_tmem, edesc);
+            else
+              tc_cp_128x128b(e_tmem, edesc);
+          }
           JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
@@ -394,18 +450,31 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
             const uint64_t bdesc = smem_desc(b_base + s * 32 * 128, kChunkB, 1024, 2);
             const uint32_t acc = (kb != kb_lo) || (s != 0);
-            if (dense)   // residual tile on the dense tensor path, K = 16
-              tc_mma_f16(d_tmem, adesc, bdesc, idesc_dense, acc);
-            else
-              tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+            if constexpr (kPair) {
+              if (dense)
+                tc_mma_f16_pair(d_tmem, adesc, bdesc, idesc_dense, acc);
+              else
+                tc_mma_sp_f16_pair(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+            } else {
+              if (dense)   // residual tile on the dense tensor path, K = 16
+                tc_mma_f16(d_tmem, adesc, bdesc, idesc_dense, acc);
+              else
+                tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+            }
           }
           JIG_TRACE_KB(5, nkb_mma);
-          tc_commit(&empty[stage]);
+          if constexpr (kPair)
+            tc_commit_pair(&empty[stage]);   // frees the stage in both CTAs
+          else
+            tc_commit(&empty[stage]);
           JIG_TRACE_KB(3, nkb_mma);
           ++nkb_mma;
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
-        tc_commit(&tfull[a]);
+        if constexpr (kPair)
+          tc_commit_pair(&tfull[a]);
+        else
+          tc_commit(&tfull[a]);
         JIG_TRACE(5);
         ++it;
       }
@@ -419,7 +488,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     for (int us = cluster_id;; us += nclusters) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
-      const Work wk = decode_unit<NT, Prm>(prm, u, rank, S, hint);
+      const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
       const int p = wk.p, n0 = wk.n0;
       const int64_t M = wk.M, N = wk.N;
       __half* const Cm = wk.C;
@@ -432,7 +501,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       }
       if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
       if constexpr (!kSplit) {
-        const int64_t row = (int64_t)p * 128 + r;
+        const int64_t row = wk.row0 + r;
         __half* crow = Cm + row * N + n0;
 #pragma unroll 1
         for (int c0 = 0; c0 < NT; c0 += 32) {
@@ -511,19 +580,29 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       if (has_acc) {
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&tempty[a]);
+        if (lane == 0) {
+          if (kPair && rank != 0)
+            mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[a]), 0));  // the pair's issuer
+          else
+            mbar_arrive(&tempty[a]);
+        }
         ++it;
       }
     }
   }
   if (threadIdx.x == 0) JIG_TRACE(10);
   tc_fence_before();
-  if constexpr (kSplit) {
+  if constexpr (kSplit || kPair) {
     cluster_sync_all();  // no CTA leaves while peers may still target its shared memory
   } else {
     __syncthreads();
   }
-  if (warp == 1) tmem_dealloc<C_::kTmemCols>(tbase);
+  if (warp == 1) {
+    if constexpr (kPair)
+      tmem_dealloc_pair<C_::kTmemCols>(tbase);
+    else
+      tmem_dealloc<C_::kTmemCols>(tbase);
+  }
   if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
     JIG_TRACE(11);
     g_trace[blockIdx.x * kTraceSlots + 13] = gtimer();
@@ -531,12 +610,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 }
 
 int g_num_sms[64] = {0};
-bool g_attr_set[64][8] = {};  // [device][variant]
+bool g_attr_set[64][16] = {};  // [device][variant]
 
-template <int NT, bool kSplit, class Prm>
+template <int NT, bool kSplit, bool kPair, class Prm>
 jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
-  using C_ = Cfg<NT, kSplit>;
-  auto kern = k_spmm<NT, kSplit, Prm>;
+  using C_ = Cfg<NT, kSplit, kPair>;
+  auto kern = k_spmm<NT, kSplit, kPair, Prm>;
   if (dev >= 0 && dev < 64 && !g_attr_set[dev][vid]) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::kSmem);
     if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(k_spmm)");
@@ -553,7 +632,7 @@ jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = kSplit ? S : 1;
+  attr[0].val.clusterDim.x = kPair ? 2 : kSplit ? S : 1;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
@@ -575,8 +654,18 @@ int spmm_num_sms() {
 
 // Tile / split selection: enough units for every SM -> NT = 128,
 // persistent; otherwise NT = 64 and, when the panels carry enough k-blocks,
-// split-K over a cluster of S = 2/4/8 CTAs.
+// split-K over a cluster of S = 2/4/8 CTAs.  256-row panels (CTA pairs): NT = 256
+// when there is a unit for every pair, else NT = 128; grid = 2 x pairs.
 void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* grid) {
+  if (f.P == kPairPanelRows) {
+    const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
+    const int64_t u256 = f.npanels * ((N + 255) / 256);
+    *NT = ((u256 >= sms / 2 && force != 128) || force == 256) ? 256 : 128;
+    *S = 1;
+    const int64_t units = f.npanels * ((N + *NT - 1) / *NT);
+    *grid = 2 * (int)std::min<int64_t>(units, sms / 2);
+    return;
+  }
   const int64_t u256 = f.npanels * ((N + 255) / 256), u128 = f.npanels * ((N + 127) / 128);
   const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
   int64_t kbs = 0;
@@ -616,6 +705,8 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
     prm.use_pin = 0;
   P.Aimg = f.d_Aimg;
   P.Eimg = f.d_Eimg;
+  P.planeA = f.planeA();
+  P.planeE = f.planeE();
   P.G = f.d_G;
   P.pin = f.d_pin;
   P.B = reinterpret_cast<const __half*>(dB);
@@ -631,11 +722,11 @@ int g_trace_ctas = 0;
 int g_sched_next[64] = {0};
 
 template <class Prm>
-static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, cudaStream_t s) {
+static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, bool pair, cudaStream_t s) {
   prm.S = S;
   // persistent launches use the dynamic scheduler on a rotating counter slot
   prm.sched = -1;
-  if (S == 1 && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
+  if (S == 1 && !pair && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
     prm.sched = (g_sched_next[dev]++) % kSchedSlots;
   const char* tr = getenv("JIGSAW_TRACE");
   prm.trace = (tr && tr[0] == '1') ? 1 : 0;
@@ -646,11 +737,16 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
     u += (int)(prm.pr[i].npanels * ((prm.pr[i].N + NT - 1) / NT));
   }
   prm.nunits = u;
-  constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 4;
-  if (NT == 256) return launch_variant<256, false>(prm, grid, 1, dev, vb + 3, s);
-  if (NT == 128) return launch_variant<128, false>(prm, grid, 1, dev, vb + 0, s);
-  if (S == 1) return launch_variant<64, false>(prm, grid, 1, dev, vb + 1, s);
-  if constexpr (std::is_same<Prm, ParamsOne>::value) return launch_variant<64, true>(prm, grid, S, dev, vb + 2, s);
+  constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 8;
+  if (pair) {
+    if (NT == 256) return launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s);
+    return launch_variant<128, false, true>(prm, grid, 2, dev, vb + 4, s);
+  }
+  if (NT == 256) return launch_variant<256, false, false>(prm, grid, 1, dev, vb + 3, s);
+  if (NT == 128) return launch_variant<128, false, false>(prm, grid, 1, dev, vb + 0, s);
+  if (S == 1) return launch_variant<64, false, false>(prm, grid, 1, dev, vb + 1, s);
+  if constexpr (std::is_same<Prm, ParamsOne>::value)
+    return launch_variant<64, true, false>(prm, grid, S, dev, vb + 2, s);
   return set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
 }
 
@@ -662,7 +758,8 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   fill_problem(prm, 0, f, dB, N, dC);
   int NT = 128, S = 1, grid = 1;
   choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
-  if (const char* e = getenv("JIGSAW_FORCE_SPLIT")) {  // test hook: force NT = 64 with split S
+  const bool pair = f.P == kPairPanelRows;
+  if (const char* e = pair ? nullptr : getenv("JIGSAW_FORCE_SPLIT")) {  // test hook: force NT = 64 with split S
     const int fs = atoi(e);
     if (fs == 1 || fs == 2 || fs == 4 || fs == 8) {
       NT = 64;
@@ -671,15 +768,18 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
       grid = S > 1 ? (int)(u64 * S) : (int)std::min<int64_t>(u64, spmm_num_sms());
     }
   }
-  return launch_params(prm, NT, S, grid, f.device, s);
+  return launch_params(prm, NT, S, grid, f.device, pair, s);
 }
 
 // Grouped launch: many independent products in ONE persistent kernel (units of
 // all problems are dealt round-robin to the CTAs), up to kMaxProblems per launch.
-jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
+// Products with 128-row and 256-row panels go to separate launches (one CTA vs
+// one CTA pair per unit).
+static jigsaw_status_t launch_group(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
                                     void* const* Cs, int count, cudaStream_t s) {
   thread_local ParamsGroup prm;
   const int sms = spmm_num_sms();
+  const bool pair = count > 0 && fs[0]->P == kPairPanelRows;
   for (int i0 = 0; i0 < count; i0 += kMaxProblems) {
     const int n = std::min(kMaxProblems, count - i0);
     prm.nprob = n;
@@ -698,14 +798,20 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
       npan += f.npanels;
     }
     const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
-    int NT = u128 >= 2 * sms ? 128 : 64;
-    if ((u256 >= sms && kbs >= 24 * npan && force == 0) || force == 256) NT = 256;
-    if (force == 128 || force == 64) NT = force;
+    int NT;
+    if (pair) {
+      NT = ((u256 >= sms / 2 && force != 128) || force == 256) ? 256 : 128;
+    } else {
+      NT = u128 >= 2 * sms ? 128 : 64;
+      if ((u256 >= sms && kbs >= 24 * npan && force == 0) || force == 256) NT = 256;
+      if (force == 128 || force == 64) NT = force;
+    }
     const int64_t units = NT == 256 ? u256 : NT == 128 ? u128 : u64;
-    const int grid = (int)std::min<int64_t>(units, sms);
+    const int slots = (int)std::min<int64_t>(units, pair ? sms / 2 : sms);  // CTAs or CTA pairs
+    const int grid = pair ? 2 * slots : slots;
     // Static schedule: units sorted by cost (k-blocks of their panel), longest
-    // first, dealt to the persistent CTAs in snake order (CTA c takes slots
-    // c, c + grid, ...), so the per-CTA loads even out (LPT-like).
+    // first, dealt to the persistent CTAs (pairs) in snake order (slot c takes
+    // schedule positions c, c + slots, ...), so the per-CTA loads even out (LPT-like).
     prm.use_ulist = 0;
     if (units <= ParamsGroup::kMaxUnits) {
       thread_local std::vector<std::pair<int, uint32_t>> order;
@@ -722,14 +828,38 @@ jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* 
       std::stable_sort(order.begin(), order.end(),
                        [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
       for (size_t k = 0; k < order.size(); ++k) {
-        const int r = (int)(k / grid), c = (int)(k % grid);
-        const int mr = (int)std::min<int64_t>(grid, (int64_t)order.size() - (int64_t)r * grid);
-        const int slot = r * grid + ((r & 1) ? mr - 1 - c : c);
+        const int r = (int)(k / slots), c = (int)(k % slots);
+        const int mr = (int)std::min<int64_t>(slots, (int64_t)order.size() - (int64_t)r * slots);
+        const int slot = r * slots + ((r & 1) ? mr - 1 - c : c);
         prm.ulist[slot] = order[k].second;
       }
       prm.use_ulist = 1;
     }
-    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, s);
+    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, pair, s);
+    if (st != JIGSAW_SUCCESS) return st;
+  }
+  return JIGSAW_SUCCESS;
+}
+
+jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
+                                    void* const* Cs, int count, cudaStream_t s) {
+  bool mixed = false;
+  for (int i = 1; i < count; ++i) mixed |= fs[i]->P != fs[0]->P;
+  if (!mixed) return launch_group(fs, Bs, Ns, Cs, count, s);
+  for (int P : {kPanelRows, kPairPanelRows}) {
+    std::vector<const Format*> f2;
+    std::vector<const void*> b2;
+    std::vector<int64_t> n2;
+    std::vector<void*> c2;
+    for (int i = 0; i < count; ++i)
+      if (fs[i]->P == P) {
+        f2.push_back(fs[i]);
+        b2.push_back(Bs[i]);
+        n2.push_back(Ns[i]);
+        c2.push_back(Cs[i]);
+      }
+    if (f2.empty()) continue;
+    jigsaw_status_t st = launch_group(f2.data(), b2.data(), n2.data(), c2.data(), (int)f2.size(), s);
     if (st != JIGSAW_SUCCESS) return st;
   }
   return JIGSAW_SUCCESS;

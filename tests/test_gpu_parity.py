@@ -179,6 +179,12 @@ def test_abi_errors_on_gpu():
     assert st == 1                            # misaligned B
     with pytest.raises(jig.JigsawError):
         jig.reorder(_dev(synth.vector_sparse(8, 8, 1, 0.5, 1)), 3)
+    with pytest.raises(jig.JigsawError) as e:
+        jig.reorder(_dev(A), 4, panel_rows=64)  # declared, not built
+    assert e.value.status == 2
+    with pytest.raises(jig.JigsawError) as e:
+        jig.reorder(_dev(A), 4, panel_rows=100)
+    assert e.value.status == 1
 
 
 # ---------------------------------------------------------------- full sizes
@@ -323,3 +329,85 @@ def test_tile_width_variants(nt, monkeypatch):
     torch.cuda.synchronize()
     for a, b, c in zip(mats, Bs, dC):
         spmm_check(_host(c), a, b)
+
+
+# ---------------------------------------------------------------- 256-row panels
+PAIR_CASES = [
+    # M, K, v, s, N, kind, seed, mode
+    (512, 384, 8, 0.90, 256, "uniform", 21, 0),
+    (600, 300, 4, 0.80, 136, "uniform", 22, 0),     # ragged M (last panel 88 rows), ragged K / N
+    (256, 512, 8, 0.50, 128, "uniform", 23, 0),     # residual-heavy
+    (1024, 2048, 2, 0.70, 512, "skewed", 24, 0),
+    (600, 256, 4, 0.80, 200, "uniform", 25, 1),     # DENSE residual mode
+    (130, 64, 2, 0.0, 64, "uniform", 26, 0),        # one dense panel with 2 rows in its 2nd half
+]
+
+
+@pytest.mark.parametrize("M,K,v,s,N,kind,seed,mode", PAIR_CASES)
+@pytest.mark.parametrize("nt", ["128", "256"])
+def test_pair_panels_bit_exact_and_spmm(M, K, v, s, N, kind, seed, mode, nt, monkeypatch):
+    """panel_rows = 256 (R-Q6): one CTA pair per panel (tcgen05 cta_group::2, M = 256).
+    Format bit-exact vs oracle O2 at P = 256 (incl. the two per-half planes the
+    kernel reads), C within tolerance for N tiles of 128 and 256, integers bit-exact."""
+    monkeypatch.setenv("JIGSAW_FORCE_NT", nt)
+    A = synth.vector_sparse(M, K, v, s, seed, kind=kind)
+    B = synth.dense_b(K, N, seed)
+    h = jig.reorder(_dev(A), v, panel_rows=256, residual_mode=mode)
+    g = h.export()
+    ref = oracle.reorder(A, P=256, mode=mode)
+    assert_format_equal(g, ref)
+    if mode == 1:
+        assert np.array_equal(g["D"], ref.D)
+        assert np.array_equal(g["rcol"], ref.rcol)
+        assert np.array_equal(g["dvals"], ref.dvals)
+    check.check_format(A, 256, g["T"], g["gather"], g["vals"], g["meta"], perm=g["perm"],
+                       D=g["D"] if mode == 1 else None, rcol=g["rcol"] if mode == 1 else None,
+                       dvals=g["dvals"] if mode == 1 else None)
+    info = h.info()
+    assert info["panel_rows"] == 256
+    assert info["format_bytes"] == check.format_bytes(ref.T, 256, ref.D if mode == 1 else None)
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    spmm_check(C, A, B)
+    h.free()
+    Ai = synth.vector_sparse(M, K, v, s, seed + 50, kind="int")
+    Bi = synth.dense_b(K, N, seed + 50, kind="int")
+    hi = jig.reorder(_dev(Ai), v, panel_rows=256, residual_mode=mode)
+    Ci = _host(hi.spmm(_dev(Bi)))
+    torch.cuda.synchronize()
+    C_ref, _ = oracle.spmm(Ai, Bi)
+    if np.abs(C_ref).max() <= 2048:
+        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+
+
+def test_pair_panels_grouped_mixed_with_single():
+    """A batch mixing 128-row and 256-row panel formats (two grouped launches),
+    including an all-zero matrix, against the oracle."""
+    mats, Bs, hs = [], [], []
+    for i in range(12):
+        M, K = [(512, 300), (256, 640), (384, 128)][i % 3]
+        v = [2, 4, 8][i % 3]
+        A = synth.vector_sparse(M, K, v, 0.85, 300 + i) if i != 5 else np.zeros((M, K), np.uint16)
+        mats.append(A)
+        Bs.append(synth.dense_b(K, 192, 400 + i))
+        hs.append(jig.reorder(_dev(A), v, panel_rows=256 if i % 2 else 128))
+    dB = [_dev(b) for b in Bs]
+    dC = [torch.full((a.shape[0], 192), 3.0, dtype=torch.float16, device="cuda") for a in mats]
+    jig.spmm_batched(hs, dB, dC)
+    torch.cuda.synchronize()
+    for a, b, c in zip(mats, Bs, dC):
+        spmm_check(_host(c), a, b)
+
+
+def test_pair_panels_full_size_sampled():
+    """BASELINE C4-sized product with 256-row panels, sampled rows of both halves."""
+    M, K, N, v, s = 4096, 4096, 4096, 8, 0.9
+    A = synth.vector_sparse(M, K, v, s, 31)
+    B = synth.dense_b(K, N, 31)
+    h = jig.reorder(_dev(A), v, panel_rows=256)
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    rows = np.array([0, 127, 128, 255, 256 * 7 + 5, 256 * 7 + 200, M - 129, M - 1])
+    spmm_check(C, A, B, rows=rows)
+    ref = oracle.reorder(A, P=256, panels=(7, 8))
+    assert_format_equal(h.export(), ref, panels=(7, 8))
