@@ -59,8 +59,9 @@ struct Cfg {
   static constexpr uint32_t kTmemCols = kAccBufs * NT + 4 * kStages <= 256 ? 256 : 512;
   static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
   static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
+  static constexpr int kStageC = 4 * 32 * 64;  // epilogue: per warp 32 rows x 32 fp16 columns
   static constexpr size_t kSmem =
-      1024 + (size_t)kStages * (kStageB + kStageA + kStageE + kStageG) + kRecvBytes + 512;
+      1024 + (size_t)kStages * (kStageB + kStageA + kStageE + kStageG) + kRecvBytes + kStageC + 512;
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
@@ -89,7 +90,13 @@ struct ParamsT {
   static constexpr int kMaxUnits = MAXU;
   Problem pr[MAXP];
   int4 pin[MAXPIN];
-  uint32_t ulist[MAXU];  // grouped launches: schedule slot -> (problem << 26) | local unit
+  // grouped launches: schedule position -> work piece, packed as
+  //   problem (6 bits) | local unit (11) | piece (3) | pieces - 1 (3) | partial slot (9)
+  // a unit split into `pieces` k-ranges (split-K inside the persistent launch)
+  // reduces its fp32 partials through `ws` (slots pslot .. pslot + pieces - 1)
+  uint32_t ulist[MAXU];
+  float* ws;        // partial tiles: [slot][rank][NT / 32][128][32] fp32
+  int* wcnt;        // per split unit and CTA rank: pieces finished (reset by the last)
   int nprob, nunits, S, use_pin, use_ulist;
   int sched;  // >= 0: dynamic tile scheduler on counter slot `sched`; -1: static round-robin
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
@@ -134,6 +141,8 @@ struct Work {
   __half* C;
   int64_t M, N, K;
   int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
+  int piece, npieces, pslot;  // split-K piece of a grouped launch (npieces = 1: whole unit)
+  bool valid;                 // false: padding entry of a static per-slot schedule
   int64_t ks0, kb0;  // first k-step / E block of the panel
   int64_t row0;      // first C row written by this CTA
   // k-block kb of the panel: the first nkb_s are 2:4 sparse (4 k-steps of 32
@@ -146,17 +155,27 @@ struct Work {
   }
   __device__ __forceinline__ int64_t gks(int kb) const { return ks0 + (int64_t)kb * kStepsPerBlock; }
 };
+constexpr uint32_t kNoWork = 0xFFFFFFFFu;  // schedule padding
 // `hint` = problem index of this thread's previous unit: units are visited in
 // increasing order, so the scan is amortised O(1) instead of O(problems).
 // kPair: `rank` selects this CTA's 128-row half of the 256-row panel (its A / E
 // plane); otherwise it selects the CTA's k-block share of a split-K cluster of S.
 template <int NT, bool kPair, class Prm>
 __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank, int S, int& hint) {
-  int i, lu;
-  if (Prm::kMaxUnits > 1 && prm.use_ulist) {  // host-ordered schedule (longest units first, snake)
+  int i, lu, piece = 0, npieces = 1, pslot = 0;
+  Work w;
+  w.valid = true;
+  if (Prm::kMaxUnits > 1 && prm.use_ulist) {  // host-ordered schedule (longest pieces first)
     const uint32_t code = prm.ulist[u];
+    if (code == kNoWork) {
+      w.valid = false;
+      return w;
+    }
     i = (int)(code >> 26);
-    lu = (int)(code & ((1u << 26) - 1));
+    lu = (int)((code >> 15) & 0x7FFu);
+    piece = (int)((code >> 12) & 7u);
+    npieces = (int)((code >> 9) & 7u) + 1;
+    pslot = (int)(code & 0x1FFu);
   } else {
     i = hint;
     if (prm.pr[i].unit0 > u) i = 0;
@@ -164,7 +183,6 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
     hint = i;
     lu = u - prm.pr[i].unit0;
   }
-  Work w;
   w.Aimg = prm.pr[i].Aimg;
   w.Eimg = prm.pr[i].Eimg;
   w.G = prm.pr[i].G;
@@ -184,12 +202,19 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.ndk = pi.w;
   w.nkb_s = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
   const int nkb = w.nkb_s + (w.ndk + kStepsPerBlock - 1) / kStepsPerBlock;
+  w.piece = piece;
+  w.npieces = npieces;
+  w.pslot = pslot;
   if constexpr (kPair) {
     w.Aimg += rank * prm.pr[i].planeA;
     w.Eimg += rank * prm.pr[i].planeE;
     w.row0 = (int64_t)w.p * kPairPanelRows + rank * kPanelRows;
-    w.kb_lo = 0;
-    w.kb_hi = nkb;
+    w.kb_lo = piece * nkb / npieces;
+    w.kb_hi = (piece + 1) * nkb / npieces;
+  } else if (npieces > 1) {
+    w.row0 = (int64_t)w.p * kPanelRows;
+    w.kb_lo = piece * nkb / npieces;
+    w.kb_hi = (piece + 1) * nkb / npieces;
   } else {
     w.row0 = (int64_t)w.p * kPanelRows;
     w.kb_lo = (int)(rank * nkb / S);
@@ -239,7 +264,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint8_t* sE = sA + C_::kStages * kStageA;             // kStages x 2 KB
   int32_t* sG = reinterpret_cast<int32_t*>(sE + C_::kStages * kStageE);  // kStages x 128 gather rows
   uint8_t* sRecv = reinterpret_cast<uint8_t*>(sG) + C_::kStages * kStageG;  // split-K receive buffer
-  uint64_t* full = reinterpret_cast<uint64_t*>(sRecv + C_::kRecvBytes);
+  uint8_t* sC = sRecv + C_::kRecvBytes;                                       // epilogue staging
+  uint64_t* full = reinterpret_cast<uint64_t*>(sC + C_::kStageC);
   uint64_t* empty = full + C_::kStages;
   uint64_t* gfull = empty + C_::kStages;  // gather list of the stage has landed
   uint64_t* tfull = gfull + C_::kStages;
@@ -250,6 +276,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint64_t* pfull = rempty + kSD;    // kPair, even CTA: the odd CTA's stage has landed
   volatile int* ring = reinterpret_cast<volatile int*>(pfull + C_::kStages);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pfull + C_::kStages) + kSD;
+  volatile int* s_last = reinterpret_cast<volatile int*>(tmem_slot + 1);  // split piece: this CTA reduces
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = kSplit ? prm.S : 1;
@@ -313,6 +340,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         if (u < 0) break;
         un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : u + nclusters;  // latency hidden by the loads below
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+        if (!wk.valid) continue;
         const int64_t kb0 = wk.kb0;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           const int steps = wk.steps(kb);
@@ -355,6 +383,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
       const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+      if (!wk.valid) continue;
       const int col = wk.n0 + (kPair ? (int)rank * C_::kNTL : 0) + 8 * c;
       const bool colok = col < wk.N;
       const __half* Bp = wk.B;
@@ -394,6 +423,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const uint32_t rpfull = mapa_shared(smem_u32(pfull), 0);
       for (int us = cluster_id; us < prm.nunits; us += nclusters) {
         const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
+        if (!wk.valid) continue;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           mbar_wait(&full[stage], phase);
           fence_proxy_async();
@@ -413,10 +443,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       int stage = 0, hint = 0, nkb_mma = 0, rslot = 0;
       uint32_t phase = 0, rph = 0;
       int it = 0;
+      long long wait_cycles = 0;
       for (int us = cluster_id;; us += nclusters) {
         const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, false, 0) : (us < prm.nunits ? us : -1);
         if (u < 0) break;
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+        if (!wk.valid) continue;
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
         const int a = it % C_::kAccBufs;
@@ -430,8 +462,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         for (int kb = kb_lo; kb < kb_hi; ++kb) {
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
+          const long long tw0 = prm.trace ? clock64() : 0;
           mbar_wait(&full[stage], phase);
           if (kPair) mbar_wait_cluster(&pfull[stage], phase);
+          if (prm.trace) wait_cycles += clock64() - tw0;
           tc_fence_after();
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
@@ -478,6 +512,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         JIG_TRACE(5);
         ++it;
       }
+      if (!kSplit && prm.trace && blockIdx.x < kTraceCTAs) {  // slots 7/8 are split-K-only otherwise
+        g_trace[blockIdx.x * kTraceSlots + 7] = wait_cycles;  // MMA issuer: cycles waiting for data
+        g_trace[blockIdx.x * kTraceSlots + 8] = nkb_mma;      // k-blocks issued
+      }
     }
     __syncwarp();
   } else {
@@ -489,6 +527,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
       const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+      if (!wk.valid) continue;
       const int p = wk.p, n0 = wk.n0;
       const int64_t M = wk.M, N = wk.N;
       __half* const Cm = wk.C;
@@ -501,10 +540,45 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       }
       if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
       if constexpr (!kSplit) {
-        const int64_t row = wk.row0 + r;
-        __half* crow = Cm + row * N + n0;
+        uint8_t* stg = sC + q * (32 * 64);
+        bool write_c = true;
+        const int npc = wk.npieces;
+        if (npc > 1) {
+          // split-K piece: publish the fp32 partial tile, count the pieces done;
+          // the last piece of the unit adds the others' partials to its own and
+          // writes C (the last-arriver reduction never waits on another CTA)
+          constexpr size_t kTile = (size_t)128 * NT;  // floats per partial tile
+          float* part = prm.ws + ((size_t)(wk.pslot + wk.piece) * CS + rank) * kTile;
 #pragma unroll 1
-        for (int c0 = 0; c0 < NT; c0 += 32) {
+          for (int c0 = 0; c0 < NT; c0 += 32) {
+            uint32_t v[32];
+            if (has_acc) {
+              tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * C_::kAccCols + c0, v);
+              tc_wait_ld();
+            } else {
+#pragma unroll
+              for (int j = 0; j < 32; ++j) v[j] = 0;
+            }
+            float4* dst = reinterpret_cast<float4*>(part + ((size_t)(c0 / 32) * 128 + r) * 32);
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              __stcg(dst + j, make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
+                                         __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
+          }
+          __threadfence();
+          asm volatile("bar.sync 1, 128;" ::: "memory");
+          if (threadIdx.x == 64) {
+            int* cnt = prm.wcnt + wk.pslot * CS + rank;
+            const int done = atomicAdd(cnt, 1);
+            *s_last = done == npc - 1;
+            if (done == npc - 1) atomicExch(cnt, 0);  // ready for the next launch
+          }
+          asm volatile("bar.sync 1, 128;" ::: "memory");
+          write_c = *s_last != 0;
+          if (write_c) __threadfence();
+        }
+#pragma unroll 1
+        for (int c0 = 0; write_c && c0 < NT; c0 += 32) {
           uint32_t v[32];
           if (has_acc) {
             tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * C_::kAccCols + c0, v);
@@ -513,19 +587,44 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 #pragma unroll
             for (int j = 0; j < 32; ++j) v[j] = 0;     // all-zero panel (R-Q21)
           }
-          if (row < M) {
+          if (npc > 1) {
+            constexpr size_t kTile = (size_t)128 * NT;
+            for (int pc = 0; pc < npc; ++pc) {
+              if (pc == wk.piece) continue;
+              const float4* src = reinterpret_cast<const float4*>(
+                  prm.ws + ((size_t)(wk.pslot + pc) * CS + rank) * kTile + ((size_t)(c0 / 32) * 128 + r) * 32);
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              if (n0 + c0 + 8 * j < N) {
-                uint4 pk;
-                pk.x = pack_h2(__uint_as_float(v[8 * j + 0]), __uint_as_float(v[8 * j + 1]));
-                pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
-                pk.z = pack_h2(__uint_as_float(v[8 * j + 4]), __uint_as_float(v[8 * j + 5]));
-                pk.w = pack_h2(__uint_as_float(v[8 * j + 6]), __uint_as_float(v[8 * j + 7]));
-                *reinterpret_cast<uint4*>(crow + c0 + 8 * j) = pk;
+              for (int j = 0; j < 8; ++j) {
+                const float4 x = __ldcg(src + j);
+                v[4 * j] = __float_as_uint(__uint_as_float(v[4 * j]) + x.x);
+                v[4 * j + 1] = __float_as_uint(__uint_as_float(v[4 * j + 1]) + x.y);
+                v[4 * j + 2] = __float_as_uint(__uint_as_float(v[4 * j + 2]) + x.z);
+                v[4 * j + 3] = __float_as_uint(__uint_as_float(v[4 * j + 3]) + x.w);
               }
             }
           }
+          // fp16 (RN), transposed through shared memory so that each store
+          // instruction writes 8 rows x 64 contiguous bytes (4 lanes per row)
+          // instead of 32 rows x 16 bytes; 16-byte chunks swizzled by (row >> 1) & 3
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            uint4 pk;
+            pk.x = pack_h2(__uint_as_float(v[8 * j + 0]), __uint_as_float(v[8 * j + 1]));
+            pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
+            pk.z = pack_h2(__uint_as_float(v[8 * j + 4]), __uint_as_float(v[8 * j + 5]));
+            pk.w = pack_h2(__uint_as_float(v[8 * j + 6]), __uint_as_float(v[8 * j + 7]));
+            *reinterpret_cast<uint4*>(stg + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)) = pk;
+          }
+          __syncwarp();
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const int rr = 8 * i + (lane >> 2), c = lane & 3;
+            const int64_t grow = wk.row0 + q * 32 + rr;
+            const uint4 pk = *reinterpret_cast<const uint4*>(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
+            if (grow < M && n0 + c0 + 8 * c < N)
+              *reinterpret_cast<uint4*>(Cm + grow * N + n0 + c0 + 8 * c) = pk;
+          }
+          __syncwarp();
         }
       } else {
         // reduce-scatter of the fp32 partial tile through DSMEM
@@ -589,6 +688,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         ++it;
       }
     }
+    if (warp == 2 && lane == 0 && prm.trace && blockIdx.x < kTraceCTAs)
+      g_trace[blockIdx.x * kTraceSlots + 12] = it;  // units with an accumulator run by this CTA
   }
   if (threadIdx.x == 0) JIG_TRACE(10);
   tc_fence_before();
@@ -722,7 +823,8 @@ int g_trace_ctas = 0;
 int g_sched_next[64] = {0};
 
 template <class Prm>
-static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, bool pair, cudaStream_t s) {
+static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, bool pair, cudaStream_t s,
+                                     int npieces_total = -1) {
   prm.S = S;
   // persistent launches use the dynamic scheduler on a rotating counter slot
   prm.sched = -1;
@@ -736,7 +838,7 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
     prm.pr[i].unit0 = u;
     u += (int)(prm.pr[i].npanels * ((prm.pr[i].N + NT - 1) / NT));
   }
-  prm.nunits = u;
+  prm.nunits = npieces_total >= 0 ? npieces_total : u;
   constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 8;
   if (pair) {
     if (NT == 256) return launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s);
@@ -753,6 +855,8 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
   thread_local ParamsOne prm;  // host-side scratch for the parameter block
   prm.nprob = 1;
+  prm.ws = nullptr;
+  prm.wcnt = nullptr;
   prm.use_pin = 1;
   prm.use_ulist = 0;
   fill_problem(prm, 0, f, dB, N, dC);
@@ -769,6 +873,49 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
     }
   }
   return launch_params(prm, NT, S, grid, f.device, pair, s);
+}
+
+// Device workspace for the fp32 partial tiles of split units: R regions used
+// round-robin by successive launches (so back-to-back or concurrently replayed
+// launches do not share partials), each region = [counters | partial tiles].
+// Grown outside stream capture only; counters are zeroed once at allocation and
+// reset by the last piece of every unit.
+struct SplitWs {
+  char* base = nullptr;
+  size_t region = 0;
+  int next = 0;
+};
+constexpr int kWsRegions = 4;
+SplitWs g_ws[64];
+
+static bool split_workspace(int dev, size_t tile_bytes, size_t cnt_bytes, cudaStream_t s, float** ws, int** wcnt) {
+  if (dev < 0 || dev >= 64) return false;
+  SplitWs& w = g_ws[dev];
+  const size_t need = ((cnt_bytes + 255) & ~size_t(255)) + tile_bytes;
+  if (need > w.region) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return false;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return false;
+    if (w.base) cudaFree(w.base);
+    w.base = nullptr;
+    w.region = 0;
+    const size_t region = std::max(need, (size_t)8 << 20);
+    if (cudaMalloc(&w.base, region * kWsRegions) != cudaSuccess) {
+      cudaGetLastError();
+      w.base = nullptr;
+      return false;
+    }
+    if (cudaMemset(w.base, 0, region * kWsRegions) != cudaSuccess) {
+      cudaFree(w.base);
+      w.base = nullptr;
+      return false;
+    }
+    w.region = region;
+  }
+  char* r = w.base + (size_t)(w.next++ % kWsRegions) * w.region;
+  *wcnt = reinterpret_cast<int*>(r);
+  *ws = reinterpret_cast<float*>(r + ((cnt_bytes + 255) & ~size_t(255)));
+  return true;
 }
 
 // Grouped launch: many independent products in ONE persistent kernel (units of
@@ -807,35 +954,112 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       if (force == 128 || force == 64) NT = force;
     }
     const int64_t units = NT == 256 ? u256 : NT == 128 ? u128 : u64;
-    const int slots = (int)std::min<int64_t>(units, pair ? sms / 2 : sms);  // CTAs or CTA pairs
-    const int grid = pair ? 2 * slots : slots;
-    // Static schedule: units sorted by cost (k-blocks of their panel), longest
-    // first, dealt to the persistent CTAs (pairs) in snake order (slot c takes
-    // schedule positions c, c + slots, ...), so the per-CTA loads even out (LPT-like).
+    const int slots_max = pair ? sms / 2 : sms;                  // CTAs or CTA pairs
+    int slots = (int)std::min<int64_t>(units, slots_max);
+    // Schedule: units sorted by cost (k-blocks of their panel), longest first;
+    // pair launches deal them to the pairs in snake order (slot c takes positions
+    // c, c + slots, ...), single-CTA launches hand them out through the dynamic
+    // scheduler in this order (LPT-like either way).  A unit much longer than the
+    // per-slot average is split into up to 8 k-range pieces (split-K inside the
+    // persistent launch) so one long panel does not set the makespan.
     prm.use_ulist = 0;
+    prm.ws = nullptr;
+    prm.wcnt = nullptr;
+    int npieces_total = -1;
     if (units <= ParamsGroup::kMaxUnits) {
-      thread_local std::vector<std::pair<int, uint32_t>> order;
-      order.clear();
+      struct U { int cost; int nkb; uint32_t code; };
+      thread_local std::vector<U> us;
+      us.clear();
+      int64_t total = 0;
       for (int i = 0; i < n; ++i) {
         const Format& f = *fs[i0 + i];
         const int ntn = (int)((Ns[i0 + i] + NT - 1) / NT);
         for (int t = 0; t < ntn; ++t)
           for (int p = 0; p < f.npanels; ++p) {
-            const int cost = (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4 + 1;
-            order.push_back({-cost, ((uint32_t)i << 26) | (uint32_t)(t * f.npanels + p)});
+            const int nkb = (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
+            us.push_back({nkb + 1, nkb, ((uint32_t)i << 26) | ((uint32_t)(t * f.npanels + p) << 15)});
+            total += nkb + 1;
           }
+      }
+      const int64_t target = std::max<int64_t>(4, (total + slots_max - 1) / slots_max);
+      const bool allow_split = !getenv("JIGSAW_NO_PIECES");
+      thread_local std::vector<std::pair<int, uint32_t>> order;
+      order.clear();
+      int pslots = 0;
+      std::stable_sort(us.begin(), us.end(), [](const U& a, const U& b) { return a.cost > b.cost; });
+      for (const U& x : us) {
+        int np = 1;
+        if (allow_split && x.cost > target + target / 4 && x.nkb >= 8) {
+          np = (int)std::min<int64_t>({8, (x.cost + target - 1) / target, x.nkb / 4});
+          if (pslots + np > 511 || (int64_t)order.size() + np > ParamsGroup::kMaxUnits) np = 1;
+        }
+        if (np > 1) {
+          for (int pc = 0; pc < np; ++pc)
+            order.push_back({-(x.cost / np), x.code | ((uint32_t)pc << 12) | ((uint32_t)(np - 1) << 9) |
+                                                 (uint32_t)pslots});
+          pslots += np;
+        } else {
+          order.push_back({-x.cost, x.code});
+        }
+      }
+      if (pslots > 0) {
+        const size_t tile = (size_t)128 * NT * sizeof(float) * (pair ? 2 : 1);
+        if (!split_workspace(fs[i0]->device, (size_t)pslots * tile, 2 * 512 * sizeof(int), s, &prm.ws, &prm.wcnt)) {
+          // no workspace (e.g. first use inside a stream capture): run whole units
+          order.clear();
+          for (const U& x : us) order.push_back({-x.cost, x.code});
+          pslots = 0;
+        }
       }
       std::stable_sort(order.begin(), order.end(),
                        [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
-      for (size_t k = 0; k < order.size(); ++k) {
-        const int r = (int)(k / slots), c = (int)(k % slots);
-        const int mr = (int)std::min<int64_t>(slots, (int64_t)order.size() - (int64_t)r * slots);
-        const int slot = r * slots + ((r & 1) ? mr - 1 - c : c);
-        prm.ulist[slot] = order[k].second;
+      const int nslots = (int)std::min<int64_t>(slots_max, (int64_t)order.size());
+      npieces_total = (int)order.size();
+      if (!pair) {
+        for (size_t k = 0; k < order.size(); ++k) prm.ulist[k] = order[k].second;
+      } else {
+        // static schedule: greedy LPT (each piece, longest first, to the least
+        // loaded pair); pair c runs positions c, c + nslots, ... of the list,
+        // padded with kNoWork where its queue is shorter than the longest
+        thread_local std::vector<std::vector<uint32_t>> q;
+        q.assign(nslots, {});
+        std::vector<std::pair<int64_t, int>> heap;  // (load, slot), min-heap
+        for (int c = 0; c < nslots; ++c) heap.push_back({0, c});
+        auto cmp = [](const std::pair<int64_t, int>& a, const std::pair<int64_t, int>& b) { return a > b; };
+        std::make_heap(heap.begin(), heap.end(), cmp);
+        size_t maxlen = 0;
+        for (const auto& o : order) {
+          std::pop_heap(heap.begin(), heap.end(), cmp);
+          auto& h = heap.back();
+          q[h.second].push_back(o.second);
+          h.first += -o.first;
+          maxlen = std::max(maxlen, q[h.second].size());
+          std::push_heap(heap.begin(), heap.end(), cmp);
+        }
+        if (getenv("JIGSAW_DEBUG_SCHED")) {
+          int64_t lo = INT64_MAX, hi = 0;
+          for (const auto& h : heap) lo = std::min(lo, h.first), hi = std::max(hi, h.first);
+          fprintf(stderr, "[jigsaw] pair schedule: %zu pieces (%d split slots) on %d pairs, load min %lld max %lld "
+                  "(target %lld), longest queue %zu\n", order.size(), pslots, nslots, (long long)lo, (long long)hi,
+                  (long long)target, maxlen);
+        }
+        if (maxlen * nslots <= (size_t)ParamsGroup::kMaxUnits) {
+          for (size_t r = 0; r < maxlen; ++r)
+            for (int c = 0; c < nslots; ++c) prm.ulist[r * nslots + c] = r < q[c].size() ? q[c][r] : kNoWork;
+          npieces_total = (int)(maxlen * nslots);
+        } else {  // snake order (no padding)
+          for (size_t k = 0; k < order.size(); ++k) {
+            const int r = (int)(k / nslots), c = (int)(k % nslots);
+            const int mr = (int)std::min<int64_t>(nslots, (int64_t)order.size() - (int64_t)r * nslots);
+            prm.ulist[r * nslots + ((r & 1) ? mr - 1 - c : c)] = order[k].second;
+          }
+        }
       }
       prm.use_ulist = 1;
+      slots = nslots;
     }
-    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, pair, s);
+    const int grid = pair ? 2 * slots : slots;
+    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, pair, s, npieces_total);
     if (st != JIGSAW_SUCCESS) return st;
   }
   return JIGSAW_SUCCESS;

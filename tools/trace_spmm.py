@@ -26,7 +26,16 @@ def report(tag, ev_us, tr, ghz):
     start, end = tr[:, 15], tr[:, 13]
     span = (end.max() - start.min()) / 1e3
     print(f"\n== {tag}: event {ev_us:.1f} us, CTA span {span:.1f} us, CTAs {len(tr)}, "
-          f"start spread {(start.max() - start.min()) / 1e3:.2f} us")
+          f"start spread {(start.max() - start.min()) / 1e3:.2f} us, units/CTA min {tr[:, 12].min()} "
+          f"median {int(np.median(tr[:, 12]))} max {tr[:, 12].max()}")
+    last = np.where(tr[:, 5] > 0, (tr[:, 5] - tr[:, 0]) / ghz / 1e3, 0)
+    order = np.argsort(-last)[:8]
+    print("   slowest CTAs (last MMA commit us, units, k-blocks, us waiting for data): " +
+          ", ".join(f"#{i}: {last[i]:.1f} ({tr[i, 12]}, {tr[i, 8]}, {tr[i, 7] / ghz / 1e3:.1f})" for i in order))
+    fast = np.argsort(last)
+    fast = [i for i in fast if last[i] > 0][:4]
+    print("   fastest CTAs: " + ", ".join(f"#{i}: {last[i]:.1f} ({tr[i, 12]}, {tr[i, 8]}, {tr[i, 7] / ghz / 1e3:.1f})"
+                                         for i in fast))
     for k, name in NAMES.items():
         d = (tr[:, k] - tr[:, 0]) / ghz / 1e3
         d = d[(tr[:, k] != 0) & (d > -1) & (d < 1e4)]
