@@ -238,8 +238,9 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--workload", default="c2")
-    ap.add_argument("--panel-rows", type=int, default=128, choices=[128, 256],
-                    help="reorder panel height: 128 (one CTA per panel) or 256 (CTA pairs)")
+    ap.add_argument("--panel-rows", type=int, default=0, choices=[0, 128, 256],
+                    help="reorder panel height: 0 = library auto (256 for M >= 4096), 128 (one CTA "
+                         "per panel) or 256 (CTA pairs)")
     ap.add_argument("--impl", default="jigsaw", choices=["jigsaw", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-cublas", action="store_true")
@@ -477,7 +478,7 @@ def main():
         "config": {"workload": desc, "matrices_on_rank0": len(points),
                    "flops": "dense-equivalent 2*M*N*K per matrix",
                    "l2": "flushed (256 MB write) before every timed step", "launch": "step = jigsaw_spmm_batched over the batch (one grouped k_spmm launch per 64 matrices), captured in a CUDA graph",
-                   "seeds": f"synth.SEED_BASE + 1000*rank + index", "format": f"P={args.panel_rows}, SPTC residual"},
+                   "seeds": f"synth.SEED_BASE + 1000*rank + index", "format": f"panel_rows={args.panel_rows or 'auto'} (P used: {sorted(set(h.info()['panel_rows'] for h in hs))}), SPTC residual"},
         "roofline": roof,
         "cpu_baseline": cpu,
         "e2e": {"value": total_eff / e2e_s / 1e12, "unit": "TFLOP/s",

@@ -59,8 +59,9 @@ typedef enum {
 
 typedef struct {
   int panel_rows;    /* rows per panel (the BLOCK_TILE analogue, R-Q5/R-Q6): 128 (one CTA per
-                        panel, default) or 256 (a CTA pair per panel: tcgen05 cta_group::2,
-                        M = 256, each dense B tile staged once per pair); 64 -> UNSUPPORTED */
+                        panel; the default when opt is NULL), 256 (a CTA pair per panel:
+                        tcgen05 cta_group::2, M = 256, each dense B tile staged once per
+                        pair) or 0 = auto (256 when M >= 4096, else 128); 64 -> UNSUPPORTED */
   int residual_mode; /* jigsaw_residual_mode_t */
   int reserved[6];   /* must be zero */
 } jigsaw_options_t;

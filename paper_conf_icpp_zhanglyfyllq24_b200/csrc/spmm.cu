@@ -29,6 +29,10 @@
 #include "internal.h"
 #include "ptx.cuh"
 
+#ifndef JIG_HALVES
+#define JIG_HALVES 0  // pair N = 256 as two 128-column halves (see Cfg::kHalves); measured slower
+#endif
+
 namespace jig {
 
 namespace {
@@ -54,14 +58,22 @@ struct Cfg {
   static constexpr int kStageB = kChunks * kChunkB;
   static constexpr int kStages = kPair ? (NT == 256 ? 4 : 6) : NT == 256 ? 2 : NT == 128 ? 4 : 5;
   static constexpr int kAccCols = NT;
-  static constexpr int kAccBufs = NT == 256 ? 1 : 2;   // TMEM: 512 columns total
-  static constexpr int kEColBase = kAccBufs * NT;
+  // kHalves (pair, N = 256): the accumulator is two 128-column halves taken from
+  // a ring of three half-buffers, each MMA k-step issued as two N = 128 MMAs, so
+  // the next unit starts as soon as the epilogue has drained one half.
+  static constexpr bool kHalves = JIG_HALVES && kPair && NT == 256;
+  static constexpr int kAccBufs = kHalves ? 3 : NT == 256 ? 1 : 2;   // TMEM: 512 columns total
+  static constexpr int kEColBase = kHalves ? 3 * 128 : kAccBufs * NT;
   static constexpr uint32_t kTmemCols = kAccBufs * NT + 4 * kStages <= 256 ? 256 : 512;
   static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
   static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
   static constexpr int kStageC = 4 * 32 * 64;  // epilogue: per warp 32 rows x 32 fp16 columns
+  // gather-list ring: twice as deep as the stage ring, filled kStages k-blocks
+  // ahead of the A/E copies, so the B producers never wait on the gather list
+  static constexpr int kGS = 2 * kStages;
+  static constexpr int kGAhead = kStages;
   static constexpr size_t kSmem =
-      1024 + (size_t)kStages * (kStageB + kStageA + kStageE + kStageG) + kRecvBytes + kStageC + 512;
+      1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 512;
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
@@ -95,11 +107,13 @@ struct ParamsT {
   // a unit split into `pieces` k-ranges (split-K inside the persistent launch)
   // reduces its fp32 partials through `ws` (slots pslot .. pslot + pieces - 1)
   uint32_t ulist[MAXU];
-  float* ws;        // partial tiles: [slot][rank][NT / 32][128][32] fp32
+  float* ws;        // partial tiles: [slot][rank][NT / 32][warp 4][8][lane 32][4] fp32
   int* wcnt;        // per split unit and CTA rank: pieces finished (reset by the last)
   int nprob, nunits, S, use_pin, use_ulist;
   int sched;  // >= 0: dynamic tile scheduler on counter slot `sched`; -1: static round-robin
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
+  int prefetch;  // 1: prefetch each unit's gather lists / metadata into L2 at unit start
+  int dbg;       // developer timing experiments (JIGSAW_DBG, results invalid): 1 skip tcgen05.cp, 2 skip MMAs
 };
 using ParamsOne = ParamsT<1, 128, 1>;        // single product (~2.2 KB of parameters)
 using ParamsGroup = ParamsT<64, 1024, 2048>; // grouped launch (~31 KB)
@@ -262,21 +276,22 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint8_t* sB = smem;                                   // kStages x kStageB (1024-aligned)
   uint8_t* sA = sB + C_::kStages * C_::kStageB;         // kStages x 16 KB
   uint8_t* sE = sA + C_::kStages * kStageA;             // kStages x 2 KB
-  int32_t* sG = reinterpret_cast<int32_t*>(sE + C_::kStages * kStageE);  // kStages x 128 gather rows
-  uint8_t* sRecv = reinterpret_cast<uint8_t*>(sG) + C_::kStages * kStageG;  // split-K receive buffer
+  int32_t* sG = reinterpret_cast<int32_t*>(sE + C_::kStages * kStageE);  // kGS x 128 gather rows
+  uint8_t* sRecv = reinterpret_cast<uint8_t*>(sG) + C_::kGS * kStageG;     // split-K receive buffer
   uint8_t* sC = sRecv + C_::kRecvBytes;                                       // epilogue staging
   uint64_t* full = reinterpret_cast<uint64_t*>(sC + C_::kStageC);
   uint64_t* empty = full + C_::kStages;
-  uint64_t* gfull = empty + C_::kStages;  // gather list of the stage has landed
-  uint64_t* tfull = gfull + C_::kStages;
-  uint64_t* tempty = tfull + 2;
-  uint64_t* recv_full = tempty + 2;
+  uint64_t* gfull = empty + C_::kStages;  // gather-list ring slot has landed
+  uint64_t* gempty = gfull + C_::kGS;     // gather-list ring slot read by all B producers
+  uint64_t* tfull = gempty + C_::kGS;
+  uint64_t* tempty = tfull + 3;
+  uint64_t* recv_full = tempty + 3;
   uint64_t* rfull = recv_full + 1;   // unit ring (dynamic scheduler)
   uint64_t* rempty = rfull + kSD;
   uint64_t* pfull = rempty + kSD;    // kPair, even CTA: the odd CTA's stage has landed
   volatile int* ring = reinterpret_cast<volatile int*>(pfull + C_::kStages);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pfull + C_::kStages) + kSD;
-  volatile int* s_last = reinterpret_cast<volatile int*>(tmem_slot + 1);  // split piece: this CTA reduces
+  const uint32_t s_last = smem_u32(tmem_slot + 1);  // split piece: this CTA reduces (int flag)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = kSplit ? prm.S : 1;
@@ -294,10 +309,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     for (int s = 0; s < C_::kStages; ++s) {
       mbar_init(&full[s], 1 + 32 * kBProdWarps);  // A/E expect_tx arrival + B-producer cp.async arrivals
       mbar_init(&empty[s], 1);
-      mbar_init(&gfull[s], 1);
       mbar_init(&pfull[s], 1);
     }
-    for (int a = 0; a < 2; ++a) {
+    for (int s = 0; s < C_::kGS; ++s) {
+      mbar_init(&gfull[s], 1);
+      mbar_init(&gempty[s], kBProdWarps);
+    }
+    for (int a = 0; a < 3; ++a) {
       mbar_init(&tfull[a], 1);
       mbar_init(&tempty[a], kPair ? 8 : 4);  // epilogue warps (of both CTAs of a pair)
     }
@@ -329,8 +347,59 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       int stage = 0, hint = 0, nkb_issued = 0, rslot = 0;
       uint32_t phase = 0, rph = 0;
       int* ctr = dyn ? &g_sched[prm.sched][0] : nullptr;
-      for (int un = cluster_id;;) {
-        const int u = un < prm.nunits ? un : -1;
+      // Unit sequence of this CTA (static stride or dynamic scheduler), fetched
+      // into a small queue shared by two cursors over the same (unit, k-block)
+      // sequence: the gather-list cursor runs kGAhead k-blocks ahead of the A/E
+      // cursor, so gather lists land long before their B rows are needed
+      // (the P:220-226 dependency, pipelined one level further).
+      constexpr int kQ = 16;
+      int uq[kQ];
+      int qn = 0, mq = 0, next_un = cluster_id;
+      auto fetch = [&]() {
+        const int un = next_un < prm.nunits ? next_un : -1;
+        if (un >= 0) next_un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : un + nclusters;
+        uq[qn % kQ] = un;
+        ++qn;
+      };
+      // gather-list cursor
+      int gq = 0, ghint = 0, gkb = 0, gkbe = 0, gslot = 0;
+      uint32_t gph = 0;
+      int64_t gj = 0;
+      bool gend = false;
+      Work gwk;
+      auto g_issue_upto = [&](int64_t limit) {
+        while (gj < limit && !gend) {
+          if (gkb >= gkbe) {  // next unit with work
+            if (gq == qn) {
+              if (qn - mq >= kQ) return;  // queue full: the A/E cursor catches up first
+              fetch();
+            }
+            const int u = uq[gq % kQ];
+            if (u < 0) {
+              gend = true;
+              return;
+            }
+            ++gq;
+            gwk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, ghint);
+            if (!gwk.valid) continue;
+            gkb = gwk.kb_lo;
+            gkbe = gwk.kb_hi;
+            continue;
+          }
+          const int steps = gwk.steps(gkb);
+          mbar_wait(&gempty[gslot], gph ^ 1);
+          mbar_arrive_expect_tx(&gfull[gslot], (uint32_t)(steps * 128));
+          bulk_g2s(sG + gslot * kRowsPerBlock, gwk.G + gwk.gks(gkb) * 32, steps * 128, &gfull[gslot]);
+          ++gkb;
+          ++gj;
+          if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
+        }
+      };
+      int64_t mi = 0;  // k-blocks issued by the A/E cursor
+      for (;;) {
+        if (mq == qn) fetch();
+        const int u = uq[mq % kQ];
+        ++mq;
         if (dyn) {  // publish the unit to the other warp roles
           mbar_wait(&rempty[rslot], rph ^ 1);
           ring[rslot] = u;
@@ -338,25 +407,28 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (++rslot == kSD) { rslot = 0; rph ^= 1; }
         }
         if (u < 0) break;
-        un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : u + nclusters;  // latency hidden by the loads below
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
         if (!wk.valid) continue;
         const int64_t kb0 = wk.kb0;
+        if (prm.prefetch && wk.kb_hi > wk.kb_lo) {
+          // the unit's metadata into L2 up front
+          const int kbe = min(wk.kb_hi, wk.nkb_s);
+          if (kbe > wk.kb_lo)
+            bulk_prefetch_l2(wk.Eimg + (kb0 + wk.kb_lo) * kEBlockBytes, (uint32_t)(kbe - wk.kb_lo) * kEBlockBytes);
+        }
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
+          g_issue_upto(mi + 1 + C_::kGAhead);
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
           const int64_t gks = wk.gks(kb);
           mbar_wait(&empty[stage], phase ^ 1);
-          // gather list first, through the TMA path: the B producers wait only on
-          // it, never on an L1 load queued behind earlier cp.async traffic
-          mbar_arrive_expect_tx(&gfull[stage], (uint32_t)(steps * 128));
-          bulk_g2s(sG + stage * kRowsPerBlock, wk.G + gks * 32, steps * 128, &gfull[stage]);
           mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
           bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
           if (!dense) bulk_g2s(sE + stage * kStageE, wk.Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
           if (u == cluster_id && kb == wk.kb_lo) JIG_TRACE(2);
           JIG_TRACE_KB(0, nkb_issued);
           ++nkb_issued;
+          ++mi;
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
@@ -377,8 +449,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     constexpr int LPR = C_::kNTL / 8;      // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
-    int stage = 0, hint = 0, traced = 0, rslot = 0;
-    uint32_t phase = 0, rph = 0;
+    int stage = 0, hint = 0, traced = 0, rslot = 0, gslot = 0;
+    uint32_t phase = 0, rph = 0, gph = 0;
     for (int us = cluster_id;; us += nclusters) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
@@ -390,10 +462,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int64_t ldb = wk.N, K = wk.K;
       for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
         const int steps = wk.steps(kb);
+        const bool active = w < steps && !(half && wk.dense(kb));   // a dense step uses 16 B rows
+        int32_t gl = 0;
+        if (active) {
+          mbar_wait(&gfull[gslot], gph);
+          gl = ld_shared_s32(smem_u32(sG + gslot * kRowsPerBlock + 32 * w + lane));
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&gempty[gslot]);
+        if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
         mbar_wait(&empty[stage], phase ^ 1);
-        if (w < steps && !(half && wk.dense(kb))) {   // a dense step uses 16 B rows
-          mbar_wait(&gfull[stage], phase);
-          const int32_t gl = sG[stage * kRowsPerBlock + 32 * w + lane];
+        if (active) {
           uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
 #pragma unroll
           for (int it = 0; it < 16 / RPI; ++it) {
@@ -435,11 +514,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     __syncwarp();
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
+    // One lane runs the loop and issues the tcgen05 ops (a whole-warp loop with
+    // an elected issuer measured 5-8 % slower end to end).
     if (lane == 0) {
+      constexpr bool issuer = true;
       constexpr int MM = kPair ? 256 : 128;
       const uint32_t idesc0 = idesc_f16(MM, NT, 0, 1, 1, 0);
       const uint32_t idesc1 = idesc_f16(MM, NT, 0, 1, 1, 1);
       const uint32_t idesc_dense = idesc_f16(MM, NT, 0, 1, 0, 0);
+      constexpr int NH = C_::kHalves ? 128 : NT;   // N of one MMA instruction
+      const uint32_t hdesc0 = idesc_f16(MM, NH, 0, 1, 1, 0);
+      const uint32_t hdesc1 = idesc_f16(MM, NH, 0, 1, 1, 1);
+      const uint32_t hdesc_dense = idesc_f16(MM, NH, 0, 1, 0, 0);
       int stage = 0, hint = 0, nkb_mma = 0, rslot = 0;
       uint32_t phase = 0, rph = 0;
       int it = 0;
@@ -451,64 +537,103 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         if (!wk.valid) continue;
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
-        const int a = it % C_::kAccBufs;
-        const uint32_t use = (uint32_t)(it / C_::kAccBufs);
+        // accumulator buffer(s) of this unit; kHalves: half-uses 2it, 2it+1 of the 3-ring
+        const int a = C_::kHalves ? (2 * it) % 3 : it % C_::kAccBufs;
+        const int a1 = (2 * it + 1) % 3;
+        const uint32_t use = C_::kHalves ? (uint32_t)((2 * it) / 3) : (uint32_t)(it / C_::kAccBufs);
+        const uint32_t use1 = (uint32_t)((2 * it + 1) / 3);
         if (kPair)
           mbar_wait_cluster(&tempty[a], (use & 1) ^ 1);
         else
           mbar_wait(&tempty[a], (use & 1) ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tbase + a * C_::kAccCols;
+        const uint32_t d_tmem = tbase + (C_::kHalves ? a * 128 : a * C_::kAccCols);
+        const uint32_t d_tmem1 = tbase + a1 * 128;
         for (int kb = kb_lo; kb < kb_hi; ++kb) {
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
           const long long tw0 = prm.trace ? clock64() : 0;
           mbar_wait(&full[stage], phase);
-          if (kPair) mbar_wait_cluster(&pfull[stage], phase);
+          // pfull: CTA-scope acquire.  The odd CTA released its stage at cluster scope
+          // after observing its own copies complete; the data is read by the tensor
+          // core (async proxy, ordered by tcgen05.fence), not by this thread, and a
+          // cluster-scope acquire would add an L1 invalidate (CCTL.IVALL) per k-block.
+          if (kPair) mbar_wait(&pfull[stage], phase);
           if (prm.trace) wait_cycles += clock64() - tw0;
           tc_fence_after();
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
           const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
-          if (!dense) {
+          if (!dense && !(prm.dbg & 1)) {
             const uint64_t edesc = smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0);
-            if constexpr (kPair)
-              tc_cp_128x128b_pair(e_tmem, edesc);
-            else
-              tc_cp_128x128b(e_tmem, edesc);
+            if (issuer) {
+              if constexpr (kPair)
+                tc_cp_128x128b_pair(e_tmem, edesc);
+              else
+                tc_cp_128x128b(e_tmem, edesc);
+            }
           }
           JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
-          for (int s = 0; s < steps; ++s) {
+          for (int s = 0; s < (prm.dbg & 2 ? 0 : steps); ++s) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
             const uint64_t bdesc = smem_desc(b_base + s * 32 * 128, kChunkB, 1024, 2);
             const uint32_t acc = (kb != kb_lo) || (s != 0);
-            if constexpr (kPair) {
-              if (dense)
-                tc_mma_f16_pair(d_tmem, adesc, bdesc, idesc_dense, acc);
-              else
-                tc_mma_sp_f16_pair(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+            if constexpr (C_::kHalves) {
+              // low half: SW128 chunk 0 of each CTA (unit columns [0,64) and [128,192));
+              // high half: chunk 1 (unit columns [64,128) and [192,256))
+              const uint64_t bdesc1 = smem_desc(b_base + kChunkB + s * 32 * 128, kChunkB, 1024, 2);
+              if (dense) {
+                if (issuer) tc_mma_f16_pair(d_tmem, adesc, bdesc, hdesc_dense, acc);
+              } else {
+                if (issuer) tc_mma_sp_f16_pair(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? hdesc1 : hdesc0, acc);
+              }
+              if (kb == kb_lo && s == 0) {  // the high half-buffer: drained by the previous epilogue?
+                mbar_wait_cluster(&tempty[a1], (use1 & 1) ^ 1);
+                tc_fence_after();
+              }
+              if (issuer) {
+                if (dense)
+                  tc_mma_f16_pair(d_tmem1, adesc, bdesc1, hdesc_dense, acc);
+                else
+                  tc_mma_sp_f16_pair(d_tmem1, adesc, bdesc1, e_tmem + (s & 2), (s & 1) ? hdesc1 : hdesc0, acc);
+              }
+            } else if constexpr (kPair) {
+              if (issuer) {
+                if (dense)
+                  tc_mma_f16_pair(d_tmem, adesc, bdesc, idesc_dense, acc);
+                else
+                  tc_mma_sp_f16_pair(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+              }
             } else {
-              if (dense)   // residual tile on the dense tensor path, K = 16
-                tc_mma_f16(d_tmem, adesc, bdesc, idesc_dense, acc);
-              else
-                tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+              if (issuer) {   // residual tile on the dense tensor path, K = 16
+                if (dense)
+                  tc_mma_f16(d_tmem, adesc, bdesc, idesc_dense, acc);
+                else
+                  tc_mma_sp_f16(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? idesc1 : idesc0, acc);
+              }
             }
           }
           JIG_TRACE_KB(5, nkb_mma);
-          if constexpr (kPair)
-            tc_commit_pair(&empty[stage]);   // frees the stage in both CTAs
-          else
-            tc_commit(&empty[stage]);
+          if (issuer) {
+            if constexpr (kPair)
+              tc_commit_pair(&empty[stage]);   // frees the stage in both CTAs
+            else
+              tc_commit(&empty[stage]);
+          }
           JIG_TRACE_KB(3, nkb_mma);
           ++nkb_mma;
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
-        if constexpr (kPair)
-          tc_commit_pair(&tfull[a]);
-        else
-          tc_commit(&tfull[a]);
+        if (issuer) {
+          if constexpr (kPair) {
+            tc_commit_pair(&tfull[a]);
+            if constexpr (C_::kHalves) tc_commit_pair(&tfull[a1]);
+          } else {
+            tc_commit(&tfull[a]);
+          }
+        }
         JIG_TRACE(5);
         ++it;
       }
@@ -533,14 +658,42 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       __half* const Cm = wk.C;
       const bool has_acc = wk.kb_hi > wk.kb_lo;
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
-      const int a = it % C_::kAccBufs;
+      const int a = C_::kHalves ? (2 * it) % 3 : it % C_::kAccBufs;
+      const int a1 = (2 * it + 1) % 3;                   // kHalves: the high half-buffer
       if (has_acc) {
-        mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
+        mbar_wait(&tfull[a], (uint32_t)(C_::kHalves ? (2 * it) / 3 : it / C_::kAccBufs) & 1);
+        if constexpr (C_::kHalves) mbar_wait(&tfull[a1], (uint32_t)((2 * it + 1) / 3) & 1);
         tc_fence_after();
       }
+      // 32-column chunk k of the unit: its TMEM column and its C column offset.
+      // kHalves: chunks 0-3 are the low half-buffer = unit columns [0,64) ++ [128,192),
+      // chunks 4-7 the high one = [64,128) ++ [192,256) (B is split across the pair
+      // by 64-column SW128 chunks, see the MMA issuer)
+      auto tcol = [&](int k) -> uint32_t {
+        if constexpr (C_::kHalves) return (uint32_t)((k < 4 ? a : a1) * 128 + 32 * (k & 3));
+        return (uint32_t)(a * C_::kAccCols + 32 * k);
+      };
+      auto ucol = [&](int k) -> int {
+        if constexpr (C_::kHalves) {
+          const int j = k >> 2, cc = 32 * (k & 3);
+          return cc < 64 ? 64 * j + cc : 128 + 64 * j + (cc - 64);
+        }
+        return 32 * k;
+      };
+      auto release = [&](int buf) {  // this warp is done reading accumulator buffer `buf`
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if (kPair && rank != 0)
+            mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[buf]), 0));  // the pair's issuer
+          else
+            mbar_arrive(&tempty[buf]);
+        }
+      };
+      bool released_lo = false;
       if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
       if constexpr (!kSplit) {
-        uint8_t* stg = sC + q * (32 * 64);
+        const uint32_t stg = smem_u32(sC + q * (32 * 64));
         bool write_c = true;
         const int npc = wk.npieces;
         if (npc > 1) {
@@ -553,16 +706,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           for (int c0 = 0; c0 < NT; c0 += 32) {
             uint32_t v[32];
             if (has_acc) {
-              tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * C_::kAccCols + c0, v);
+              tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + tcol(c0 / 32), v);
               tc_wait_ld();
             } else {
 #pragma unroll
               for (int j = 0; j < 32; ++j) v[j] = 0;
             }
-            float4* dst = reinterpret_cast<float4*>(part + ((size_t)(c0 / 32) * 128 + r) * 32);
+            // [chunk][warp][j][lane] float4s: each store instruction is 512 contiguous bytes
+            float4* dst = reinterpret_cast<float4*>(part + ((size_t)(c0 / 32) * 128 + q * 32) * 32) + lane;
 #pragma unroll
             for (int j = 0; j < 8; ++j)
-              __stcg(dst + j, make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
+              __stcg(dst + 32 * j, make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
                                          __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
           }
           __threadfence();
@@ -570,19 +724,23 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (threadIdx.x == 64) {
             int* cnt = prm.wcnt + wk.pslot * CS + rank;
             const int done = atomicAdd(cnt, 1);
-            *s_last = done == npc - 1;
+            st_shared_s32(s_last, done == npc - 1);
             if (done == npc - 1) atomicExch(cnt, 0);  // ready for the next launch
           }
           asm volatile("bar.sync 1, 128;" ::: "memory");
-          write_c = *s_last != 0;
+          write_c = ld_shared_s32(s_last) != 0;
           if (write_c) __threadfence();
         }
 #pragma unroll 1
         for (int c0 = 0; write_c && c0 < NT; c0 += 32) {
           uint32_t v[32];
           if (has_acc) {
-            tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + a * C_::kAccCols + c0, v);
+            tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + tcol(c0 / 32), v);
             tc_wait_ld();
+            if (C_::kHalves && npc == 1 && c0 == 96) {  // low half drained: the next unit may start
+              release(a);
+              released_lo = true;
+            }
           } else {
 #pragma unroll
             for (int j = 0; j < 32; ++j) v[j] = 0;     // all-zero panel (R-Q21)
@@ -592,10 +750,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             for (int pc = 0; pc < npc; ++pc) {
               if (pc == wk.piece) continue;
               const float4* src = reinterpret_cast<const float4*>(
-                  prm.ws + ((size_t)(wk.pslot + pc) * CS + rank) * kTile + ((size_t)(c0 / 32) * 128 + r) * 32);
+                  prm.ws + ((size_t)(wk.pslot + pc) * CS + rank) * kTile + ((size_t)(c0 / 32) * 128 + q * 32) * 32) + lane;
 #pragma unroll
               for (int j = 0; j < 8; ++j) {
-                const float4 x = __ldcg(src + j);
+                const float4 x = __ldcg(src + 32 * j);
                 v[4 * j] = __float_as_uint(__uint_as_float(v[4 * j]) + x.x);
                 v[4 * j + 1] = __float_as_uint(__uint_as_float(v[4 * j + 1]) + x.y);
                 v[4 * j + 2] = __float_as_uint(__uint_as_float(v[4 * j + 2]) + x.z);
@@ -613,16 +771,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
             pk.z = pack_h2(__uint_as_float(v[8 * j + 4]), __uint_as_float(v[8 * j + 5]));
             pk.w = pack_h2(__uint_as_float(v[8 * j + 6]), __uint_as_float(v[8 * j + 7]));
-            *reinterpret_cast<uint4*>(stg + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)) = pk;
+            st_shared_v4u(stg + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4), pk);
           }
           __syncwarp();
 #pragma unroll
           for (int i = 0; i < 4; ++i) {
             const int rr = 8 * i + (lane >> 2), c = lane & 3;
             const int64_t grow = wk.row0 + q * 32 + rr;
-            const uint4 pk = *reinterpret_cast<const uint4*>(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
-            if (grow < M && n0 + c0 + 8 * c < N)
-              *reinterpret_cast<uint4*>(Cm + grow * N + n0 + c0 + 8 * c) = pk;
+            const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
+            const int col = n0 + ucol(c0 / 32) + 8 * c;
+            if (grow < M && col < N) *reinterpret_cast<uint4*>(Cm + grow * N + col) = pk;
           }
           __syncwarp();
         }
@@ -677,14 +835,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       }
       if (warp == 2 && lane == 0) JIG_TRACE(9);
       if (has_acc) {
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) {
-          if (kPair && rank != 0)
-            mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[a]), 0));  // the pair's issuer
-          else
-            mbar_arrive(&tempty[a]);
-        }
+        if (!released_lo) release(a);
+        if constexpr (C_::kHalves) release(a1);
         ++it;
       }
     }
@@ -830,6 +982,8 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   prm.sched = -1;
   if (S == 1 && !pair && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
     prm.sched = (g_sched_next[dev]++) % kSchedSlots;
+  prm.prefetch = getenv("JIGSAW_NO_PREFETCH") ? 0 : 1;
+  prm.dbg = getenv("JIGSAW_DBG") ? atoi(getenv("JIGSAW_DBG")) : 0;
   const char* tr = getenv("JIGSAW_TRACE");
   prm.trace = (tr && tr[0] == '1') ? 1 : 0;
   if (prm.trace) g_trace_ctas = std::min(grid, kTraceCTAs);
@@ -852,6 +1006,9 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   return set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
 }
 
+static jigsaw_status_t launch_group(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
+                                    void* const* Cs, int count, cudaStream_t s);
+
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
   thread_local ParamsOne prm;  // host-side scratch for the parameter block
   prm.nprob = 1;
@@ -863,7 +1020,14 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   int NT = 128, S = 1, grid = 1;
   choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
   const bool pair = f.P == kPairPanelRows;
-  if (const char* e = pair ? nullptr : getenv("JIGSAW_FORCE_SPLIT")) {  // test hook: force NT = 64 with split S
+  const char* force_split = getenv("JIGSAW_FORCE_SPLIT");
+  if (pair || (S == 1 && NT >= 128 && !force_split)) {
+    // large products: the grouped persistent path (cost-ordered schedule, long
+    // units split into pieces; CTA pairs are only scheduled there)
+    const Format* fp = &f;
+    return launch_group(&fp, &dB, &N, &dC, 1, s);
+  }
+  if (const char* e = force_split) {  // test hook: force NT = 64 with split S
     const int fs = atoi(e);
     if (fs == 1 || fs == 2 || fs == 4 || fs == 8) {
       NT = 64;

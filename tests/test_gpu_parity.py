@@ -404,7 +404,9 @@ def test_pair_panels_full_size_sampled():
     M, K, N, v, s = 4096, 4096, 4096, 8, 0.9
     A = synth.vector_sparse(M, K, v, s, 31)
     B = synth.dense_b(K, N, 31)
-    h = jig.reorder(_dev(A), v, panel_rows=256)
+    h = jig.reorder(_dev(A), v, panel_rows=0)           # auto: M >= 4096 -> 256-row panels
+    assert h.info()["panel_rows"] == 256
+    assert jig.reorder(_dev(A[:512]), v, panel_rows=0).info()["panel_rows"] == 128
     C = _host(h.spmm(_dev(B)))
     torch.cuda.synchronize()
     rows = np.array([0, 127, 128, 255, 256 * 7 + 5, 256 * 7 + 200, M - 129, M - 1])

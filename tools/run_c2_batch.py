@@ -17,7 +17,7 @@ def main(reps=4, wl="c2"):
     hs, Bs, Cs = [], [], []
     for i, (M, K, v, s, N) in enumerate(pts):
         A = synth.vector_sparse(M, K, v, s, i)
-        hs.append(jig.reorder(torch.from_numpy(A.view(np.int16)).cuda().view(torch.float16), v))
+        hs.append(jig.reorder(torch.from_numpy(A.view(np.int16)).cuda().view(torch.float16), v, panel_rows=0))
         Bs.append(torch.from_numpy(synth.dense_b(K, N, i).view(np.int16)).cuda().view(torch.float16))
         Cs.append(torch.empty((M, N), dtype=torch.float16, device="cuda"))
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")

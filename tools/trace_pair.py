@@ -24,8 +24,9 @@ def main():
     A = synth.vector_sparse(M, K, v, s, 3)
     B = dev(synth.dense_b(K, N, 3))
     C = torch.empty((M, N), dtype=torch.float16, device="cuda")
-    for P, nt in [(128, "128"), (128, "256"), (256, "128"), (256, "256")]:
+    for P, nt, dbg in [(256, "256", "0"), (128, "128", "0")]:
         os.environ["JIGSAW_FORCE_NT"] = nt
+        os.environ["JIGSAW_DBG"] = dbg
         h = jig.reorder(dev(A), v, panel_rows=P)
         for rep in range(3):
             flush.zero_()
@@ -35,14 +36,14 @@ def main():
             e1.record()
             torch.cuda.synchronize()
         tr = jig.debug_trace()
-        report(f"P={P} NT={nt} {M}x{K} v{v} s{s} N{N}", e0.elapsed_time(e1) * 1e3, tr, ghz)
+        report(f"dbg={dbg} P={P} NT={nt} {M}x{K} v{v} s{s} N{N}", e0.elapsed_time(e1) * 1e3, tr, ghz)
         kb = np.zeros(8 * 6 * 32, np.int64)
         jig.lib().jigsaw_debug_trace(kb.ctypes.data_as(ctypes.c_void_p), -1)
         kb = kb.reshape(8, 6, 32)
-        for cta in range(2):
+        for cta in range(1):
             t0 = tr[cta, 0]
             print(f"  CTA {cta} per k-block (us after entry): AE-issue / B-issue / full-seen / after-cp / after-mma / commit")
-            for k in range(0, 32, 2):
+            for k in range(8, 16, 2):
                 row = [(kb[cta, r, k] - t0) / ghz / 1e3 if kb[cta, r, k] > t0 else float('nan') for r in (0, 1, 2, 4, 5, 3)]
                 print("   kb %2d  " % k + "  ".join(f"{x:7.2f}" for x in row))
         h.free()

@@ -24,7 +24,7 @@ def main():
             for i, (M, K, v, s, N) in enumerate(pts)]
     B2 = [dev(b) for _, b, _ in mats]
     C2 = [torch.empty((a.shape[0], b.shape[1]), dtype=torch.float16, device="cuda") for a, b, _ in mats]
-    for P, nt in [(128, ""), (256, "128"), (256, "256")]:
+    for P, nt in [(128, ""), (256, "256"), (256, "256")]:
         if nt:
             os.environ["JIGSAW_FORCE_NT"] = nt
         else:

@@ -28,7 +28,8 @@ def report(tag, ev_us, tr, ghz):
     print(f"\n== {tag}: event {ev_us:.1f} us, CTA span {span:.1f} us, CTAs {len(tr)}, "
           f"start spread {(start.max() - start.min()) / 1e3:.2f} us, units/CTA min {tr[:, 12].min()} "
           f"median {int(np.median(tr[:, 12]))} max {tr[:, 12].max()}")
-    last = np.where(tr[:, 5] > 0, (tr[:, 5] - tr[:, 0]) / ghz / 1e3, 0)
+    last = (tr[:, 5] - tr[:, 0]) / ghz / 1e3
+    last = np.where((last > 0) & (last < 1e4) & (tr[:, 8] > 0), last, 0)
     order = np.argsort(-last)[:8]
     print("   slowest CTAs (last MMA commit us, units, k-blocks, us waiting for data): " +
           ", ".join(f"#{i}: {last[i]:.1f} ({tr[i, 12]}, {tr[i, 8]}, {tr[i, 7] / ghz / 1e3:.1f})" for i in order))
