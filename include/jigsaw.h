@@ -61,7 +61,10 @@ typedef struct {
   int panel_rows;    /* rows per panel (the BLOCK_TILE analogue, R-Q5/R-Q6): 128 (one CTA per
                         panel; the default when opt is NULL), 256 (a CTA pair per panel:
                         tcgen05 cta_group::2, M = 256, each dense B tile staged once per
-                        pair) or 0 = auto (256 when M >= 4096, else 128); 64 -> UNSUPPORTED */
+                        pair) or 0 = auto (256 when M >= 4096, else 128).  16, 32 and 64
+                        (the paper's BLOCK_TILE sizes) build the format for
+                        export / statistics only: jigsaw_spmm on such a handle returns
+                        JIGSAW_ERROR_UNSUPPORTED (no tcgen05 M below 128 is built) */
   int residual_mode; /* jigsaw_residual_mode_t */
   int reserved[6];   /* must be zero */
 } jigsaw_options_t;

@@ -92,9 +92,9 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
   if (!(v == 1 || v == 2 || v == 4 || v == 8)) return set_status(JIGSAW_ERROR_INVALID_VALUE, "v must be 1, 2, 4 or 8");
   if (M % v) return set_status(JIGSAW_ERROR_INVALID_VALUE, "M must be a multiple of v");
   if (opt) {
-    if (opt->panel_rows != 0 && opt->panel_rows != kPanelRows && opt->panel_rows != kPairPanelRows)
-      return set_status(opt->panel_rows == 64 ? JIGSAW_ERROR_UNSUPPORTED : JIGSAW_ERROR_INVALID_VALUE,
-                        "panel_rows must be 0 (auto), 128 or 256 (64 is not built in this version)");
+    const int pr = opt->panel_rows;
+    if (!(pr == 0 || pr == 16 || pr == 32 || pr == 64 || pr == kPanelRows || pr == kPairPanelRows))
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "panel_rows must be 0 (auto), 16, 32, 64, 128 or 256");
     if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC && opt->residual_mode != JIGSAW_RESIDUAL_DENSE)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
     for (int i = 0; i < 6; ++i)
@@ -113,6 +113,10 @@ jigsaw_status_t validate_spmm(jigsaw_handle_t h, const void* B, int64_t N, const
   int dev = -1;
   cudaGetDevice(&dev);
   if (dev != h->f.device) return set_status(JIGSAW_ERROR_WRONG_DEVICE, "current device differs from the handle's");
+  if (h->f.P < kPanelRows)
+    return set_status(JIGSAW_ERROR_UNSUPPORTED,
+                      "formats with panel_rows < 128 are for analysis (export / statistics); the SpMM needs "
+                      "128 or 256 (tcgen05 M)");
   return JIGSAW_SUCCESS;
 }
 

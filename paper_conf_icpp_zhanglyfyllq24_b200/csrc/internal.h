@@ -41,7 +41,7 @@ struct Format {
   uint8_t* d_Aimg = nullptr;  // [halves][nksteps][4096]: UMMA K-major no-swizzle core matrices
   uint8_t* d_Eimg = nullptr;  // [halves][nkblocks][128][4] u32: TMEM metadata lanes
   int32_t* d_G = nullptr;     // [nksteps][32]: B row per logical column (PAD -> K, TMA zero fill)
-  int halves() const { return P / kPanelRows; }
+  int halves() const { return P > kPanelRows ? P / kPanelRows : 1; }
   int64_t planeA() const { return nksteps * (int64_t)kKStepBytesA; }
   int64_t planeE() const { return nkblocks * (int64_t)kEBlockBytes; }
   // stats

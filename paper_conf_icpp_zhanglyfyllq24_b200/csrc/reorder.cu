@@ -537,6 +537,7 @@ __global__ void __launch_bounds__(256) k_emit(const uint16_t* __restrict__ A, in
   uint8_t* Ah = Aimg + half * planeA + gks * kKStepBytesA;
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
+    if (r >= P) break;  // P = 16: 32 threads (the gather list), 16 rows
     uint16_t v[8];
     uint16_t meta = 0;
 #pragma unroll
@@ -575,7 +576,7 @@ __global__ void __launch_bounds__(256) k_emit(const uint16_t* __restrict__ A, in
     smeta[h][r] = meta;
   }
   __syncthreads();
-  {
+  if (tid < P) {
     const int L = tid & 127, m0 = L & 7, h = (L >> 3) & 1, m2 = L >> 4;
     const int r0 = half * 128 + 16 * m2 + m0;
     const uint32_t w = (uint32_t)smeta[h][r0] | ((uint32_t)smeta[h][r0 + 8] << 16);
@@ -611,6 +612,7 @@ __global__ void __launch_bounds__(256) k_emit_dense(const uint16_t* __restrict__
   uint8_t* Ah = Aimg + (r >> 7) * planeA + gks * kKStepBytesA;
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
+    if (r >= P) break;
     uint16_t v[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
@@ -771,12 +773,12 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
     JIG_CU(cudaMemcpyAsync(tile_off, f->tile_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemsetAsync(f->d_Eimg, 0, (size_t)kEBlockBytes * f->nkblocks * f->halves(), stream), "memset E");
     if (maxks > 0)
-      k_emit<<<dim3(maxks, npan), P, 0, stream>>>(dA, M, K, P, sc, T, tile_off, d_ksoff, d_kboff, f->d_Aimg,
+      k_emit<<<dim3(maxks, npan), P < 32 ? 32 : P, 0, stream>>>(dA, M, K, P, sc, T, tile_off, d_ksoff, d_kboff, f->d_Aimg,
                                                 f->planeA(), reinterpret_cast<uint32_t*>(f->d_Eimg),
                                                 f->planeE() / 4, f->d_G, f->d_colidx, f->d_perm, f->d_kind,
                                                 f->d_nevict, Kp);
     if (maxdk > 0)
-      k_emit_dense<<<dim3(maxdk, npan), P, 0, stream>>>(dA, M, K, P, queue, qcap, nres, f->d_pin, f->d_Aimg,
+      k_emit_dense<<<dim3(maxdk, npan), P < 32 ? 32 : P, 0, stream>>>(dA, M, K, P, queue, qcap, nres, f->d_pin, f->d_Aimg,
                                                       f->planeA(), f->d_G);
     JIG_CU(cudaGetLastError(), "k_emit launch");
     JIG_CU(cudaEventRecord(ev1, stream), "cudaEventRecord");

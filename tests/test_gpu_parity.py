@@ -179,8 +179,9 @@ def test_abi_errors_on_gpu():
     assert st == 1                            # misaligned B
     with pytest.raises(jig.JigsawError):
         jig.reorder(_dev(synth.vector_sparse(8, 8, 1, 0.5, 1)), 3)
+    h64 = jig.reorder(_dev(A), 4, panel_rows=64)   # analysis-only format: no M = 64 MMA
     with pytest.raises(jig.JigsawError) as e:
-        jig.reorder(_dev(A), 4, panel_rows=64)  # declared, not built
+        h64.spmm(B)
     assert e.value.status == 2
     with pytest.raises(jig.JigsawError) as e:
         jig.reorder(_dev(A), 4, panel_rows=100)
@@ -449,3 +450,22 @@ def test_grouped_split_pieces(P, pieces, monkeypatch):
                     spmm_check(_host(c), a, b)
             else:
                 spmm_check(_host(c), a, b)
+
+
+@pytest.mark.parametrize("P", [16, 32, 64])
+@pytest.mark.parametrize("M,K,v,s,mode", [(256, 512, 8, 0.90, 0), (200, 300, 4, 0.70, 0), (128, 256, 2, 0.5, 1)])
+def test_small_panel_formats_bit_exact(P, M, K, v, s, mode):
+    """The paper's BLOCK_TILE heights through the GPU builder: format
+    bit-exact vs oracle O2 at the same P (the reorder-study path)."""
+    A = synth.vector_sparse(M, K, v, s, 40 + P)
+    h = jig.reorder(_dev(A), v, panel_rows=P, residual_mode=mode)
+    g = h.export()
+    ref = oracle.reorder(A, P=P, mode=mode)
+    assert_format_equal(g, ref)
+    if mode == 1:
+        assert np.array_equal(g["rcol"], ref.rcol)
+        assert np.array_equal(g["dvals"], ref.dvals)
+    check.check_format(A, P, g["T"], g["gather"], g["vals"], g["meta"], perm=g["perm"],
+                       D=g["D"] if mode == 1 else None, rcol=g["rcol"] if mode == 1 else None,
+                       dvals=g["dvals"] if mode == 1 else None)
+    h.free()
