@@ -41,7 +41,21 @@ constexpr unsigned kFullMask = 0xFFFFFFFFu;
 constexpr int kBProdWarp0 = 6;
 constexpr int kBProdWarps = 8;   // two warps per k-step (16 B rows each): 8 cp.async warps
                                  // reach ~36 B/clk/SM vs ~28 with 4 (profiles/r01_gather_bench.txt)
-constexpr int kThreads = 32 * (kBProdWarp0 + kBProdWarps);
+// Warps 6-15 except 9 and 13 are the B producers: warp w runs on SM
+// sub-partition w % 4, and sub-partition 1 is left to the MMA warp (1) and one
+// epilogue warp (5), so the single-thread tcgen05 issue loop is not starved of
+// issue slots by producer warps (warps 9 and 13 idle).
+#ifndef JIG_SPARE_SMSP1
+#define JIG_SPARE_SMSP1 1
+#endif
+constexpr int kThreads = JIG_SPARE_SMSP1 ? 32 * 16 : 32 * (kBProdWarp0 + kBProdWarps);
+__device__ __forceinline__ int bprod_index(int warp) {  // -1: not a B producer
+  if (warp < kBProdWarp0) return -1;
+  if (!JIG_SPARE_SMSP1) return warp - kBProdWarp0;
+  if ((warp & 3) == 1) return -1;
+  const int i = warp - kBProdWarp0;  // 0..9 -> skip 3 (warp 9) and 7 (warp 13)
+  return i - (i > 3) - (i > 7);
+}
 constexpr int kRowsPerBlock = 32 * kStepsPerBlock;  // B rows per k-block (128)
 constexpr int kChunkB = kRowsPerBlock * 128;        // one 64-column SW128 chunk: 16 KB
 constexpr int kStageA = kStepsPerBlock * kKStepBytesA;  // 16 KB
@@ -440,12 +454,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         }
       }
     }
-  } else if (warp >= kBProdWarp0) {
+  } else if (bprod_index(warp) >= 0) {
     // ------------------------------------------------------------ B producers
     // Warp w copies the 32 B rows of k-step w of each k-block; the row indices
     // come from the stage's gather list in shared memory (TMA-loaded by warp 0).
-    const int w = (warp - kBProdWarp0) >> 1;   // k-step within the k-block
-    const int half = (warp - kBProdWarp0) & 1;  // rows [16*half, 16*half + 16) of it
+    const int bw = bprod_index(warp);
+    const int w = bw >> 1;     // k-step within the k-block
+    const int half = bw & 1;   // rows [16*half, 16*half + 16) of it
     constexpr int LPR = C_::kNTL / 8;      // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
@@ -576,6 +591,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
+          if (!C_::kHalves && !dense && steps == kStepsPerBlock && !(prm.dbg & 2)) {
+            // full sparse k-block: one asm block for the 4 MMAs (descriptors stepped in PTX)
+            tc_mma_sp_f16_x4<kPair>(d_tmem, smem_desc(a_base, 128, 256, 0), smem_desc(b_base, kChunkB, 1024, 2),
+                                    kKStepBytesA >> 4, (32 * 128) >> 4, e_tmem, idesc0, kb != kb_lo);
+          } else
           for (int s = 0; s < (prm.dbg & 2 ? 0 : steps); ++s) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
             const uint64_t bdesc = smem_desc(b_base + s * 32 * 128, kChunkB, 1024, 2);
@@ -643,7 +663,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       }
     }
     __syncwarp();
-  } else {
+  } else if (warp >= 2 && warp <= 5) {
     // ------------------------------------------------------------ epilogue (warps 2-5)
     const int q = warp & 3;  // TMEM lane quarter this warp may access
     int it = 0, hint = 0, rslot = 0;
