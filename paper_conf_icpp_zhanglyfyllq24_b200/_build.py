@@ -26,7 +26,9 @@ def _stale() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
-    cmd = [NVCC, *FLAGS, "-o", LIB, *[os.path.join(CSRC, s) for s in SOURCES]]
+    # developer defines, e.g. JIGSAW_NVCC_DEFINES="JIG_TRACE_KB_ON=1" for the per-k-block timeline
+    defs = [f"-D{d}" for d in os.environ.get("JIGSAW_NVCC_DEFINES", "").split() if d]
+    cmd = [NVCC, *FLAGS, *defs, "-o", LIB, *[os.path.join(CSRC, s) for s in SOURCES]]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + r.stdout + r.stderr)

@@ -217,6 +217,69 @@ __device__ __forceinline__ void tc_mma_sp_f16_pair(uint32_t d_tmem, uint64_t ade
 // desc0 + s * step (16-byte units in the address field), metadata column
 // e + (s & 2), selector id2 = s & 1 (idesc1 = idesc0 | 1).  `acc0` = accumulate
 // flag of the first step (the others always accumulate).
+// Metadata copy / commit executed by the whole converged warp (one elected lane).
+template <bool kPairT>
+__device__ __forceinline__ void tc_cp_128x128b_warp(uint32_t taddr, uint64_t sdesc) {
+  if constexpr (kPairT)
+    asm volatile("{\n\t.reg .pred q;\n\telect.sync _|q, 0xffffffff;\n\t"
+                 "@q tcgen05.cp.cta_group::2.128x128b [%0], %1;\n\t}" ::"r"(taddr), "l"(sdesc) : "memory");
+  else
+    asm volatile("{\n\t.reg .pred q;\n\telect.sync _|q, 0xffffffff;\n\t"
+                 "@q tcgen05.cp.cta_group::1.128x128b [%0], %1;\n\t}" ::"r"(taddr), "l"(sdesc) : "memory");
+}
+template <bool kPairT>
+__device__ __forceinline__ void tc_commit_warp(uint64_t* bar) {
+  if constexpr (kPairT)
+    asm volatile(
+        "{\n\t.reg .pred q;\n\telect.sync _|q, 0xffffffff;\n\t"
+        "@q tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
+            smem_u32(bar)),
+        "h"((uint16_t)3)
+        : "memory");
+  else
+    asm volatile("{\n\t.reg .pred q;\n\telect.sync _|q, 0xffffffff;\n\t"
+                 "@q tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(
+                     smem_u32(bar))
+                 : "memory");
+}
+// Same, executed by the whole converged warp: one lane is elected inside the
+// asm, so the compiler sees warp-uniform code around the tcgen05 ops.
+template <bool kPairT>
+__device__ __forceinline__ void tc_mma_sp_f16_x4_warp(uint32_t d_tmem, uint64_t adesc0, uint64_t bdesc0,
+                                                      uint32_t astep, uint32_t bstep, uint32_t e_tmem,
+                                                      uint32_t idesc0, uint32_t acc0) {
+  if constexpr (kPairT) {
+    asm volatile(
+        "{\n\t.reg .pred p, q;\n\t.reg .b64 a1, a2, a3, b1, b2, b3, as, bs;\n\t.reg .b32 e2, i1;\n\t"
+        "elect.sync _|q, 0xffffffff;\n\t"
+        "cvt.u64.u32 as, %3;\n\tcvt.u64.u32 bs, %4;\n\t"
+        "add.s64 a1, %1, as;\n\tadd.s64 a2, a1, as;\n\tadd.s64 a3, a2, as;\n\t"
+        "add.s64 b1, %2, bs;\n\tadd.s64 b2, b1, bs;\n\tadd.s64 b3, b2, bs;\n\t"
+        "add.u32 e2, %5, 2;\n\tor.b32 i1, %6, 1;\n\t"
+        "setp.ne.b32 p, %7, 0;\n\t"
+        "@q tcgen05.mma.sp.cta_group::2.kind::f16 [%0], %1, %2, [%5], %6, p;\n\t"
+        "@q tcgen05.mma.sp.cta_group::2.kind::f16 [%0], a1, b1, [%5], i1, 1;\n\t"
+        "@q tcgen05.mma.sp.cta_group::2.kind::f16 [%0], a2, b2, [e2], %6, 1;\n\t"
+        "@q tcgen05.mma.sp.cta_group::2.kind::f16 [%0], a3, b3, [e2], i1, 1;\n\t}" ::"r"(d_tmem),
+        "l"(adesc0), "l"(bdesc0), "r"(astep), "r"(bstep), "r"(e_tmem), "r"(idesc0), "r"(acc0)
+        : "memory");
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p, q;\n\t.reg .b64 a1, a2, a3, b1, b2, b3, as, bs;\n\t.reg .b32 e2, i1;\n\t"
+        "elect.sync _|q, 0xffffffff;\n\t"
+        "cvt.u64.u32 as, %3;\n\tcvt.u64.u32 bs, %4;\n\t"
+        "add.s64 a1, %1, as;\n\tadd.s64 a2, a1, as;\n\tadd.s64 a3, a2, as;\n\t"
+        "add.s64 b1, %2, bs;\n\tadd.s64 b2, b1, bs;\n\tadd.s64 b3, b2, bs;\n\t"
+        "add.u32 e2, %5, 2;\n\tor.b32 i1, %6, 1;\n\t"
+        "setp.ne.b32 p, %7, 0;\n\t"
+        "@q tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%5], %6, p;\n\t"
+        "@q tcgen05.mma.sp.cta_group::1.kind::f16 [%0], a1, b1, [%5], i1, 1;\n\t"
+        "@q tcgen05.mma.sp.cta_group::1.kind::f16 [%0], a2, b2, [e2], %6, 1;\n\t"
+        "@q tcgen05.mma.sp.cta_group::1.kind::f16 [%0], a3, b3, [e2], i1, 1;\n\t}" ::"r"(d_tmem),
+        "l"(adesc0), "l"(bdesc0), "r"(astep), "r"(bstep), "r"(e_tmem), "r"(idesc0), "r"(acc0)
+        : "memory");
+  }
+}
 template <bool kPairT>
 __device__ __forceinline__ void tc_mma_sp_f16_x4(uint32_t d_tmem, uint64_t adesc0, uint64_t bdesc0, uint32_t astep,
                                                  uint32_t bstep, uint32_t e_tmem, uint32_t idesc0, uint32_t acc0) {

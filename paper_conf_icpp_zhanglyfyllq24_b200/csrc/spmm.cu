@@ -138,9 +138,14 @@ constexpr int kTraceCTAs = 1024, kTraceSlots = 16;
 __device__ long long g_trace[kTraceCTAs * kTraceSlots];
 constexpr int kTraceKB = 32;
 __device__ long long g_trace_kb[8 * 6 * kTraceKB];  // [cta<8][AE issue, B issue, full seen, commit, after cp, after mma][kb]
+// Per-k-block timeline (developer builds only: -DJIG_TRACE_KB_ON=1); in the
+// product build the hot loops carry no per-k-block trace code.
+#ifndef JIG_TRACE_KB_ON
+#define JIG_TRACE_KB_ON 0
+#endif
 #define JIG_TRACE_KB(role, n)                                                        \
   do {                                                                               \
-    if (prm.trace && blockIdx.x < 8 && (n) < kTraceKB)                               \
+    if (JIG_TRACE_KB_ON && prm.trace && blockIdx.x < 8 && (n) < kTraceKB)            \
       g_trace_kb[(blockIdx.x * 6 + (role)) * kTraceKB + (n)] = clock64();            \
   } while (0)
 __device__ __forceinline__ long long gtimer() {
@@ -529,10 +534,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     __syncwarp();
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
-    // One lane runs the loop and issues the tcgen05 ops (a whole-warp loop with
-    // an elected issuer measured 5-8 % slower end to end).
-    if (lane == 0) {
-      constexpr bool issuer = true;
+    // The whole warp runs the loop; the tcgen05 ops are issued by a lane elected
+    // inside their asm blocks, so the compiler sees warp-uniform code and moves
+    // the operands to uniform registers without a per-instruction R2UR
+    // waterfall (the single-lane loop spent more issue slots than the MMAs took).
+    {
+      const bool issuer = lane == 0;
+      const uint32_t tbase_u = __shfl_sync(kFullMask, tbase, 0);
       constexpr int MM = kPair ? 256 : 128;
       const uint32_t idesc0 = idesc_f16(MM, NT, 0, 1, 1, 0);
       const uint32_t idesc1 = idesc_f16(MM, NT, 0, 1, 1, 1);
@@ -546,7 +554,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       int it = 0;
       long long wait_cycles = 0;
       for (int us = cluster_id;; us += nclusters) {
-        const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, false, 0) : (us < prm.nunits ? us : -1);
+        const int u = dyn ? __shfl_sync(kFullMask, ring_take(ring, rfull, rempty, rslot, rph, true, lane), 0) : (us < prm.nunits ? us : -1);
         if (u < 0) break;
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
         if (!wk.valid) continue;
@@ -562,39 +570,35 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         else
           mbar_wait(&tempty[a], (use & 1) ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tbase + (C_::kHalves ? a * 128 : a * C_::kAccCols);
-        const uint32_t d_tmem1 = tbase + a1 * 128;
+        const uint32_t d_tmem = tbase_u + (C_::kHalves ? a * 128 : a * C_::kAccCols);
+        const uint32_t d_tmem1 = tbase_u + a1 * 128;
         for (int kb = kb_lo; kb < kb_hi; ++kb) {
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
-          const long long tw0 = prm.trace ? clock64() : 0;
+          const long long tw0 = JIG_TRACE_KB_ON && prm.trace ? clock64() : 0;
           mbar_wait(&full[stage], phase);
           // pfull: CTA-scope acquire.  The odd CTA released its stage at cluster scope
           // after observing its own copies complete; the data is read by the tensor
           // core (async proxy, ordered by tcgen05.fence), not by this thread, and a
           // cluster-scope acquire would add an L1 invalidate (CCTL.IVALL) per k-block.
           if (kPair) mbar_wait(&pfull[stage], phase);
-          if (prm.trace) wait_cycles += clock64() - tw0;
+          if (JIG_TRACE_KB_ON && prm.trace) wait_cycles += clock64() - tw0;
           tc_fence_after();
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
-          const uint32_t e_tmem = tbase + C_::kEColBase + 4 * stage;
+          const uint32_t e_tmem = tbase_u + C_::kEColBase + 4 * stage;
           if (!dense && !(prm.dbg & 1)) {
             const uint64_t edesc = smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0);
-            if (issuer) {
-              if constexpr (kPair)
-                tc_cp_128x128b_pair(e_tmem, edesc);
-              else
-                tc_cp_128x128b(e_tmem, edesc);
-            }
+            tc_cp_128x128b_warp<kPair>(e_tmem, edesc);
           }
           JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
           if (!C_::kHalves && !dense && steps == kStepsPerBlock && !(prm.dbg & 2)) {
             // full sparse k-block: one asm block for the 4 MMAs (descriptors stepped in PTX)
-            tc_mma_sp_f16_x4<kPair>(d_tmem, smem_desc(a_base, 128, 256, 0), smem_desc(b_base, kChunkB, 1024, 2),
-                                    kKStepBytesA >> 4, (32 * 128) >> 4, e_tmem, idesc0, kb != kb_lo);
+            tc_mma_sp_f16_x4_warp<kPair>(d_tmem, smem_desc(a_base, 128, 256, 0),
+                                         smem_desc(b_base, kChunkB, 1024, 2), kKStepBytesA >> 4,
+                                         (32 * 128) >> 4, e_tmem, idesc0, kb != kb_lo);
           } else
           for (int s = 0; s < (prm.dbg & 2 ? 0 : steps); ++s) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
@@ -636,24 +640,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             }
           }
           JIG_TRACE_KB(5, nkb_mma);
-          if (issuer) {
-            if constexpr (kPair)
-              tc_commit_pair(&empty[stage]);   // frees the stage in both CTAs
-            else
-              tc_commit(&empty[stage]);
-          }
+          tc_commit_warp<kPair>(&empty[stage]);   // frees the stage (in both CTAs of a pair)
           JIG_TRACE_KB(3, nkb_mma);
           ++nkb_mma;
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
-        if (issuer) {
-          if constexpr (kPair) {
-            tc_commit_pair(&tfull[a]);
-            if constexpr (C_::kHalves) tc_commit_pair(&tfull[a1]);
-          } else {
-            tc_commit(&tfull[a]);
-          }
-        }
+        tc_commit_warp<kPair>(&tfull[a]);
+        if constexpr (C_::kHalves) tc_commit_warp<kPair>(&tfull[a1]);
         JIG_TRACE(5);
         ++it;
       }
