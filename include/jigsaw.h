@@ -176,11 +176,14 @@ JIGSAW_API int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N);
 
 /* Per-CTA timeline of the most recent k_spmm launch made with the environment
  * variable JIGSAW_TRACE=1 (otherwise nothing is recorded).  Copies up to
- * max_ctas records of 16 int64 each into `out` (host): slots 0-11 are SM clock
+ * max_ctas records of 24 int64 each into `out` (host): slots 0-11 are SM clock
  * (clock64) stamps at fixed points of the kernel (entry, setup done, first A/E
  * copy, first B copies, first full stage, last MMA commit, accumulator ready,
  * sends done, reduction data ready, stores done, exit), 13 / 15 are
- * %globaltimer (ns) at exit / entry, 14 is the SM id.  max_ctas < 0 instead
+ * %globaltimer (ns) at exit / entry, 14 is the SM id; 16-23 are prologue /
+ * teardown stamps (A/E producer: first unit fetched, decoded, gather list
+ * issued; B producer: unit decoded, gather list landed; MMA warp: unit decoded;
+ * 23: exit barrier passed).  max_ctas < 0 instead
  * copies the per-k-block timeline of CTAs 0..7 (8 x 6 x 32 int64: A/E copy
  * issued, B copies issued, stage full seen by the MMA thread, commit issued,
  * metadata copy issued, MMAs issued).

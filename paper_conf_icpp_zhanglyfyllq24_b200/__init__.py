@@ -227,8 +227,8 @@ def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: in
 
 
 def debug_trace(max_ctas: int = 1024) -> np.ndarray:
-    """Timeline of the last k_spmm launch made with JIGSAW_TRACE=1: [ctas, 16] int64."""
-    out = np.zeros((max_ctas, 16), np.int64)
+    """Timeline of the last k_spmm launch made with JIGSAW_TRACE=1: [ctas, 24] int64."""
+    out = np.zeros((max_ctas, 24), np.int64)
     n = lib().jigsaw_debug_trace(out.ctypes.data_as(ctypes.c_void_p), max_ctas)
     if n < 0:
         raise JigsawError(4, "jigsaw_debug_trace failed")

@@ -29,6 +29,9 @@
 #include "internal.h"
 #include "ptx.cuh"
 
+#ifndef JIG_BGROUPS
+#define JIG_BGROUPS 1  // B-producer warp groups (see Cfg::kBGroups); > 1 measured slower in k_spmm
+#endif
 #ifndef JIG_HALVES
 #define JIG_HALVES 0  // pair N = 256 as two 128-column halves (see Cfg::kHalves); measured slower
 #endif
@@ -68,7 +71,9 @@ constexpr int kStageG = kRowsPerBlock * 4;          // gather list of a k-block:
 template <int NT, bool kSplit, bool kPair = false>
 struct Cfg {
   static constexpr int kNTL = kPair ? NT / 2 : NT;  // B columns staged by this CTA
-  static constexpr int kChunks = kNTL / 64;
+  // B is staged as 64-column SW128 chunks; NT = 32 fills the first half of one
+  // chunk (the MMA with N = 32 reads only those columns of the swizzled atom)
+  static constexpr int kChunks = kNTL >= 64 ? kNTL / 64 : 1;
   static constexpr int kStageB = kChunks * kChunkB;
   static constexpr int kStages = kPair ? (NT == 256 ? 4 : 6) : NT == 256 ? 2 : NT == 128 ? 4 : 5;
   static constexpr int kAccCols = NT;
@@ -84,7 +89,17 @@ struct Cfg {
   static constexpr int kStageC = 4 * 32 * 64;  // epilogue: per warp 32 rows x 32 fp16 columns
   // gather-list ring: twice as deep as the stage ring, filled kStages k-blocks
   // ahead of the A/E copies, so the B producers never wait on the gather list
-  static constexpr int kGS = 2 * kStages;
+  // B-producer warp groups: group g fills the k-blocks j (CTA-wide k-block
+  // sequence number) with j % kBGroups == g, its 8 / kBGroups warps splitting the
+  // 128 rows.  A warp's cp.async batches complete one after another, so k_spmm's
+  // gather rate grows with the number of k-blocks in flight from DIFFERENT warps
+  // (tools/ldgsts_probe.cu, profiles/r01s_ldgsts_probe.txt: 64-byte rows 9.6 ->
+  // 22.6 B/clk/SM, 256-byte rows 18.7 -> 32.6).  kBGroups <= kStages keeps every
+  // parity wait within one phase; kGS is a multiple of kBGroups so each gather
+  // ring slot always belongs to the same group.
+  static constexpr int kBGroups = JIG_BGROUPS < kStages ? JIG_BGROUPS : kStages;
+  static constexpr int kWPG = kBProdWarps / kBGroups;  // warps per group
+  static constexpr int kGS = (2 * kStages + kBGroups - 1) / kBGroups * kBGroups;
   static constexpr int kGAhead = kStages;
   static constexpr size_t kSmem =
       1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 512;
@@ -134,7 +149,7 @@ using ParamsGroup = ParamsT<64, 1024, 2048>; // grouped launch (~31 KB)
 constexpr int kMaxProblems = ParamsGroup::kMaxProblems;
 
 // Opt-in per-CTA timeline (clock64 / %globaltimer), read by jigsaw_debug_trace.
-constexpr int kTraceCTAs = 1024, kTraceSlots = 16;
+constexpr int kTraceCTAs = 1024, kTraceSlots = 24;
 __device__ long long g_trace[kTraceCTAs * kTraceSlots];
 constexpr int kTraceKB = 32;
 __device__ long long g_trace_kb[8 * 6 * kTraceKB];  // [cta<8][AE issue, B issue, full seen, commit, after cp, after mma][kb]
@@ -326,13 +341,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < C_::kStages; ++s) {
-      mbar_init(&full[s], 1 + 32 * kBProdWarps);  // A/E expect_tx arrival + B-producer cp.async arrivals
+      mbar_init(&full[s], 1 + 32 * C_::kWPG);  // A/E expect_tx arrival + the owning B group's cp.async arrivals
       mbar_init(&empty[s], 1);
       mbar_init(&pfull[s], 1);
     }
     for (int s = 0; s < C_::kGS; ++s) {
       mbar_init(&gfull[s], 1);
-      mbar_init(&gempty[s], kBProdWarps);
+      mbar_init(&gempty[s], C_::kWPG);
     }
     for (int a = 0; a < 3; ++a) {
       mbar_init(&tfull[a], 1);
@@ -344,6 +359,42 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       mbar_init(&rempty[i], kBProdWarps + 1 + 4);  // B-producer warps + MMA + epilogue warps
     }
     fence_barrier_init();
+    fence_proxy_async();
+  }
+  // Parallel initial fill (before the block-wide sync, overlapping the TMEM
+  // allocation): lane l of warp 0 issues the gather list of the CTA's first unit's
+  // k-block l (ring slot l) and, for l < kStages, its A / E copies (stage l), so
+  // the first loads leave at kernel start instead of one after another from a
+  // single thread (each mbarrier / bulk-copy operation costs ~100 cycles of issue).
+  int nA0 = 0, nG0 = 0;
+  Work w0;
+  w0.valid = false;
+  if (warp == 0) {
+    __syncwarp();
+    if (cluster_id < prm.nunits) {
+      int h0 = 0;
+      w0 = decode_unit<NT, kPair, Prm>(prm, cluster_id, rank, S, h0);
+      if (w0.valid) {
+        const int nkb = w0.kb_hi - w0.kb_lo;
+        nA0 = min(nkb, C_::kStages);
+        nG0 = min(nkb, C_::kGAhead + 1);
+      }
+    }
+    if (lane < nG0) {
+      const int kb = w0.kb_lo + lane;
+      const int steps = w0.steps(kb);
+      mbar_arrive_expect_tx(&gfull[lane], (uint32_t)(steps * 128));
+      bulk_g2s(sG + lane * kRowsPerBlock, w0.G + w0.gks(kb) * 32, steps * 128, &gfull[lane]);
+    }
+    if (lane < nA0) {
+      const int kb = w0.kb_lo + lane;
+      const int steps = w0.steps(kb);
+      const bool dense = w0.dense(kb);
+      mbar_arrive_expect_tx(&full[lane], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
+      bulk_g2s(sA + lane * kStageA, w0.Aimg + w0.gks(kb) * kKStepBytesA, steps * kKStepBytesA, &full[lane]);
+      if (!dense) bulk_g2s(sE + lane * kStageE, w0.Eimg + (w0.kb0 + kb) * kEBlockBytes, kStageE, &full[lane]);
+    }
+    if (lane == 0 && nA0 > 0) JIG_TRACE(2);
   }
   if (warp == 1) {
     if constexpr (kPair)
@@ -363,8 +414,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   if (warp == 0) {
     // ------------------------------------------------------------ A / E producer
     if (lane == 0) {
-      int stage = 0, hint = 0, nkb_issued = 0, rslot = 0;
-      uint32_t phase = 0, rph = 0;
+      // state after the parallel initial fill: stages 0..nA0-1 and gather slots
+      // 0..nG0-1 hold the first unit's first k-blocks
+      int stage = nA0 % C_::kStages, hint = 0, nkb_issued = nA0, rslot = 0;
+      uint32_t phase = nA0 == C_::kStages ? 1u : 0u, rph = 0;
       int* ctr = dyn ? &g_sched[prm.sched][0] : nullptr;
       // Unit sequence of this CTA (static stride or dynamic scheduler), fetched
       // into a small queue shared by two cursors over the same (unit, k-block)
@@ -381,11 +434,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         ++qn;
       };
       // gather-list cursor
-      int gq = 0, ghint = 0, gkb = 0, gkbe = 0, gslot = 0;
-      uint32_t gph = 0;
-      int64_t gj = 0;
+      int gq = 0, ghint = 0, gkb = 0, gkbe = 0, gslot = nG0 % C_::kGS;
+      uint32_t gph = nG0 == C_::kGS ? 1u : 0u;
+      int64_t gj = nG0;
       bool gend = false;
-      Work gwk;
+      Work gwk = w0;
+      if (nG0 > 0) {  // the gather cursor continues inside the first unit
+        fetch();
+        gq = 1;
+        gkb = w0.kb_lo + nG0;
+        gkbe = w0.kb_hi;
+      }
       auto g_issue_upto = [&](int64_t limit) {
         while (gj < limit && !gend) {
           if (gkb >= gkbe) {  // next unit with work
@@ -414,9 +473,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
         }
       };
-      int64_t mi = 0;  // k-blocks issued by the A/E cursor
+      int64_t mi = nA0;  // k-blocks issued by the A/E cursor
       for (;;) {
         if (mq == qn) fetch();
+        if (mq == 0) JIG_TRACE(16);
         const int u = uq[mq % kQ];
         ++mq;
         if (dyn) {  // publish the unit to the other warp roles
@@ -427,6 +487,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         }
         if (u < 0) break;
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+        if (mi == 0) JIG_TRACE(17);
         if (!wk.valid) continue;
         const int64_t kb0 = wk.kb0;
         if (prm.prefetch && wk.kb_hi > wk.kb_lo) {
@@ -435,8 +496,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (kbe > wk.kb_lo)
             bulk_prefetch_l2(wk.Eimg + (kb0 + wk.kb_lo) * kEBlockBytes, (uint32_t)(kbe - wk.kb_lo) * kEBlockBytes);
         }
-        for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
+        for (int kb = wk.kb_lo + (mq == 1 ? nA0 : 0); kb < wk.kb_hi; ++kb) {
           g_issue_upto(mi + 1 + C_::kGAhead);
+          if (mi == 0) JIG_TRACE(18);
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
           const int64_t gks = wk.gks(kb);
@@ -461,56 +523,71 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     }
   } else if (bprod_index(warp) >= 0) {
     // ------------------------------------------------------------ B producers
-    // Warp w copies the 32 B rows of k-step w of each k-block; the row indices
-    // come from the stage's gather list in shared memory (TMA-loaded by warp 0).
+    // Group grp copies the B rows of the k-blocks j with j % kBGroups == grp; warp
+    // wi of the group copies rows [wi*R, wi*R + R) of the k-block (R = 128 / kWPG,
+    // 32 rows per k-step), their indices taken from the k-block's gather list in
+    // shared memory (TMA-loaded by warp 0).
     const int bw = bprod_index(warp);
-    const int w = bw >> 1;     // k-step within the k-block
-    const int half = bw & 1;   // rows [16*half, 16*half + 16) of it
+    const int grp = bw / C_::kWPG, wi = bw % C_::kWPG;
+    constexpr int R = kRowsPerBlock / C_::kWPG;   // rows per warp and k-block
     constexpr int LPR = C_::kNTL / 8;      // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
     const int c = lane % LPR;
-    int stage = 0, hint = 0, traced = 0, rslot = 0, gslot = 0;
-    uint32_t phase = 0, rph = 0, gph = 0;
+    int hint = 0, traced = 0, rslot = 0;
+    uint32_t rph = 0;
+    int64_t j = 0;  // CTA-wide k-block sequence number (the stage ring's order)
     for (int us = cluster_id;; us += nclusters) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
       const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+      if (bw == 0 && lane == 0 && traced == 0) JIG_TRACE(19);
       if (!wk.valid) continue;
       const int col = wk.n0 + (kPair ? (int)rank * C_::kNTL : 0) + 8 * c;
       const bool colok = col < wk.N;
       const __half* Bp = wk.B;
       const int64_t ldb = wk.N, K = wk.K;
-      for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
+      int kb = wk.kb_lo + (int)((grp - j % C_::kBGroups + C_::kBGroups) % C_::kBGroups);
+      j += kb - wk.kb_lo;
+      for (; kb < wk.kb_hi; kb += C_::kBGroups, j += C_::kBGroups) {
+        const int stage = (int)(j % C_::kStages), gslot = (int)(j % C_::kGS);
+        const uint32_t phase = (uint32_t)((j / C_::kStages) & 1), gph = (uint32_t)((j / C_::kGS) & 1);
         const int steps = wk.steps(kb);
-        const bool active = w < steps && !(half && wk.dense(kb));   // a dense step uses 16 B rows
-        int32_t gl = 0;
-        if (active) {
-          mbar_wait(&gfull[gslot], gph);
-          gl = ld_shared_s32(smem_u32(sG + gslot * kRowsPerBlock + 32 * w + lane));
-        }
+        const bool dense = wk.dense(kb);   // a dense step uses 16 B rows
+        mbar_wait(&gfull[gslot], gph);
+        int32_t gl[(R + 31) / 32];
+#pragma unroll
+        for (int t = 0; t < (R + 31) / 32; ++t)
+          gl[t] = ld_shared_s32(smem_u32(sG + gslot * kRowsPerBlock + ((wi * R) & ~31) + 32 * t + lane));
+        if (bw == grp * C_::kWPG && lane == 0 && traced == 0) JIG_TRACE(20);
         __syncwarp();
         if (lane == 0) mbar_arrive(&gempty[gslot]);
-        if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
         mbar_wait(&empty[stage], phase ^ 1);
-        if (active) {
-          uint8_t* sb = sB + stage * C_::kStageB + (32 * w) * 128 + (c >> 3) * kChunkB;
+        uint8_t* sb = sB + stage * C_::kStageB + (c >> 3) * kChunkB;
 #pragma unroll
-          for (int it = 0; it < 16 / RPI; ++it) {
-            const int j = 16 * half + it * RPI + lane / LPR;
-            const int32_t g = __shfl_sync(kFullMask, gl, j);
+        for (int t = 0; t < (R + 31) / 32; ++t) {
+          const int ks = (wi * R) / 32 + t;          // k-step of these rows
+          const int jlo = R < 32 ? (wi * R) & 31 : 0;  // rows [jlo, jlo + min(R, 32)) of the k-step
+          if (ks >= steps || (dense && jlo >= 16)) continue;
+          const int jn = dense ? 16 - jlo : (R < 32 ? R : 32);
+#pragma unroll
+          for (int it = 0; it < (R < 32 ? R : 32) / RPI; ++it) {
+            const int jr = jlo + it * RPI + lane / LPR;
+            if (it * RPI >= jn) break;
+            const int32_t g = __shfl_sync(kFullMask, gl[t], jr);
             const bool ok = colok && g < K;
             const __half* src = ok ? Bp + (int64_t)g * ldb + col : Bp;
-            cp_async_16(sb + j * 128 + (((c & 7) ^ (j & 7)) << 4), src, ok ? 16u : 0u);
+            const int row = 32 * ks + jr;
+            cp_async_16(sb + row * 128 + (((c & 7) ^ (row & 7)) << 4), src, ok ? 16u : 0u);
           }
         }
         cp_async_mbar_arrive_noinc(&full[stage]);
-        if (lane == 0 && w == 0 && half == 0) {
+        if (lane == 0 && bw == 0) {
           if (traced == 0) JIG_TRACE(3);
           JIG_TRACE_KB(1, traced);
           ++traced;
         }
-        if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
       }
+      j -= kb - wk.kb_hi;  // the k-blocks of this unit past the last one of this group
     }
   } else if (warp == 1 && kPair && rank != 0) {
     // ------------------------------------------------------------ pair relay (odd CTA)
@@ -557,6 +634,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         const int u = dyn ? __shfl_sync(kFullMask, ring_take(ring, rfull, rempty, rslot, rph, true, lane), 0) : (us < prm.nunits ? us : -1);
         if (u < 0) break;
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+        if (it == 0 && lane == 0) JIG_TRACE(21);
         if (!wk.valid) continue;
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
@@ -859,10 +937,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   if (threadIdx.x == 0) JIG_TRACE(10);
   tc_fence_before();
   if constexpr (kSplit || kPair) {
-    cluster_sync_all();  // no CTA leaves while peers may still target its shared memory
+    // no CTA leaves while peers may still target its shared memory (DSMEM
+    // sends, pair commits); the C stores need no cluster-scope release here
+    cluster_sync_relaxed();
   } else {
     __syncthreads();
   }
+  if (threadIdx.x == 0) JIG_TRACE(23);
   if (warp == 1) {
     if constexpr (kPair)
       tmem_dealloc_pair<C_::kTmemCols>(tbase);
@@ -918,9 +999,9 @@ int spmm_num_sms() {
   return g_num_sms[dev];
 }
 
-// Tile / split selection: enough units for every SM -> NT = 128,
-// persistent; otherwise NT = 64 and, when the panels carry enough k-blocks,
-// split-K over a cluster of S = 2/4/8 CTAs.  256-row panels (CTA pairs): NT = 256
+// Tile / split selection: enough units for every SM -> NT = 128
+// (or 256), persistent; otherwise NT = 32 / 64 and split-K over a cluster of
+// S = 1/2/4 CTAs by the cost model below.  256-row panels (CTA pairs): NT = 256
 // when there is a unit for every pair, else NT = 128; grid = 2 x pairs.
 void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* grid) {
   if (f.P == kPairPanelRows) {
@@ -949,16 +1030,40 @@ void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* gr
     *grid = (int)std::min<int64_t>(u128, sms);
     return;
   }
-  const int64_t u64 = f.npanels * ((N + 63) / 64);
-  int64_t kb_total = 0;
-  for (int64_t p = 0; p < f.npanels; ++p) kb_total += (f.T[p] + 7) / 8 + (f.D[p] + 3) / 4;
-  const double kb_avg = f.npanels ? (double)kb_total / f.npanels : 0.0;
-  int s = 1;
-  // clusters of 8 do not all fit in one wave of 148 SMs (GPC granularity): S <= 4
-  while (s < 4 && u64 * (2 * s) <= sms && kb_avg >= 2.0 * s) s *= 2;
+  // Small products (fewer 128-column units than SMs): latency-bound.  Pick the
+  // tile width NT (32 or 64 columns) and the split-K factor S (1, 2, 4 CTAs of a
+  // cluster per unit, one wave) that minimise a per-CTA cost model in SM cycles
+  // (profiles/r01s_*: compressed A/E arrive by bulk TMA at ~70 B/clk/SM, the B
+  // row gather by 16-byte cp.async at ~35 B/clk/SM, the two overlap; the split
+  // reduction moves (S-1)/S of the fp32 partial tile through DSMEM at ~15 B/clk
+  // plus ~1500 cycles of cluster-wide skew and synchronisation).
+  int64_t kb_max = 0;
+  for (int64_t p = 0; p < f.npanels; ++p)
+    kb_max = std::max<int64_t>(kb_max, (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4);
+  double best = 1e30;
   *NT = 64;
-  *S = s;
-  *grid = s > 1 ? (int)(u64 * s) : (int)std::min<int64_t>(u64, sms);
+  *S = 1;
+  *grid = (int)std::min<int64_t>(f.npanels * ((N + 63) / 64), sms);
+  for (int nt : {32, 64}) {
+    if (force && force != nt) continue;
+    const int64_t units = f.npanels * ((N + nt - 1) / nt);
+    for (int s = 1; s <= 4; s *= 2) {
+      if (units * s > sms && !(s == 1 && units > sms && nt == 64)) continue;  // one wave (S = 1 may loop)
+      if (s > 1 && kb_max < 2 * s) continue;
+      const double waves = (double)((units * s + sms - 1) / sms);
+      const double nkb = (double)((kb_max + s - 1) / s) * waves;
+      const double t_ae = nkb * (kStepsPerBlock * kKStepBytesA + kEBlockBytes) / 70.0;
+      const double t_b = nkb * 128.0 * nt * 2 / 35.0;
+      const double t_red = s > 1 ? (double)(s - 1) / s * 128.0 * nt * 4 / 15.0 + 1500.0 : 0.0;
+      const double cost = std::max(t_ae, t_b) + t_red + 128.0 * nt * 2 / 32.0;
+      if (cost < best - 1.0) {
+        best = cost;
+        *NT = nt;
+        *S = s;
+        *grid = s > 1 ? (int)(units * s) : (int)std::min<int64_t>(units, sms);
+      }
+    }
+  }
 }
 
 template <class Prm>
@@ -993,8 +1098,6 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   prm.S = S;
   // persistent launches use the dynamic scheduler on a rotating counter slot
   prm.sched = -1;
-  if (S == 1 && !pair && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
-    prm.sched = (g_sched_next[dev]++) % kSchedSlots;
   prm.prefetch = getenv("JIGSAW_NO_PREFETCH") ? 0 : 1;
   prm.dbg = getenv("JIGSAW_DBG") ? atoi(getenv("JIGSAW_DBG")) : 0;
   const char* tr = getenv("JIGSAW_TRACE");
@@ -1006,6 +1109,9 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
     u += (int)(prm.pr[i].npanels * ((prm.pr[i].N + NT - 1) / NT));
   }
   prm.nunits = npieces_total >= 0 ? npieces_total : u;
+  // (a CTA per unit needs no scheduler: its one unit is known at kernel start)
+  if (S == 1 && !pair && grid < prm.nunits && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
+    prm.sched = (g_sched_next[dev]++) % kSchedSlots;
   constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 8;
   if (pair) {
     if (NT == 256) return launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s);
@@ -1013,9 +1119,12 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   }
   if (NT == 256) return launch_variant<256, false, false>(prm, grid, 1, dev, vb + 3, s);
   if (NT == 128) return launch_variant<128, false, false>(prm, grid, 1, dev, vb + 0, s);
+  if (NT == 32 && S == 1) return launch_variant<32, false, false>(prm, grid, 1, dev, vb + 6, s);
   if (S == 1) return launch_variant<64, false, false>(prm, grid, 1, dev, vb + 1, s);
-  if constexpr (std::is_same<Prm, ParamsOne>::value)
+  if constexpr (std::is_same<Prm, ParamsOne>::value) {
+    if (NT == 32) return launch_variant<32, true, false>(prm, grid, S, dev, vb + 7, s);
     return launch_variant<64, true, false>(prm, grid, S, dev, vb + 2, s);
+  }
   return set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
 }
 

@@ -36,13 +36,13 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
   __shared__ uint64_t full[kStages], empty[kStages];
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int nprod = mode == 1 ? 8 : mode == 4 ? 12 : (mode == 5 || mode == 6 || mode == 8 || mode == 9) ? 16
-                    : mode == 7 ? 8 : 4;
+                    : (mode == 7 || mode == 10) ? 8 : 4;
   const bool ldgsts = mode <= 1 || mode == 4 || mode == 5;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) {
       mbar_init(&full[s], (ldgsts || mode == 6) ? nprod * 32
                           : mode == 9 ? 8 * 32 + 8
-                          : (mode == 7 || mode == 8) ? nprod : 1 + (mode == 3 ? 3 : 0));
+                          : (mode == 7 || mode == 8 || mode == 10) ? nprod : 1 + (mode == 3 ? 3 : 0));
       mbar_init(&empty[s], 1);
     }
     fence_barrier_init();
@@ -126,8 +126,17 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
           mbar_arrive_expect_tx(&full[stage], kStageBytes);
           for (int q = 0; q < kRows / 4; ++q)
             for (int ch = 0; ch < 2; ++ch)
-              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, ri[4 * q], ri[4 * q + 1], ri[4 * q + 2],
-                          ri[4 * q + 3], &full[stage]);
+              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, hrow(blockIdx.x, kb, 4 * q, K),
+                          hrow(blockIdx.x, kb, 4 * q + 1, K), hrow(blockIdx.x, kb, 4 * q + 2, K),
+                          hrow(blockIdx.x, kb, 4 * q + 3, K), &full[stage]);
+        }
+      } else if (mode == 10) {
+        // TMA 2-D tile per row (box {64, 1}, SW128): 8 issuing warps, 32 rows x 2 chunks each
+        if (lane == 0) {
+          mbar_arrive_expect_tx(&full[stage], kStageBytes / nprod);
+          for (int row = w; row < kRows; row += nprod)
+            for (int ch = 0; ch < 2; ++ch)
+              tma_load_2d(st + ch * (kRows * 128) + row * 128, &tm, 64 * ch, hrow(blockIdx.x, kb, row, K), &full[stage]);
         }
       } else {
         if (lane == 0) {
@@ -135,8 +144,9 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
           else mbar_arrive(&full[stage]);
           for (int q = w * 8; q < w * 8 + 8; ++q)
             for (int ch = 0; ch < 2; ++ch)
-              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, ri[4 * q], ri[4 * q + 1], ri[4 * q + 2],
-                          ri[4 * q + 3], &full[stage]);
+              tma_gather4(st + ch * (kRows * 128) + q * 512, &tm, 64 * ch, hrow(blockIdx.x, kb, 4 * q, K),
+                          hrow(blockIdx.x, kb, 4 * q + 1, K), hrow(blockIdx.x, kb, 4 * q + 2, K),
+                          hrow(blockIdx.x, kb, 4 * q + 3, K), &full[stage]);
         }
       }
       if (++stage == kStages) { stage = 0; ph ^= 1; }
@@ -175,8 +185,8 @@ int main() {
   cudaFuncSetAttribute(gather_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   const char* names[] = {"LDGSTS 4 warps", "LDGSTS 8 warps", "TMA gather4, 1 issuer", "TMA gather4, 4 issuers",
                          "LDGSTS 12 warps", "LDGSTS 16 warps", "LDG+STS 16 warps", "TMA gather4, 8 issuers",
-                         "TMA gather4, 16 issuers", "LDGSTS 8w + gather4 8w"};
-  for (int mode = 0; mode < 10; ++mode) {
+                         "TMA gather4, 16 issuers", "LDGSTS 8w + gather4 8w", "TMA tile row, 8 issuers"};
+  for (int mode = 0; mode < 11; ++mode) {
     for (int rep = 0; rep < 3; ++rep) {
       cudaEvent_t a, b;
       cudaEventCreate(&a);
