@@ -24,6 +24,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <string>
 #include <type_traits>
 
 #include "internal.h"
@@ -42,7 +43,10 @@ namespace {
 
 constexpr unsigned kFullMask = 0xFFFFFFFFu;
 constexpr int kBProdWarp0 = 6;
-constexpr int kBProdWarps = 8;   // two warps per k-step (16 B rows each): 8 cp.async warps
+#ifndef JIG_BWARPS
+#define JIG_BWARPS 8
+#endif
+constexpr int kBProdWarps = JIG_BWARPS;  // B-producer (cp.async) warps
                                  // reach ~36 B/clk/SM vs ~28 with 4 (profiles/r01_gather_bench.txt)
 // Warps 6-15 except 9 and 13 are the B producers: warp w runs on SM
 // sub-partition w % 4, and sub-partition 1 is left to the MMA warp (1) and one
@@ -124,13 +128,24 @@ struct Problem {
 // (read with LDC, no dependent global load at kernel start).  Two sizes: a
 // small block for single products (cheap to launch) and a large one for grouped
 // launches.
-template <int MAXP, int MAXPIN, int MAXU>
+template <int MAXP, int MAXPIN, int MAXU, int MAXC = 1>
 struct ParamsT {
   static constexpr int kMaxProblems = MAXP;
   static constexpr int kMaxPin = MAXPIN;
   static constexpr int kMaxUnits = MAXU;
+  static constexpr int kMaxCta = MAXC;
   Problem pr[MAXP];
   int4 pin[MAXPIN];
+  // single products: the first unit of every CTA pre-decoded on the host, indexed
+  // by blockIdx.x (one level of parameter loads instead of a dependent chain):
+  // [c][0] = {panel, first C column, kb_lo, kb_hi}, [c][1] = {k-steps, dense
+  // k-steps, first k-step, first E block} of the panel
+  int4 ctab[MAXC][2];
+  int use_ctab;
+  // L2 prefetch of B at kernel start (single products with a small B): CTA c
+  // prefetches bytes [c*bpf_chunk, min(bpf_bytes, (c+1)*bpf_chunk)) of B, in
+  // parallel with the gather-list fetch that B's row gather depends on
+  int64_t bpf_bytes, bpf_chunk;
   // grouped launches: schedule position -> work piece, packed as
   //   problem (6 bits) | local unit (11) | piece (3) | pieces - 1 (3) | partial slot (9)
   // a unit split into `pieces` k-ranges (split-K inside the persistent launch)
@@ -144,7 +159,7 @@ struct ParamsT {
   int prefetch;  // 1: prefetch each unit's gather lists / metadata into L2 at unit start
   int dbg;       // developer timing experiments (JIGSAW_DBG, results invalid): 1 skip tcgen05.cp, 2 skip MMAs
 };
-using ParamsOne = ParamsT<1, 128, 1>;        // single product (~2.2 KB of parameters)
+using ParamsOne = ParamsT<1, 128, 1, 160>;   // single product (~7.3 KB of parameters)
 using ParamsGroup = ParamsT<64, 1024, 2048>; // grouped launch (~31 KB)
 constexpr int kMaxProblems = ParamsGroup::kMaxProblems;
 
@@ -213,6 +228,33 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   int i, lu, piece = 0, npieces = 1, pslot = 0;
   Work w;
   w.valid = true;
+  if constexpr (Prm::kMaxCta > 1 && !kPair) {
+    if (prm.use_ctab && (int)blockIdx.x == u * S + (int)rank) {  // the CTA's first unit, host-decoded
+      const int4 a = prm.ctab[blockIdx.x][0], b = prm.ctab[blockIdx.x][1];
+      w.Aimg = prm.pr[0].Aimg;
+      w.Eimg = prm.pr[0].Eimg;
+      w.G = prm.pr[0].G;
+      w.B = prm.pr[0].B;
+      w.C = prm.pr[0].C;
+      w.M = prm.pr[0].M;
+      w.N = prm.pr[0].N;
+      w.K = prm.pr[0].K;
+      w.p = a.x;
+      w.n0 = a.y;
+      w.kb_lo = a.z;
+      w.kb_hi = a.w;
+      w.nks = b.x;
+      w.ndk = b.y;
+      w.ks0 = b.z;
+      w.kb0 = b.w;
+      w.nkb_s = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
+      w.piece = 0;
+      w.npieces = 1;
+      w.pslot = 0;
+      w.row0 = (int64_t)w.p * kPanelRows;
+      return w;
+    }
+  }
   if (Prm::kMaxUnits > 1 && prm.use_ulist) {  // host-ordered schedule (longest pieces first)
     const uint32_t code = prm.ulist[u];
     if (code == kNoWork) {
@@ -339,27 +381,30 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     JIG_TRACE(0);
   }
 
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < C_::kStages; ++s) {
-      mbar_init(&full[s], 1 + 32 * C_::kWPG);  // A/E expect_tx arrival + the owning B group's cp.async arrivals
-      mbar_init(&empty[s], 1);
-      mbar_init(&pfull[s], 1);
-    }
-    for (int s = 0; s < C_::kGS; ++s) {
-      mbar_init(&gfull[s], 1);
-      mbar_init(&gempty[s], C_::kWPG);
-    }
-    for (int a = 0; a < 3; ++a) {
-      mbar_init(&tfull[a], 1);
-      mbar_init(&tempty[a], kPair ? 8 : 4);  // epilogue warps (of both CTAs of a pair)
-    }
-    mbar_init(recv_full, 1);
-    for (int i = 0; i < kSD; ++i) {
-      mbar_init(&rfull[i], 1);
-      mbar_init(&rempty[i], kBProdWarps + 1 + 4);  // B-producer warps + MMA + epilogue warps
+  // Barrier initialisation spread over the lanes of warp 0 (~50 barriers; one
+  // thread initialising them all costs ~0.5 us of kernel start).  The barriers
+  // are contiguous in shared memory: full, empty, gfull, gempty, tfull, tempty,
+  // recv_full, rfull, rempty, pfull.
+  if (warp == 0) {
+    constexpr int nb = 3 * C_::kStages + 2 * C_::kGS + 7 + 2 * kSD;
+    for (int i = lane; i < nb; i += 32) {
+      int k = i;
+      uint32_t cnt;
+      if (k < C_::kStages) cnt = 1 + 32 * C_::kWPG;        // full: A/E expect_tx + the B group's cp.async arrivals
+      else if ((k -= C_::kStages) < C_::kStages) cnt = 1;  // empty
+      else if ((k -= C_::kStages) < C_::kGS) cnt = 1;      // gfull
+      else if ((k -= C_::kGS) < C_::kGS) cnt = C_::kWPG;   // gempty
+      else if ((k -= C_::kGS) < 3) cnt = 1;                // tfull
+      else if ((k -= 3) < 3) cnt = kPair ? 8 : 4;          // tempty: epilogue warps (of both CTAs of a pair)
+      else if ((k -= 3) < 1) cnt = 1;                      // recv_full
+      else if ((k -= 1) < kSD) cnt = 1;                    // rfull
+      else if ((k -= kSD) < kSD) cnt = kBProdWarps + 1 + 4;  // rempty: B-producer warps + MMA + epilogue warps
+      else cnt = 1;                                        // pfull
+      mbar_init(full + i, cnt);
     }
     fence_barrier_init();
     fence_proxy_async();
+    if (lane == 0) JIG_TRACE(17);
   }
   // Parallel initial fill (before the block-wide sync, overlapping the TMEM
   // allocation): lane l of warp 0 issues the gather list of the CTA's first unit's
@@ -370,6 +415,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   Work w0;
   w0.valid = false;
   if (warp == 0) {
+    if (lane == 31 && prm.bpf_bytes > 0) {
+      const int64_t lo = (int64_t)blockIdx.x * prm.bpf_chunk;
+      if (lo < prm.bpf_bytes)
+        bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(prm.pr[0].B) + lo,
+                         (uint32_t)min(prm.bpf_chunk, prm.bpf_bytes - lo));
+      JIG_TRACE(22);
+    }
     __syncwarp();
     if (cluster_id < prm.nunits) {
       int h0 = 0;
@@ -380,6 +432,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         nG0 = min(nkb, C_::kGAhead + 1);
       }
     }
+    if (lane == 0) JIG_TRACE(18);
     if (lane < nG0) {
       const int kb = w0.kb_lo + lane;
       const int steps = w0.steps(kb);
@@ -487,7 +540,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         }
         if (u < 0) break;
         const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
-        if (mi == 0) JIG_TRACE(17);
         if (!wk.valid) continue;
         const int64_t kb0 = wk.kb0;
         if (prm.prefetch && wk.kb_hi > wk.kb_lo) {
@@ -498,7 +550,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         }
         for (int kb = wk.kb_lo + (mq == 1 ? nA0 : 0); kb < wk.kb_hi; ++kb) {
           g_issue_upto(mi + 1 + C_::kGAhead);
-          if (mi == 0) JIG_TRACE(18);
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
           const int64_t gks = wk.gks(kb);
@@ -1149,6 +1200,9 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
     const Format* fp = &f;
     return launch_group(&fp, &dB, &N, &dC, 1, s);
   }
+  prm.use_ctab = 0;
+  prm.bpf_bytes = 0;
+  prm.bpf_chunk = 0;
   if (const char* e = force_split) {  // test hook: force NT = 64 with split S
     const int fs = atoi(e);
     if (fs == 1 || fs == 2 || fs == 4 || fs == 8) {
@@ -1157,6 +1211,30 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
       const int64_t u64 = f.npanels * ((N + 63) / 64);
       grid = S > 1 ? (int)(u64 * S) : (int)std::min<int64_t>(u64, spmm_num_sms());
     }
+  }
+  // host-decoded first unit of every CTA (see ParamsT::ctab)
+  if (grid <= ParamsOne::kMaxCta && !getenv("JIGSAW_NO_CTAB")) {
+    const int64_t nkb_units = f.npanels * ((N + NT - 1) / NT);
+    for (int c = 0; c < grid; ++c) {
+      const int u = S > 1 ? c / S : c, r = S > 1 ? c % S : 0;
+      if (u >= nkb_units) {
+        prm.ctab[c][0] = make_int4(0, 0, 0, 0);
+        prm.ctab[c][1] = make_int4(0, 0, 0, 0);
+        continue;
+      }
+      const int p = (int)(u % f.npanels), n0 = (int)(u / f.npanels) * NT;
+      const int4 pi = f.pin[p];  // {k-steps, first k-step, first E block, dense k-steps}
+      const int nkb = (pi.x + 3) / 4 + (pi.w + 3) / 4;
+      prm.ctab[c][0] = make_int4(p, n0, r * nkb / S, (r + 1) * nkb / S);
+      prm.ctab[c][1] = make_int4(pi.x, pi.w, pi.y, pi.z);
+    }
+    prm.use_ctab = 1;
+  }
+  // small B: prefetch it into L2 at kernel start, spread over the CTAs
+  const int64_t bbytes = f.K * N * 2;
+  if (bbytes <= ((int64_t)16 << 20) && !getenv("JIGSAW_NO_BPF")) {
+    prm.bpf_bytes = bbytes;
+    prm.bpf_chunk = ((bbytes + grid - 1) / grid + 255) & ~int64_t(255);
   }
   return launch_params(prm, NT, S, grid, f.device, pair, s);
 }
@@ -1217,6 +1295,9 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
     const int n = std::min(kMaxProblems, count - i0);
     prm.nprob = n;
     prm.use_pin = 1;
+    prm.use_ctab = 0;
+    prm.bpf_bytes = 0;
+    prm.bpf_chunk = 0;
     int64_t u128 = 0, u64 = 0;
     for (int i = 0; i < n; ++i) {
       fill_problem(prm, i, *fs[i0 + i], Bs[i0 + i], Ns[i0 + i], Cs[i0 + i]);
@@ -1260,19 +1341,22 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       for (int i = 0; i < n; ++i) {
         const Format& f = *fs[i0 + i];
         const int ntn = (int)((Ns[i0 + i] + NT - 1) / NT);
-        for (int t = 0; t < ntn; ++t)
-          for (int p = 0; p < f.npanels; ++p) {
+        for (int p = 0; p < f.npanels; ++p)
+          for (int t = 0; t < ntn; ++t) {  // N tiles of a panel adjacent: they share its A stream
             const int nkb = (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
             us.push_back({nkb + 1, nkb, ((uint32_t)i << 26) | ((uint32_t)(t * f.npanels + p) << 15)});
             total += nkb + 1;
           }
       }
+      // JIGSAW_SCHED=loc: locality order (problem, panel, N tile) dealt round-robin,
+      // no cost sort and no split pieces (developer experiment)
+      const bool loc = getenv("JIGSAW_SCHED") && std::string(getenv("JIGSAW_SCHED")) == "loc";
       const int64_t target = std::max<int64_t>(4, (total + slots_max - 1) / slots_max);
-      const bool allow_split = !getenv("JIGSAW_NO_PIECES");
+      const bool allow_split = !getenv("JIGSAW_NO_PIECES") && !loc;
       thread_local std::vector<std::pair<int, uint32_t>> order;
       order.clear();
       int pslots = 0;
-      std::stable_sort(us.begin(), us.end(), [](const U& a, const U& b) { return a.cost > b.cost; });
+      if (!loc) std::stable_sort(us.begin(), us.end(), [](const U& a, const U& b) { return a.cost > b.cost; });
       for (const U& x : us) {
         int np = 1;
         if (allow_split && x.cost > target + target / 4 && x.nkb >= 8) {
@@ -1297,8 +1381,9 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
           pslots = 0;
         }
       }
-      std::stable_sort(order.begin(), order.end(),
-                       [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
+      if (!loc)
+        std::stable_sort(order.begin(), order.end(),
+                         [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
       const int nslots = (int)std::min<int64_t>(slots_max, (int64_t)order.size());
       npieces_total = (int)order.size();
       if (!pair) {
@@ -1314,7 +1399,14 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
         auto cmp = [](const std::pair<int64_t, int>& a, const std::pair<int64_t, int>& b) { return a > b; };
         std::make_heap(heap.begin(), heap.end(), cmp);
         size_t maxlen = 0;
+        size_t k_rr = 0;
         for (const auto& o : order) {
+          if (loc) {  // round-robin: consecutive (same-panel) units run concurrently
+            const int c = (int)(k_rr++ % nslots);
+            q[c].push_back(o.second);
+            maxlen = std::max(maxlen, q[c].size());
+            continue;
+          }
           std::pop_heap(heap.begin(), heap.end(), cmp);
           auto& h = heap.back();
           q[h.second].push_back(o.second);

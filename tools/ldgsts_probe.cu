@@ -29,7 +29,7 @@ __global__ void __launch_bounds__(544, 1) probe(const uint16_t* B, int K, int ld
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int wpg = nw / ng;  // warps per group
+  const int wpg = ng > 0 ? nw / ng : nw;  // warps per group
   const int stage_bytes = kRows * rowbytes;
   if (threadIdx.x == 0) {
     for (int s = 0; s < stages; ++s) {
@@ -50,6 +50,38 @@ __global__ void __launch_bounds__(544, 1) probe(const uint16_t* B, int K, int ld
         if (++stage == stages) { stage = 0; ph ^= 1; }
       }
       out[blockIdx.x] = clock64() - t0;
+    }
+  } else if (warp - 1 < nw && ng < 0) {
+    // one group, completion tracked with commit_group / wait_group: up to D = -ng
+    // k-blocks in flight per warp, then a plain arrive for the oldest
+    const int D = -ng, w = warp - 1;
+    const int lpr = rowbytes / 16, rpi = 32 / lpr;
+    const int c = lane % lpr;
+    const int rows_per_warp = kRows / nw;
+    for (int kb = 0; kb < KB + D - 1; ++kb) {
+      if (kb < KB) {
+        const int stage = kb % stages;
+        const uint32_t ph = (uint32_t)((kb / stages) & 1);
+        mbar_wait(&empty[stage], ph ^ 1);
+        uint8_t* st = sm + stage * stage_bytes;
+        for (int r0 = w * rows_per_warp; r0 < (w + 1) * rows_per_warp; r0 += rpi) {
+          const int row = r0 + lane / lpr;
+          const int gr = hrow(blockIdx.x, kb, row, K);
+          cp_async_16(st + row * rowbytes + ((c ^ (row & 7)) & (lpr - 1)) * 16, B + (size_t)gr * ldb + 8 * c, 16);
+        }
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      const int old = kb - (D - 1);
+      if (old >= 0) {
+        switch (D) {
+          case 1: asm volatile("cp.async.wait_group 0;" ::: "memory"); break;
+          case 2: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
+          case 3: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
+          default: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
+        }
+        fence_proxy_async();
+        mbar_arrive(&full[old % stages]);
+      }
     }
   } else if (warp - 1 < nw) {
     const int w = warp - 1, g = w / wpg, wi = w % wpg;
@@ -84,6 +116,7 @@ int main() {
   struct Case { int nw, ng, rowbytes, stages; };
   std::vector<Case> cases = {
       // groups <= stages (a group's parity waits must stay within one phase)
+      {8, -2, 64, 6}, {8, -4, 64, 6}, {8, -2, 256, 4}, {8, -4, 256, 4}, {16, -4, 256, 4},
       {8, 1, 64, 6},  {8, 2, 64, 6},  {8, 4, 64, 6},  {12, 6, 64, 6}, {16, 4, 64, 6},
       {8, 1, 128, 6}, {8, 2, 128, 6}, {8, 4, 128, 6}, {16, 4, 128, 6}, {12, 6, 128, 6},
       {8, 1, 256, 4}, {8, 2, 256, 4}, {8, 4, 256, 4}, {16, 2, 256, 4}, {16, 4, 256, 4},

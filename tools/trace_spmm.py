@@ -15,7 +15,7 @@ import paper_conf_icpp_zhanglyfyllq24_b200 as jig  # noqa: E402
 
 NAMES = {1: "setup", 2: "A/E issued", 3: "B issued", 4: "1st stage full", 5: "last MMA commit",
          6: "acc ready", 7: "sends done", 8: "recv ready", 9: "stores done", 10: "exit sync",
-         11: "dealloc", 16: "AE fetched", 17: "AE decoded", 18: "G issued", 19: "B decoded",
+         11: "dealloc", 16: "AE fetched", 17: "bar init done", 18: "fill decoded", 22: "B prefetch issued", 19: "B decoded",
          20: "G landed", 21: "MMA decoded", 23: "exit barrier"}
 
 
