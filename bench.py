@@ -374,24 +374,31 @@ def main():
     except Exception:
         pass
 
-    # per-point detail: jigsaw vs cuBLAS (torch.matmul on the dense fp16 A), median of reps
+    # per-point detail: jigsaw vs cuBLAS (torch.matmul on the dense fp16 A).  Each
+    # call's device time in a stream of back-to-back kernels, L2 flushed before
+    # every call: [graph of R x (flush, call)] - [graph of R x (flush)], / R (median
+    # of reps) -- the event clock here moves in ~2 us steps, too coarse for
+    # single-call events; the difference over R calls resolves ~0.1 us.
     detail = []
     cublas_ms = jig_ms = 0.0
     if not args.no_cublas:
-        reps = 20
+        reps, R = 7, 8
 
         def graphed(fn):
-            fn()
+            if fn is not None:
+                fn()
             torch.cuda.synchronize()
             g = torch.cuda.CUDAGraph()
             with torch.cuda.graph(g):
-                fn()
+                for _ in range(R):
+                    flush.zero_()
+                    if fn is not None:
+                        fn()
             return g
 
         def timeit(g):
             ts = []
             for _ in range(reps):
-                flush.zero_()          # ~40 us of GPU work: hides the host-side replay latency
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(stream)
                 g.replay()
@@ -399,10 +406,12 @@ def main():
                 e1.synchronize()
                 ts.append(e0.elapsed_time(e1))
             return float(np.median(ts))
+        g_flush = graphed(None)
         for i, (M, K, v, s, N) in enumerate(points):
-            tj = timeit(graphed(lambda: hs[i].spmm(dB[i], C=dC[i])))
+            t0 = timeit(g_flush)
+            tj = (timeit(graphed(lambda: hs[i].spmm(dB[i], C=dC[i]))) - t0) / R
             Cref = torch.empty_like(dC[i])
-            tc = timeit(graphed(lambda: torch.matmul(dA[i], dB[i], out=Cref)))
+            tc = (timeit(graphed(lambda: torch.matmul(dA[i], dB[i], out=Cref))) - t0) / R
             cublas_ms += tc
             jig_ms += tj
             detail.append({"M": M, "K": K, "v": v, "s": s, "N": N, "jigsaw_us": tj * 1e3,
@@ -493,7 +502,7 @@ def main():
                    "speedup_total_time": (cublas_ms / jig_ms) if jig_ms else None,
                    "speedup_geomean_by_v_s": speed_gm,
                    "cublas_eff_tflops": (eff_flops / (cublas_ms * 1e-3) / 1e12) if cublas_ms else None,
-                   "how": "torch.matmul fp16 (cuBLAS) on the dense A: per matrix (graph replay, median of 20) and the whole batch as one CUDA graph (median of 30), same L2 flush"},
+                   "how": "torch.matmul fp16 (cuBLAS) on the dense A: per matrix as [graph of 8 x (L2 flush, call)] - [graph of 8 x (L2 flush)], / 8 (median of 7), and the whole batch as one CUDA graph (median of 30), same L2 flush"},
         "reorder_ms_total": reorder_ms,
     }
     if args.detail and rank == 0:
