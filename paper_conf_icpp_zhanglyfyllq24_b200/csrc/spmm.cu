@@ -120,6 +120,7 @@ struct Problem {
   __half* C;
   int64_t M, N, K;
   int64_t planeA, planeE;  // bytes between the A / E planes of the two 128-row halves (P = 256)
+  int64_t boff;  // offset of this problem's B in the concatenation of all B's (L2 prefetch)
   int npanels;
   int unit0;  // first global work unit of this problem
   int pin0;   // offset of this problem's panels in ParamsT::pin (if use_pin)
@@ -142,9 +143,10 @@ struct ParamsT {
   // k-steps, first k-step, first E block} of the panel
   int4 ctab[MAXC][2];
   int use_ctab;
-  // L2 prefetch of B at kernel start (single products with a small B): CTA c
-  // prefetches bytes [c*bpf_chunk, min(bpf_bytes, (c+1)*bpf_chunk)) of B, in
-  // parallel with the gather-list fetch that B's row gather depends on
+  // L2 prefetch of B at kernel start (when all B's of the launch fit in L2 with
+  // room to spare): CTA c prefetches bytes [c*bpf_chunk, (c+1)*bpf_chunk) of the
+  // concatenation of the problems' B matrices (bpf_bytes in total), in parallel
+  // with the gather-list fetches the B row gathers depend on
   int64_t bpf_bytes, bpf_chunk;
   // grouped launches: schedule position -> work piece, packed as
   //   problem (6 bits) | local unit (11) | piece (3) | pieces - 1 (3) | partial slot (9)
@@ -415,12 +417,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   Work w0;
   w0.valid = false;
   if (warp == 0) {
-    if (lane == 31 && prm.bpf_bytes > 0) {
-      const int64_t lo = (int64_t)blockIdx.x * prm.bpf_chunk;
-      if (lo < prm.bpf_bytes)
-        bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(prm.pr[0].B) + lo,
-                         (uint32_t)min(prm.bpf_chunk, prm.bpf_bytes - lo));
-      JIG_TRACE(22);
+    if (prm.bpf_bytes > 0) {
+      const int64_t lo = (int64_t)blockIdx.x * prm.bpf_chunk, hi = min(prm.bpf_bytes, lo + prm.bpf_chunk);
+      for (int i = 31 - lane; i < prm.nprob; i += 32) {  // lane 31 takes problem 0
+        const int64_t b0 = prm.pr[i].boff, b1 = b0 + prm.pr[i].K * prm.pr[i].N * 2;
+        const int64_t x0 = max(lo, b0), x1 = min(hi, b1);
+        if (x0 < x1)
+          bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(prm.pr[i].B) + (x0 - b0), (uint32_t)(x1 - x0));
+      }
+      if (lane == 31) JIG_TRACE(22);
     }
     __syncwarp();
     if (cluster_id < prm.nunits) {
@@ -1137,6 +1142,7 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
   P.N = N;
   P.K = f.K;
   P.npanels = (int)f.npanels;
+  P.boff = i == 0 ? 0 : prm.pr[i - 1].boff + prm.pr[i - 1].K * prm.pr[i - 1].N * 2;
 }
 
 int g_trace_ctas = 0;
@@ -1203,13 +1209,14 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   prm.use_ctab = 0;
   prm.bpf_bytes = 0;
   prm.bpf_chunk = 0;
-  if (const char* e = force_split) {  // test hook: force NT = 64 with split S
+  if (const char* e = force_split) {  // test hook: force split S (NT = 64, or 32 with JIGSAW_FORCE_NT=32)
     const int fs = atoi(e);
     if (fs == 1 || fs == 2 || fs == 4 || fs == 8) {
-      NT = 64;
+      const char* fn = getenv("JIGSAW_FORCE_NT");
+      NT = (fn && atoi(fn) == 32) ? 32 : 64;
       S = fs;
-      const int64_t u64 = f.npanels * ((N + 63) / 64);
-      grid = S > 1 ? (int)(u64 * S) : (int)std::min<int64_t>(u64, spmm_num_sms());
+      const int64_t un = f.npanels * ((N + NT - 1) / NT);
+      grid = S > 1 ? (int)(un * S) : (int)std::min<int64_t>(un, spmm_num_sms());
     }
   }
   // host-decoded first unit of every CTA (see ParamsT::ctab)
@@ -1232,7 +1239,7 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   }
   // small B: prefetch it into L2 at kernel start, spread over the CTAs
   const int64_t bbytes = f.K * N * 2;
-  if (bbytes <= ((int64_t)16 << 20) && !getenv("JIGSAW_NO_BPF")) {
+  if (bbytes <= ((int64_t)16 << 20) && getenv("JIGSAW_BPF")) {  // opt-in: measured 0.1-0.2 us slower
     prm.bpf_bytes = bbytes;
     prm.bpf_chunk = ((bbytes + grid - 1) / grid + 255) & ~int64_t(255);
   }
@@ -1318,7 +1325,7 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
     } else {
       NT = u128 >= 2 * sms ? 128 : 64;
       if ((u256 >= sms && kbs >= 24 * npan && force == 0) || force == 256) NT = 256;
-      if (force == 128 || force == 64) NT = force;
+      if (force == 128 || force == 64 || force == 32) NT = force;
     }
     const int64_t units = NT == 256 ? u256 : NT == 128 ? u128 : u64;
     const int slots_max = pair ? sms / 2 : sms;                  // CTAs or CTA pairs
@@ -1437,6 +1444,18 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       slots = nslots;
     }
     const int grid = pair ? 2 * slots : slots;
+    // all B's of the launch small enough to sit in L2 next to the A stream:
+    // prefetch them at kernel start (JIGSAW_GROUP_BPF = cap in MB, 0 disables)
+    {
+      int64_t bsum = 0;
+      for (int i = 0; i < n; ++i) bsum += fs[i0 + i]->K * Ns[i0 + i] * 2;
+      const char* e = getenv("JIGSAW_GROUP_BPF");
+      const int64_t cap = (int64_t)(e ? atoll(e) : 0) << 20;  // measured slower for C2 (44.7 vs 41.0 us): off
+      if (cap > 0 && bsum <= cap) {
+        prm.bpf_bytes = bsum;
+        prm.bpf_chunk = ((bsum + grid - 1) / grid + 255) & ~int64_t(255);
+      }
+    }
     jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, pair, s, npieces_total);
     if (st != JIGSAW_SUCCESS) return st;
   }

@@ -236,6 +236,36 @@ def test_spmm_kernel_variants(force, M, K, v, s, N, monkeypatch):
         assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
 
 
+@pytest.mark.parametrize("force", ["1", "2", "4"])
+@pytest.mark.parametrize("M,K,v,s,N", [(512, 2048, 4, 0.9, 256), (384, 700, 8, 0.8, 200),
+                                       (256, 96, 2, 0.95, 40), (2048, 512, 8, 0.7, 104)])
+def test_spmm_nt32_variants(force, M, K, v, s, N, monkeypatch):
+    """32-column tiles (the latency path of small single products; B staged in
+    half of a 64-column SW128 chunk, N = 32 MMAs) with split-K S = 1/2/4, ragged
+    N tails (N % 32 != 0), single and grouped launches, against the oracle;
+    integer-valued inputs bit-exact."""
+    monkeypatch.setenv("JIGSAW_FORCE_NT", "32")
+    monkeypatch.setenv("JIGSAW_FORCE_SPLIT", force)
+    A = synth.vector_sparse(M, K, v, s, 13)
+    B = synth.dense_b(K, N, 13)
+    h = jig.reorder(_dev(A), v)
+    spmm_check(_host(h.spmm(_dev(B))), A, B)
+    Ai = synth.vector_sparse(M, K, v, s, 14, kind="int")
+    Bi = synth.dense_b(K, N, 14, kind="int")
+    hi = jig.reorder(_dev(Ai), v)
+    Ci = _host(hi.spmm(_dev(Bi)))
+    torch.cuda.synchronize()
+    C_ref, _ = oracle.spmm(Ai, Bi)
+    if np.abs(C_ref).max() <= 2048:
+        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+    monkeypatch.delenv("JIGSAW_FORCE_SPLIT")
+    dC = [torch.empty((M, N), dtype=torch.float16, device="cuda") for _ in range(2)]
+    jig.spmm_batched([h, hi], [_dev(B), _dev(Bi)], dC)
+    torch.cuda.synchronize()
+    spmm_check(_host(dC[0]), A, B)
+    spmm_check(_host(dC[1]), Ai, Bi)
+
+
 def test_grouped_launch_many_mixed_problems():
     """jigsaw_spmm_batched: one grouped persistent launch per 64 products; 70 mixed
     shapes / N / sparsities (incl. an all-zero matrix) against the oracle."""
