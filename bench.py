@@ -2,7 +2,8 @@
 """bench.py -- SpMM effective TFLOP/s and speedup vs cuBLAS fp16 GEMM vs sparsity
 (BASELINE.json metric) for the Jigsaw hot path on B200.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2|c4|c1|c5b] [--impl jigsaw|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2|c1|c3|c4|c5a|c5b|venom]
+                  [--impl jigsaw|reference]
 
 A STEP is one pass of the SpMM hot path over one batch of synthetic matrices
 with the prepared formats resident in HBM (the paper times the kernel only and
@@ -67,7 +68,29 @@ def workload(name: str):
     if name == "c5b":
         return [(4096, 4096, 8, 0.90, 16384)], ("C5b: 4096x4096 v=8 s=.90 N=16384, B/C column-sharded "
                                                 "across the GPUs"), "strong"
+    if name == "venom":
+        # SURVEY §8f f4 (Table 3): matrices already pruned to V:2:Mb,
+        # computed without a reorder step being needed; v = 1 (the format is
+        # v-independent), s = 1 - 2/Mb
+        pts = [(M, K, 1, 1.0 - 2.0 / mb, N) for (M, K, V, mb, N) in synth.venom_points()]
+        return pts, ("f4: VENOM-style V:2:Mb pruned 4096x4096, V=32/64/128, Mb=12/20/40/100 "
+                     "(s=.833/.90/.95/.98), N=2048 (12 matrices), vs cuBLAS and cuSPARSELt"), "weak"
     raise SystemExit(f"unknown workload {name}")
+
+
+def make_a(name: str, i: int, M: int, K: int, v: int, s: float, seed: int) -> np.ndarray:
+    """A of point i of workload `name` (uint16 fp16 bits)."""
+    if name == "venom":
+        _, _, V, mb, _ = synth.venom_points()[i]
+        return synth.venom(M, K, V, mb, seed)
+    return synth.vector_sparse(M, K, v, s, seed)
+
+
+def point_tag(name: str, i: int, v: int, s: float) -> str:
+    if name == "venom":
+        _, _, V, mb, _ = synth.venom_points()[i]
+        return f"V{V}_Mb{mb}"
+    return f"v{v}_s{int(round(s * 100))}"
 
 
 def local_jobs(name, points, rank, world):
@@ -172,7 +195,7 @@ def run_reference(args):
         os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
     except Exception:
         cores = 1
-    mats = [(synth.vector_sparse(M, K, v, s, point_seed(i, 0)), synth.dense_b(K, N, point_seed(i, 0)))
+    mats = [(make_a(args.workload, i, M, K, v, s, point_seed(i, 0)), synth.dense_b(K, N, point_seed(i, 0)))
             for i, (M, K, v, s, N) in enumerate(points)]
     # size the per-step sample so the whole run stays within ~2 minutes
     budget = max(0.2, min(4.0, 100.0 / max(1, args.steps + args.warmup)))
@@ -274,8 +297,8 @@ def main():
     mats, hs, dB, dC, dA = [], [], [], [], []
     reorder_ms = 0.0
     alg_bytes = exec_flops = eff_flops = 0
-    for (M, K, v, s, N, seed, n0, n1) in jobs:
-        A = synth.vector_sparse(M, K, v, s, seed)
+    for ji, (M, K, v, s, N, seed, n0, n1) in enumerate(jobs):
+        A = make_a(args.workload, ji, M, K, v, s, seed)
         B = synth.dense_b(K, N, seed)
         if (n0, n1) != (0, N):
             B = np.ascontiguousarray(B[:, n0:n1])
@@ -380,7 +403,17 @@ def main():
     # of reps) -- the event clock here moves in ~2 us steps, too coarse for
     # single-call events; the difference over R calls resolves ~0.1 us.
     detail = []
-    cublas_ms = jig_ms = 0.0
+    cublas_ms = jig_ms = cslt_ms = 0.0
+    # cuSPARSELt (torch._cslt_*) on natively 2:4 inputs (the f4 workload): the
+    # library 2:4 SpMM, which cannot skip all-zero columns
+    cslt_A, cslt_err = None, None
+    if not args.no_cublas and args.workload == "venom":
+        try:
+            cslt_A = [torch._cslt_compress(a) for a in dA]
+            torch._cslt_sparse_mm(cslt_A[0], dB[0])
+            torch.cuda.synchronize()
+        except Exception as e:  # library without an sm_100 build, or API absent
+            cslt_A, cslt_err = None, f"{type(e).__name__}: {str(e).splitlines()[0][:200]}"
     if not args.no_cublas:
         reps, R = 7, 8
 
@@ -414,9 +447,15 @@ def main():
             tc = (timeit(graphed(lambda: torch.matmul(dA[i], dB[i], out=Cref))) - t0) / R
             cublas_ms += tc
             jig_ms += tj
-            detail.append({"M": M, "K": K, "v": v, "s": s, "N": N, "jigsaw_us": tj * 1e3,
-                           "cublas_us": tc * 1e3, "speedup": tc / tj,
-                           "eff_tflops": 2 * M * N * K / (tj * 1e-3) / 1e12})
+            d = {"M": M, "K": K, "v": v, "s": s, "N": N, "tag": point_tag(args.workload, i, v, s),
+                 "jigsaw_us": tj * 1e3, "cublas_us": tc * 1e3, "speedup": tc / tj,
+                 "eff_tflops": 2 * M * N * K / (tj * 1e-3) / 1e12}
+            if cslt_A is not None and cslt_A[i] is not None:
+                ts = (timeit(graphed(lambda: torch._cslt_sparse_mm(cslt_A[i], dB[i]))) - t0) / R
+                d["cusparselt_us"] = ts * 1e3
+                d["speedup_vs_cusparselt"] = ts / tj
+                cslt_ms += ts
+            detail.append(d)
     # step-level comparison: the same batch as one CUDA graph of per-matrix cuBLAS
     # calls, and of per-matrix jigsaw_spmm calls (36 launches), same flush policy
     def step_ms(g, reps=30):
@@ -443,9 +482,30 @@ def main():
     cublas_step_ms = step_ms(g_cub)
     unbatched_step_ms = step_ms(graph_unb)
     speed = {}
+    speed_cs = {}
     for d in detail:
-        speed.setdefault(f"v{d['v']}_s{int(round(d['s'] * 100))}", []).append(d["speedup"])
+        speed.setdefault(d["tag"], []).append(d["speedup"])
+        if "speedup_vs_cusparselt" in d:
+            speed_cs.setdefault(d["tag"], []).append(d["speedup_vs_cusparselt"])
     speed_gm = {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(speed.items())}
+    cslt = None
+    if cslt_A is not None:
+        def cslt_step():
+            for a, b, o in zip(cslt_A, dB, outs):
+                o.copy_(torch._cslt_sparse_mm(a, b))
+        cslt_step()
+        torch.cuda.synchronize()
+        g_cs = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g_cs):
+            cslt_step()
+        cs_ms = step_ms(g_cs)
+        cslt = {"step_ms": cs_ms, "speedup_step": cs_ms / ms_per_step,
+                "speedup_total_time": (cslt_ms / jig_ms) if jig_ms else None,
+                "speedup_geomean_by_point": {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(speed_cs.items())},
+                "how": "torch._cslt_compress / torch._cslt_sparse_mm (cuSPARSELt 2:4 SpMM) on the natively 2:4 A; "
+                       "per matrix like cuBLAS; step = one CUDA graph of the batch (+ a copy into C per matrix)"}
+    elif cslt_err:
+        cslt = {"unavailable": cslt_err}
 
     # e2e through the C ABI with host buffers (every step: B in, SpMM, C out)
     pin_B = [torch.from_numpy(B.view(np.int16)).pin_memory().numpy().view(np.uint16) for (_, B) in mats]
@@ -505,6 +565,8 @@ def main():
                    "how": "torch.matmul fp16 (cuBLAS) on the dense A: per matrix as [graph of 8 x (L2 flush, call)] - [graph of 8 x (L2 flush)], / 8 (median of 7), and the whole batch as one CUDA graph (median of 30), same L2 flush"},
         "reorder_ms_total": reorder_ms,
     }
+    if cslt is not None:
+        line["cusparselt"] = cslt
     if args.detail and rank == 0:
         for d in detail:
             print(json.dumps(d), file=sys.stderr)

@@ -82,6 +82,35 @@ def nm24(M: int, K: int, seed: int) -> np.ndarray:
     return np.where(keep.reshape(M, K), u, 0.0).astype(np.float16).view(np.uint16)
 
 
+def venom(M: int, K: int, V: int, Mb: int, seed: int, kind: str = "uniform") -> np.ndarray:
+    """VENOM-style V:2:Mb matrix (the "pruned matrices ... computed directly
+    without reordering" of P:321-337 §4.5, Table 3): rows in
+    blocks of V, columns in blocks of Mb; in every V x Mb block 4 columns are
+    selected (the same for all V rows of the block) and every row keeps 2 of
+    those 4 (2:4), so the density is 2 / Mb.  A last, narrower column block
+    selects min(4, width) columns and keeps min(2, that) per row.  Values as in
+    vector_sparse.  With 4 | Mb every aligned group of 4 columns lies inside one
+    block, so the matrix is natively 2:4 (what cuSPARSELt accepts)."""
+    if M % V:
+        raise ValueError("M must be a multiple of V")
+    rng = np.random.default_rng(seed)
+    keep = np.zeros((M, K), dtype=bool)
+    for r0 in range(0, M, V):
+        for c0 in range(0, K, Mb):
+            w = min(Mb, K - c0)
+            sel = c0 + np.sort(rng.choice(w, size=min(4, w), replace=False))
+            nk = min(2, len(sel))
+            pick = np.argsort(rng.random((V, len(sel))), axis=1)[:, :nk]
+            keep[r0 + np.arange(V)[:, None], sel[pick]] = True
+    rv = np.random.default_rng(seed + 7919)
+    if kind == "int":
+        vals = rv.choice(np.array([-2.0, -1.0, 1.0, 2.0]), size=(M, K))
+    else:
+        u = rv.uniform(-1.0, 1.0, size=(M, K))
+        vals = np.where(np.abs(u) < 2.0 ** -6, np.copysign(2.0 ** -6, u), u)
+    return np.where(keep, vals, 0.0).astype(np.float16).view(np.uint16)
+
+
 # --- the paper's workload families (SURVEY §8d, BASELINE.json configs) ---------
 
 C1 = dict(M=256, K=256, v=4, s=0.80, N=64)
@@ -106,6 +135,22 @@ C4_N = 2048
 def c2_points():
     """The 36 (M, K, v, s, N) points of configs[1] (DLMC transformer, N=256)."""
     return [(M, K, v, s, C2_N) for (M, K) in C2_SHAPES for v in C2_V for s in C2_S]
+
+
+# f4 (SURVEY §8f, P:321-337 Table 3): V:2:Mb matrices, V in {32, 64, 128}, block
+# widths Mb = 12 / 20 / 40 / 100 (sparsity 83.3 / 90 / 95 / 98 %; 4 | Mb so each
+# matrix is natively 2:4 for the cuSPARSELt baseline), Llama-shaped 4096 x 4096,
+# N = 2048
+VENOM_SHAPE = (4096, 4096)
+VENOM_V = [32, 64, 128]
+VENOM_MB = [12, 20, 40, 100]
+VENOM_N = 2048
+
+
+def venom_points():
+    """(M, K, V, Mb, N) of the f4 workload."""
+    M, K = VENOM_SHAPE
+    return [(M, K, V, mb, VENOM_N) for V in VENOM_V for mb in VENOM_MB]
 
 
 def c4_points():

@@ -33,3 +33,19 @@ def test_weak_scaling_jobs_differ_by_rank():
     pts, _, _ = bench.workload("c2")
     a, b = bench.local_jobs("c2", pts, 0, 2), bench.local_jobs("c2", pts, 1, 2)
     assert len(a) == len(b) == 36 and {j[5] for j in a}.isdisjoint({j[5] for j in b})
+
+
+def test_venom_workload_points_are_natively_24():
+    """f4 workload: every point's A is V:2:Mb with 4 | Mb, so it is
+    2:4 in natural column order (the cuSPARSELt baseline's input); s = 1 - 2/Mb."""
+    import synth
+    pts, desc, scaling = bench.workload("venom")
+    assert len(pts) == len(synth.venom_points()) == 12 and scaling == "weak"
+    for i, (M, K, v, s, N) in enumerate(pts):
+        _, _, V, mb, _ = synth.venom_points()[i]
+        assert mb % 4 == 0 and abs(s - (1 - 2 / mb)) < 1e-12
+        assert bench.point_tag("venom", i, v, s) == f"V{V}_Mb{mb}"
+    A = synth.venom(256, 480, 32, 20, 5)
+    nz = (A & 0x7FFF) != 0
+    assert nz.reshape(256, -1, 4).sum(axis=2).max() <= 2
+    assert abs(nz.mean() - 2 / 20) < 1e-12

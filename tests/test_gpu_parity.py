@@ -95,6 +95,31 @@ def test_reorder_bit_exact_and_spmm(M, K, v, s, N, kind, seed):
     h.free()
 
 
+@pytest.mark.parametrize("M,K,V,Mb,N,P", [(512, 1000, 128, 20, 256, 128), (384, 600, 32, 12, 200, 128),
+                                          (512, 2048, 64, 100, 256, 128), (512, 800, 256, 40, 256, 256)])
+def test_venom_matrices(M, K, V, Mb, N, P):
+    """VENOM-style V:2:Mb matrices.  GPU format
+    bit-exact vs the oracle (identity reorder when P | V), C within tolerance,
+    integer-valued inputs bit-exact."""
+    A = synth.venom(M, K, V, Mb, 41)
+    B = synth.dense_b(K, N, 41)
+    h = jig.reorder(_dev(A), 1, panel_rows=P)
+    g = h.export()
+    ref = oracle.reorder(A, P=P)
+    assert_format_equal(g, ref)
+    if V % P == 0:
+        assert h.info()["evictions"] == 0
+    spmm_check(_host(h.spmm(_dev(B))), A, B)
+    Ai = synth.venom(M, K, V, Mb, 42, kind="int")
+    Bi = synth.dense_b(K, N, 42, kind="int")
+    hi = jig.reorder(_dev(Ai), 1, panel_rows=P)
+    Ci = _host(hi.spmm(_dev(Bi)))
+    torch.cuda.synchronize()
+    C_ref, _ = oracle.spmm(Ai, Bi)
+    if np.abs(C_ref).max() <= 2048:
+        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+
+
 @pytest.mark.parametrize("seed", [11, 12])
 def test_spmm_integer_inputs_bit_exact(seed):
     """Integer-valued A in {+-1,+-2}, B in {-2..2}, |C| <= 2048: every fp32 partial

@@ -81,6 +81,45 @@ def test_already_24_needs_no_reorder(seed):
     _check(A, f)
 
 
+@pytest.mark.parametrize("V,Mb,K", [(128, 12, 192), (128, 20, 400), (256, 40, 400), (128, 100, 256)])
+def test_venom_aligned_needs_no_reorder(V, Mb, K):
+    """SURVEY §8f f4 (§4.5): a V:2:Mb matrix with V a multiple of the
+    panel height and 4 | Mb is 2:4 inside every block of its compacted columns,
+    so CR1 must leave it as it is -- S_p = the 4 selected columns of every
+    column block in ascending order, identity permutation on every tile, no
+    eviction, T_p = ceil(K_p / 16) -- and the format decodes to A."""
+    A = synth.venom(256, K, V, Mb, 31)
+    f = oracle.reorder(A, P=128)
+    nblk = -(-K // Mb)
+    for p in range(len(f.T)):
+        blk = A[p * 128:(p + 1) * 128]
+        cols = np.flatnonzero(((blk & 0x7FFF) != 0).any(axis=0))
+        assert len(cols) == 4 * nblk - (4 - min(4, K - (nblk - 1) * Mb))  # 4 selected per block
+        assert f.T[p] == -(-len(cols) // 16)
+        toff = f.tile_off
+        assert int(f.nevict[toff[p]:toff[p + 1]].sum()) == 0
+        for t in range(toff[p], toff[p + 1]):
+            n_real = int((f.col_idx[t] >= 0).sum())
+            assert f.perm[t][:n_real].tolist() == list(range(n_real))
+        got = f.col_idx[toff[p]:toff[p + 1]].reshape(-1)
+        assert np.array_equal(got[got >= 0], cols)
+    _check(A, f)
+
+
+@pytest.mark.parametrize("V,Mb", [(32, 12), (64, 20), (32, 100)])
+def test_venom_short_vectors_reordered_validly(V, Mb):
+    """V:2:Mb with V < P: a 128-row panel spans several V-blocks with different
+    column selections, so the union is no longer 2:4 in order and CR1 has real
+    work; the format must stay valid, bounded and decode to A."""
+    A = synth.venom(256, 400, V, Mb, 32)
+    f = oracle.reorder(A, P=128)
+    _check(A, f)
+    for p in range(len(f.T)):
+        blk = A[p * 128:(p + 1) * 128]
+        Kp = int(((blk & 0x7FFF) != 0).any(axis=0).sum())
+        assert -(-Kp // 16) <= f.T[p] <= Kp // 8 + 1
+
+
 @pytest.mark.parametrize("M,K,v,s,P,kind,mode", [
     (256, 256, 4, 0.80, 128, "uniform", 0),      # C1
     (256, 256, 4, 0.80, 128, "uniform", 1),
