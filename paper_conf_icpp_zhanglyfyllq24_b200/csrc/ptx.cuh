@@ -92,6 +92,15 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+// Bulk copy shared::cta -> shared::cluster (a peer CTA's shared memory, or this
+// CTA's), completing `bytes` transaction bytes on the mbarrier at shared::cluster
+// address `rbar` (in the destination CTA).
+__device__ __forceinline__ void bulk_s2cluster(uint32_t rdst, uint32_t src, uint32_t bytes, uint32_t rbar) {
+  asm volatile("cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   rdst),
+               "r"(src), "r"(bytes), "r"(rbar)
+               : "memory");
+}
 // Four rows (r0..r3) x one box of columns starting at c0 of a 2-D tensor map.
 __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, int32_t c0, int32_t r0,
                                             int32_t r1, int32_t r2, int32_t r3, uint64_t* bar) {
@@ -374,6 +383,18 @@ __device__ __forceinline__ void cluster_sync_relaxed() {
 __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+// Split cluster barrier: arrive now, wait (acquire) later, only where needed.
+__device__ __forceinline__ void cluster_arrive_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() { asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory"); }
+// Named CTA barriers (ids 2..15 free for the kernel's own use; 0 = __syncthreads).
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+__device__ __forceinline__ void named_bar_arrive(int id, int nthreads) {
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
 // shared::cta address of this CTA -> shared::cluster address of the same offset in CTA `rank`
 __device__ __forceinline__ uint32_t mapa_shared(uint32_t saddr, uint32_t rank) {
   uint32_t r;
@@ -405,4 +426,10 @@ __device__ __forceinline__ void st_async_v4(uint32_t raddr, uint32_t a, uint32_t
                "r"(a), "r"(b), "r"(c), "r"(d), "r"(rbar)
                : "memory");
 }
+
+// ---------------------------------------------------------------- programmatic dependent launch
+// Block this thread until the grids this launch depends on (the previous kernels
+// of the stream) have completed and their memory is visible.  A no-op when the
+// launch carries no programmatic dependency.
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 }  // namespace jig

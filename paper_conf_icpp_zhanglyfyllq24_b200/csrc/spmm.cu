@@ -63,6 +63,7 @@ __device__ __forceinline__ int bprod_index(int warp) {  // -1: not a B producer
   const int i = warp - kBProdWarp0;  // 0..9 -> skip 3 (warp 9) and 7 (warp 13)
   return i - (i > 3) - (i > 7);
 }
+constexpr int kBarInit = 2, kBarTmem = 3;  // named barriers (1: epilogue warps, split pieces)
 constexpr int kRowsPerBlock = 32 * kStepsPerBlock;  // B rows per k-block (128)
 constexpr int kChunkB = kRowsPerBlock * 128;        // one 64-column SW128 chunk: 16 KB
 constexpr int kStageA = kStepsPerBlock * kKStepBytesA;  // 16 KB
@@ -383,6 +384,26 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     JIG_TRACE(0);
   }
 
+  // The CTA's first unit, decoded from parameter space by the warps that issue
+  // its first loads (the epilogue warps, idle until the first accumulator is
+  // ready) while warp 0 initialises the barriers; warp 0 decodes it afterwards
+  // for its own bookkeeping.
+  int nA0 = 0, nG0 = 0;
+  Work w0;
+  w0.valid = false;
+  auto decode_first = [&]() {
+    if (cluster_id < prm.nunits) {
+      int h0 = 0;
+      w0 = decode_unit<NT, kPair, Prm>(prm, cluster_id, rank, S, h0);
+      if (w0.valid) {
+        const int nkb = w0.kb_hi - w0.kb_lo;
+        nA0 = min(nkb, C_::kStages);
+        nG0 = min(nkb, C_::kGAhead + 1);
+      }
+    }
+  };
+  if (warp >= 2 && warp <= 5) decode_first();
+
   // Barrier initialisation spread over the lanes of warp 0 (~50 barriers; one
   // thread initialising them all costs ~0.5 us of kernel start).  The barriers
   // are contiguous in shared memory: full, empty, gfull, gempty, tfull, tempty,
@@ -407,71 +428,84 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     fence_barrier_init();
     fence_proxy_async();
     if (lane == 0) JIG_TRACE(17);
+    named_bar_arrive(kBarInit, kThreads);  // the barriers are valid
+    decode_first();
+  } else {
+    if (warp == 1) {  // the TMEM allocation overlaps the barrier initialisation
+      if constexpr (kPair)
+        tmem_alloc_pair<C_::kTmemCols>(tmem_slot);
+      else
+        tmem_alloc<C_::kTmemCols>(tmem_slot);
+    }
+    named_bar_sync(kBarInit, kThreads);
   }
-  // Parallel initial fill (before the block-wide sync, overlapping the TMEM
-  // allocation): lane l of warp 0 issues the gather list of the CTA's first unit's
-  // k-block l (ring slot l) and, for l < kStages, its A / E copies (stage l), so
-  // the first loads leave at kernel start instead of one after another from a
-  // single thread (each mbarrier / bulk-copy operation costs ~100 cycles of issue).
-  int nA0 = 0, nG0 = 0;
-  Work w0;
-  w0.valid = false;
-  if (warp == 0) {
-    if (prm.bpf_bytes > 0) {
-      const int64_t lo = (int64_t)blockIdx.x * prm.bpf_chunk, hi = min(prm.bpf_bytes, lo + prm.bpf_chunk);
-      for (int i = 31 - lane; i < prm.nprob; i += 32) {  // lane 31 takes problem 0
-        const int64_t b0 = prm.pr[i].boff, b1 = b0 + prm.pr[i].K * prm.pr[i].N * 2;
-        const int64_t x0 = max(lo, b0), x1 = min(hi, b1);
-        if (x0 < x1)
-          bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(prm.pr[i].B) + (x0 - b0), (uint32_t)(x1 - x0));
+  // Cluster variants: peers' barriers must be initialised before any remote
+  // arrive / st.async / pair MMA targets them.  Every thread arrives here; only
+  // the warps that touch peer shared memory (MMA, relay, epilogue) wait before
+  // their first remote operation, the others at exit.
+  if constexpr (kSplit || kPair) cluster_arrive_relaxed();
+  bool cl_waited = !(kSplit || kPair);
+  // Initial fill, spread over warps so the first loads leave at once (each
+  // mbarrier / bulk-copy operation costs ~100 cycles of issue from one thread,
+  // and a per-lane bulk copy is serialised): warp 2 issues the gather lists of
+  // the first unit's first k-blocks (ring slots 0 .. nG0-1; the B producers
+  // depend on them), warps 3-5 the compressed A / metadata of stages
+  // (warp - 3) + 3i.  All of it is handle-owned, immutable data, so it runs
+  // before griddepcontrol.wait.
+  if (warp == 2) {
+    if (lane == 0) {
+      JIG_TRACE(18);
+      for (int l = 0; l < nG0; ++l) {
+        const int kb = w0.kb_lo + l;
+        const int steps = w0.steps(kb);
+        mbar_arrive_expect_tx(&gfull[l], (uint32_t)(steps * 128));
+        bulk_g2s(sG + l * kRowsPerBlock, w0.G + w0.gks(kb) * 32, steps * 128, &gfull[l]);
       }
-      if (lane == 31) JIG_TRACE(22);
     }
     __syncwarp();
-    if (cluster_id < prm.nunits) {
-      int h0 = 0;
-      w0 = decode_unit<NT, kPair, Prm>(prm, cluster_id, rank, S, h0);
-      if (w0.valid) {
-        const int nkb = w0.kb_hi - w0.kb_lo;
-        nA0 = min(nkb, C_::kStages);
-        nG0 = min(nkb, C_::kGAhead + 1);
+  } else if (warp >= 3 && warp <= 5) {
+    if (lane == 0) {
+      for (int l = warp - 3; l < nA0; l += 3) {
+        const int kb = w0.kb_lo + l;
+        const int steps = w0.steps(kb);
+        const bool dense = w0.dense(kb);
+        mbar_arrive_expect_tx(&full[l], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
+        bulk_g2s(sA + l * kStageA, w0.Aimg + w0.gks(kb) * kKStepBytesA, steps * kKStepBytesA, &full[l]);
+        if (!dense) bulk_g2s(sE + l * kStageE, w0.Eimg + (w0.kb0 + kb) * kEBlockBytes, kStageE, &full[l]);
       }
+      if (warp == 3 && nA0 > 0) JIG_TRACE(2);
     }
-    if (lane == 0) JIG_TRACE(18);
-    if (lane < nG0) {
-      const int kb = w0.kb_lo + lane;
-      const int steps = w0.steps(kb);
-      mbar_arrive_expect_tx(&gfull[lane], (uint32_t)(steps * 128));
-      bulk_g2s(sG + lane * kRowsPerBlock, w0.G + w0.gks(kb) * 32, steps * 128, &gfull[lane]);
+    __syncwarp();
+  } else if (warp == 0 && prm.bpf_bytes > 0) {
+    const int64_t lo = (int64_t)blockIdx.x * prm.bpf_chunk, hi = min(prm.bpf_bytes, lo + prm.bpf_chunk);
+    for (int i = 31 - lane; i < prm.nprob; i += 32) {  // lane 31 takes problem 0
+      const int64_t b0 = prm.pr[i].boff, b1 = b0 + prm.pr[i].K * prm.pr[i].N * 2;
+      const int64_t x0 = max(lo, b0), x1 = min(hi, b1);
+      if (x0 < x1)
+        bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(prm.pr[i].B) + (x0 - b0), (uint32_t)(x1 - x0));
     }
-    if (lane < nA0) {
-      const int kb = w0.kb_lo + lane;
-      const int steps = w0.steps(kb);
-      const bool dense = w0.dense(kb);
-      mbar_arrive_expect_tx(&full[lane], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
-      bulk_g2s(sA + lane * kStageA, w0.Aimg + w0.gks(kb) * kKStepBytesA, steps * kKStepBytesA, &full[lane]);
-      if (!dense) bulk_g2s(sE + lane * kStageE, w0.Eimg + (w0.kb0 + kb) * kEBlockBytes, kStageE, &full[lane]);
+    if (lane == 31) JIG_TRACE(22);
+    __syncwarp();
+  }
+  // TMEM address: warp 1 (allocator, MMA issuer) and the epilogue warps 2-5
+  uint32_t tbase = 0;
+  if (warp >= 1 && warp <= 5) {
+    tc_fence_before();
+    named_bar_sync(kBarTmem, 5 * 32);
+    tc_fence_after();
+    tbase = *tmem_slot;
+    if (threadIdx.x == 32) JIG_TRACE(1);
+    if constexpr (kSplit || kPair) {
+      cluster_wait();
+      cl_waited = true;
     }
-    if (lane == 0 && nA0 > 0) JIG_TRACE(2);
   }
-  if (warp == 1) {
-    if constexpr (kPair)
-      tmem_alloc_pair<C_::kTmemCols>(tmem_slot);
-    else
-      tmem_alloc<C_::kTmemCols>(tmem_slot);
-  }
-  if constexpr (kSplit || kPair) {
-    cluster_sync_all();  // peers' barriers are initialised before any st.async targets them
-  } else {
-    __syncthreads();
-  }
-  tc_fence_after();
-  const uint32_t tbase = *tmem_slot;
-  if (threadIdx.x == 0) JIG_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ A / E producer
     if (lane == 0) {
+      // the dynamic scheduler's counters are shared with the previous launch
+      if (dyn) griddep_wait();
       // state after the parallel initial fill: stages 0..nA0-1 and gather slots
       // 0..nG0-1 hold the first unit's first k-blocks
       int stage = nA0 % C_::kStages, hint = 0, nkb_issued = nA0, rslot = 0;
@@ -585,6 +619,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     // shared memory (TMA-loaded by warp 0).
     const int bw = bprod_index(warp);
     const int grp = bw / C_::kWPG, wi = bw % C_::kWPG;
+    griddep_wait();  // B may be the previous kernel's output
     constexpr int R = kRowsPerBlock / C_::kWPG;   // rows per warp and k-block
     constexpr int LPR = C_::kNTL / 8;      // lanes per B row (16-byte chunks per row)
     constexpr int RPI = 32 / LPR;          // rows per iteration
@@ -793,6 +828,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   } else if (warp >= 2 && warp <= 5) {
     // ------------------------------------------------------------ epilogue (warps 2-5)
     const int q = warp & 3;  // TMEM lane quarter this warp may access
+    griddep_wait();          // C and the split workspace may still be in use by the previous kernel
     int it = 0, hint = 0, rslot = 0;
     uint32_t rph = 0;
     for (int us = cluster_id;; us += nclusters) {
@@ -932,13 +968,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           __syncwarp();
         }
       } else {
-        // reduce-scatter of the fp32 partial tile through DSMEM
+        // reduce-scatter of the fp32 partial tile through DSMEM: each warp stages
+        // its 32 rows (padded stride, the receive layout) in the B stage ring --
+        // free once the accumulator is ready, a split CTA runs exactly one unit --
+        // and sends them with ONE bulk copy to the owner's receive slot (16-byte
+        // st.async per lane moved ~15 B/clk)
         const int rpo = 128 / S;                           // rows owned per CTA
-        const uint32_t owner = (uint32_t)(r / rpo);
-        const int lr = r % rpo;
-        if (warp == 2 && lane == 0) mbar_arrive_expect_tx(recv_full, (uint32_t)(128 * NT * 4));
-        const uint32_t dst = mapa_shared(smem_u32(sRecv + (rank * rpo + lr) * C_::kRecvStride), owner);
-        const uint32_t dbar = mapa_shared(smem_u32(recv_full), owner);
+        constexpr int kMaxRun = 32;                        // rows of a warp sent by one copy
+        if (warp == 2 && lane == 0) mbar_arrive_expect_tx(recv_full, (uint32_t)(128 * C_::kRecvStride));
+        const uint32_t stg = smem_u32(sB + q * 32 * C_::kRecvStride);
 #pragma unroll 1
         for (int c0 = 0; c0 < NT; c0 += 32) {
           uint32_t v[32];
@@ -951,7 +989,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           }
 #pragma unroll
           for (int j = 0; j < 8; ++j)
-            st_async_v4(dst + (c0 + 4 * j) * 4, v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3], dbar);
+            st_shared_v4u(stg + lane * C_::kRecvStride + (c0 + 4 * j) * 4,
+                          make_uint4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]));
+        }
+        fence_proxy_async();  // the staged rows are read by the bulk copy (async proxy)
+        __syncwarp();
+        // one copy per owner of the warp's rows (S = 8: 16-row owners, two copies)
+        const int run = rpo < kMaxRun ? rpo : kMaxRun;
+        if (lane < 32 / run) {
+          const int r0 = q * 32 + lane * run;
+          const uint32_t owner = (uint32_t)(r0 / rpo);
+          bulk_s2cluster(mapa_shared(smem_u32(sRecv + (rank * rpo + r0 % rpo) * C_::kRecvStride), owner),
+                         stg + lane * run * C_::kRecvStride, run * C_::kRecvStride,
+                         mapa_shared(smem_u32(recv_full), owner));
         }
         // owner: wait for all S partial slices of its rows, sum, convert, store
         if (warp == 2 && lane == 0) JIG_TRACE(7);
@@ -995,6 +1045,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   if constexpr (kSplit || kPair) {
     // no CTA leaves while peers may still target its shared memory (DSMEM
     // sends, pair commits); the C stores need no cluster-scope release here
+    __syncwarp();
+    if (!cl_waited) cluster_wait();  // complete the prologue's barrier phase first
     cluster_sync_relaxed();
   } else {
     __syncthreads();
@@ -1013,6 +1065,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 }
 
 int g_num_sms[64] = {0};
+
+// JIGSAW_PDL=0 launches without the programmatic-dependency attribute (A/B only).
+bool spmm_pdl_enabled() {
+  static const bool on = !(getenv("JIGSAW_PDL") && atoi(getenv("JIGSAW_PDL")) == 0);
+  return on;
+}
 bool g_attr_set[64][16] = {};  // [device][variant]
 
 template <int NT, bool kSplit, bool kPair, class Prm>
@@ -1033,13 +1091,20 @@ jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid
   cfg.blockDim = dim3(kThreads);
   cfg.dynamicSmemBytes = C_::kSmem;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = kPair ? 2 : kSplit ? S : 1;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  // Programmatic dependent launch: the CTAs may start while the previous kernel
+  // of the stream drains.  The prologue (barrier init, TMEM allocation, the
+  // first k-blocks' compressed A / metadata / gather lists -- handle-owned,
+  // immutable) runs before griddepcontrol.wait; every access to B, C and the
+  // shared workspaces / scheduler counters comes after it.
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = spmm_pdl_enabled() ? 2 : 1;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, prm);
   if (e != cudaSuccess) return cuda_status(e, "k_spmm launch");
   return JIGSAW_SUCCESS;
