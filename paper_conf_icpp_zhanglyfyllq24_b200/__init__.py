@@ -75,7 +75,8 @@ def lib(build_if_missing: bool = True):
                 raise
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"libjigsaw.so not built ({LIB_PATH}); run __graft_entry__.build()")
-    L = ctypes.CDLL(LIB_PATH)
+    # developer A/B of two builds of the same library (e.g. tools/ab_*.sh)
+    L = ctypes.CDLL(os.environ.get("JIGSAW_LIB_AB") or LIB_PATH)
     vp, i64, ci = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
     sig = {
         "jigsaw_reorder": (vp, [vp, i64, i64, ci]),

@@ -364,6 +364,15 @@ __device__ __forceinline__ void cp_async_16(void* dst, const void* src, uint32_t
                "r"(src_bytes)
                : "memory");
 }
+// 16-byte cp.async to a shared::cta address; `zero` = write zeros, read nothing
+// (ignore-src predicate: maps to the LDGSTS ZFILL predicate, no size arithmetic).
+__device__ __forceinline__ void cp_async_16_zfill(uint32_t dst, const void* src, bool zero) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t"
+      "cp.async.cg.shared.global [%0], [%1], 16, p;\n\t}" ::"r"(dst),
+      "l"(src), "r"((uint32_t)zero)
+      : "memory");
+}
 // Arrive on `bar` once all prior cp.async of this thread have completed (no pending++).
 __device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint64_t* bar) {
   asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");

@@ -626,17 +626,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     const int c = lane % LPR;
     int hint = 0, traced = 0, rslot = 0;
     uint32_t rph = 0;
-    int64_t j = 0;  // CTA-wide k-block sequence number (the stage ring's order)
+    int j = 0;  // CTA-wide k-block sequence number (the stage ring's order)
     for (int us = cluster_id;; us += nclusters) {
       const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, true, lane) : (us < prm.nunits ? us : -1);
       if (u < 0) break;
       const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
       if (bw == 0 && lane == 0 && traced == 0) JIG_TRACE(19);
       if (!wk.valid) continue;
+      // Per-lane constants of the unit: the 16-byte column chunk this lane copies
+      // (global byte address of row 0), the row pitch, and the row bound -- PAD
+      // rows (index K) and chunks past column N are zero-filled.  The inner loop
+      // is then SHFL (row index) + IMAD.WIDE (address) + ISETP (bound) + LDGSTS
+      // per 16 bytes: the B producers are issue-bound (a few extra instructions
+      // per copy measured -25 % on C4).
       const int col = wk.n0 + (kPair ? (int)rank * C_::kNTL : 0) + 8 * c;
-      const bool colok = col < wk.N;
-      const __half* Bp = wk.B;
-      const int64_t ldb = wk.N, K = wk.K;
+      const char* const colbase = reinterpret_cast<const char*>(wk.B) + (int64_t)col * 2;
+      const uint32_t ldb_bytes = (uint32_t)wk.N * 2u;
+      const uint32_t kbound = col < wk.N ? (uint32_t)wk.K : 0u;
+      const uint32_t hsw = (uint32_t)((c & 7) ^ (lane / LPR));  // SW128 chunk of this lane, row phase 0
       int kb = wk.kb_lo + (int)((grp - j % C_::kBGroups + C_::kBGroups) % C_::kBGroups);
       j += kb - wk.kb_lo;
       for (; kb < wk.kb_hi; kb += C_::kBGroups, j += C_::kBGroups) {
@@ -653,22 +660,21 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&gempty[gslot]);
         mbar_wait(&empty[stage], phase ^ 1);
-        uint8_t* sb = sB + stage * C_::kStageB + (c >> 3) * kChunkB;
+        const uint32_t sb = smem_u32(sB + stage * C_::kStageB + (c >> 3) * kChunkB) + (uint32_t)(lane / LPR) * 128u;
 #pragma unroll
         for (int t = 0; t < (R + 31) / 32; ++t) {
           const int ks = (wi * R) / 32 + t;          // k-step of these rows
           const int jlo = R < 32 ? (wi * R) & 31 : 0;  // rows [jlo, jlo + min(R, 32)) of the k-step
           if (ks >= steps || (dense && jlo >= 16)) continue;
-          const int jn = dense ? 16 - jlo : (R < 32 ? R : 32);
 #pragma unroll
           for (int it = 0; it < (R < 32 ? R : 32) / RPI; ++it) {
-            const int jr = jlo + it * RPI + lane / LPR;
-            if (it * RPI >= jn) break;
-            const int32_t g = __shfl_sync(kFullMask, gl[t], jr);
-            const bool ok = colok && g < K;
-            const __half* src = ok ? Bp + (int64_t)g * ldb + col : Bp;
-            const int row = 32 * ks + jr;
-            cp_async_16(sb + row * 128 + (((c & 7) ^ (row & 7)) << 4), src, ok ? 16u : 0u);
+            if (dense && jlo + it * RPI >= 16) break;
+            const int jr0 = jlo + it * RPI;             // row of lane group 0 (multiple of RPI)
+            const uint32_t g = (uint32_t)__shfl_sync(kFullMask, gl[t], jr0 + lane / LPR);
+            const char* src = colbase + (uint64_t)g * ldb_bytes;
+            // row = 32 ks + jr0 + lane / LPR; its SW128 phase (row & 7) = (jr0 & 7) ^ (lane / LPR)
+            const uint32_t dst = sb + (uint32_t)(32 * ks + jr0) * 128u + ((hsw ^ (uint32_t)(jr0 & 7)) << 4);
+            cp_async_16_zfill(dst, src, g >= kbound);
           }
         }
         cp_async_mbar_arrive_noinc(&full[stage]);

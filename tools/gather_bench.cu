@@ -13,6 +13,7 @@
 
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 #include <vector>
 
 #include "../paper_conf_icpp_zhanglyfyllq24_b200/csrc/ptx.cuh"
@@ -38,6 +39,7 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
   const int nprod = mode == 1 ? 8 : mode == 4 ? 12 : (mode == 5 || mode == 6 || mode == 8 || mode == 9) ? 16
                     : (mode == 7 || mode == 10) ? 8 : 4;
   const bool ldgsts = mode <= 1 || mode == 4 || mode == 5;
+  const int N = ldb;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) {
       mbar_init(&full[s], (ldgsts || mode == 6) ? nprod * 32
@@ -138,6 +140,15 @@ __global__ void __launch_bounds__(544, 1) gather_kernel(const __grid_constant__ 
             for (int ch = 0; ch < 2; ++ch)
               tma_load_2d(st + ch * (kRows * 128) + row * 128, &tm, 64 * ch, hrow(blockIdx.x, kb, row, K), &full[stage]);
         }
+      } else if (mode == 11) {
+        // contiguous 1-D bulk copies (the compressed-A path): 4 x 8 KB per stage, one issuer
+        if (w == 0 && lane == 0) {
+          mbar_arrive_expect_tx(&full[stage], kStageBytes);
+          for (int i = 0; i < 4; ++i) {
+            const int off = hrow(blockIdx.x, kb, i, K * N * 2 / 8192 - 1) * 8192;
+            bulk_g2s(st + i * 8192, reinterpret_cast<const uint8_t*>(B) + off, 8192, &full[stage]);
+          }
+        }
       } else {
         if (lane == 0) {
           if (w == 0) mbar_arrive_expect_tx(&full[stage], kStageBytes);
@@ -159,8 +170,14 @@ typedef CUresult (*EncodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, v
                                 const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                 CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-int main() {
-  const int K = 4096, N = 256, grid = 148;
+int main(int argc, char** argv) {
+  const int K = 4096, N = 256, grid = argc > 1 ? atoi(argv[1]) : 148;
+  std::vector<int> modes;
+  if (argc > 2) {
+    for (char* t = strtok(argv[2], ","); t; t = strtok(nullptr, ",")) modes.push_back(atoi(t));
+  } else {
+    for (int m = 0; m < 12; ++m) modes.push_back(m);
+  }
   uint16_t* dB;
   int* didx;
   long long* dout;
@@ -185,8 +202,9 @@ int main() {
   cudaFuncSetAttribute(gather_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   const char* names[] = {"LDGSTS 4 warps", "LDGSTS 8 warps", "TMA gather4, 1 issuer", "TMA gather4, 4 issuers",
                          "LDGSTS 12 warps", "LDGSTS 16 warps", "LDG+STS 16 warps", "TMA gather4, 8 issuers",
-                         "TMA gather4, 16 issuers", "LDGSTS 8w + gather4 8w", "TMA tile row, 8 issuers"};
-  for (int mode = 0; mode < 11; ++mode) {
+                         "TMA gather4, 16 issuers", "LDGSTS 8w + gather4 8w", "TMA tile row, 8 issuers",
+                         "bulk 1-D 8 KB x 4"};
+  for (int mode : modes) {
     for (int rep = 0; rep < 3; ++rep) {
       cudaEvent_t a, b;
       cudaEventCreate(&a);
@@ -204,8 +222,8 @@ int main() {
       for (auto c : cyc) mx = c > mx ? c : mx;
       const double bytes = (double)grid * KB * kStageBytes;
       if (rep == 2)
-        printf("%-24s %8.1f us  %7.1f GB/s total  %5.1f B/clk/SM (max CTA %lld cyc, %.0f cyc per k-block)\n",
-               names[mode], ms * 1e3, bytes / ms / 1e6, (double)KB * kStageBytes / mx, mx, (double)mx / KB);
+        printf("grid %3d %-24s %8.1f us  %7.1f GB/s total  %5.1f B/clk/SM (max CTA %lld cyc, %.0f cyc per k-block)\n",
+               grid, names[mode], ms * 1e3, bytes / ms / 1e6, (double)KB * kStageBytes / mx, mx, (double)mx / KB);
     }
   }
   return 0;
