@@ -414,6 +414,11 @@ __device__ __forceinline__ uint32_t mapa_shared(uint32_t saddr, uint32_t rank) {
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t rbar) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(rbar) : "memory");
 }
+// Relaxed remote arrive: no release fence (a cluster-scope release waits for the
+// SM's outstanding memory operations, ~1000 cycles with the B gathers in flight).
+__device__ __forceinline__ void mbar_arrive_cluster_relaxed(uint32_t rbar) {
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(rbar) : "memory");
+}
 // Wait (acquire, cluster scope) for phase `parity` of a local mbarrier that remote CTAs arrive on.
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
   asm volatile(

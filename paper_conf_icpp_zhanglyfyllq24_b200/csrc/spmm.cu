@@ -33,6 +33,9 @@
 #ifndef JIG_BGROUPS
 #define JIG_BGROUPS 1  // B-producer warp groups (see Cfg::kBGroups); > 1 measured slower in k_spmm
 #endif
+#ifndef JIG_RELAY
+#define JIG_RELAY 1  // pair relay: bit 0 fence.proxy.async, bit 1 release.cluster arrive (else relaxed; release: C4 +16 %)
+#endif
 #ifndef JIG_HALVES
 #define JIG_HALVES 0  // pair N = 256 as two 128-column halves (see Cfg::kHalves); measured slower
 #endif
@@ -160,7 +163,8 @@ struct ParamsT {
   int sched;  // >= 0: dynamic tile scheduler on counter slot `sched`; -1: static round-robin
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
   int prefetch;  // 1: prefetch each unit's gather lists / metadata into L2 at unit start
-  int dbg;       // developer timing experiments (JIGSAW_DBG, results invalid): 1 skip tcgen05.cp, 2 skip MMAs
+  int dbg;       // developer timing experiments (JIGSAW_DBG, results invalid): 1 skip tcgen05.cp, 2 skip MMAs,
+                 // 8 no B reads (zero fill), 16 no A / metadata loads after the initial fill
 };
 using ParamsOne = ParamsT<1, 128, 1, 160>;   // single product (~7.3 KB of parameters)
 using ParamsGroup = ParamsT<64, 1024, 2048>; // grouped launch (~31 KB)
@@ -593,9 +597,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           const bool dense = wk.dense(kb);
           const int64_t gks = wk.gks(kb);
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
-          bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
-          if (!dense) bulk_g2s(sE + stage * kStageE, wk.Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
+          if (prm.dbg & 16) {  // timing only: no A / metadata loads
+            mbar_arrive(&full[stage]);
+          } else {
+            mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
+            bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
+            if (!dense) bulk_g2s(sE + stage * kStageE, wk.Eimg + (kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
+          }
           if (u == cluster_id && kb == wk.kb_lo) JIG_TRACE(2);
           JIG_TRACE_KB(0, nkb_issued);
           ++nkb_issued;
@@ -642,7 +650,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int col = wk.n0 + (kPair ? (int)rank * C_::kNTL : 0) + 8 * c;
       const char* const colbase = reinterpret_cast<const char*>(wk.B) + (int64_t)col * 2;
       const uint32_t ldb_bytes = (uint32_t)wk.N * 2u;
-      const uint32_t kbound = col < wk.N ? (uint32_t)wk.K : 0u;
+      const uint32_t kbound = col < wk.N && !(prm.dbg & 8) ? (uint32_t)wk.K : 0u;  // dbg 8: no B reads
       const uint32_t hsw = (uint32_t)((c & 7) ^ (lane / LPR));  // SW128 chunk of this lane, row phase 0
       int kb = wk.kb_lo + (int)((grp - j % C_::kBGroups + C_::kBGroups) % C_::kBGroups);
       j += kb - wk.kb_lo;
@@ -681,8 +689,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         if (lane == 0 && bw == 0) {
           if (traced == 0) JIG_TRACE(3);
           JIG_TRACE_KB(1, traced);
-          ++traced;
         }
+        if (kPair && rank != 0 && lane == 0 && bw == kBProdWarps - 1) JIG_TRACE_KB(3, traced);  // last B warp (odd CTA)
+        ++traced;
       }
       j -= kb - wk.kb_hi;  // the k-blocks of this unit past the last one of this group
     }
@@ -691,7 +700,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     // The even CTA issues the pair's MMAs; it may read this CTA's stage only once
     // this CTA's A/E bulk copies and B cp.async have landed: relay full -> pfull.
     if (lane == 0) {
-      int stage = 0, hint = 0;
+      int stage = 0, hint = 0, nrel = 0;
       uint32_t phase = 0;
       const uint32_t rpfull = mapa_shared(smem_u32(pfull), 0);
       for (int us = cluster_id; us < prm.nunits; us += nclusters) {
@@ -699,8 +708,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         if (!wk.valid) continue;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           mbar_wait(&full[stage], phase);
-          fence_proxy_async();
-          mbar_arrive_cluster(rpfull + 8 * stage);
+          JIG_TRACE_KB(2, nrel);  // odd CTA: own stage landed
+          ++nrel;
+          if (JIG_RELAY & 1) fence_proxy_async();
+          if (JIG_RELAY & 2)
+            mbar_arrive_cluster(rpfull + 8 * stage);
+          else
+            mbar_arrive_cluster_relaxed(rpfull + 8 * stage);
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
@@ -752,6 +766,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           const bool dense = wk.dense(kb);
           const long long tw0 = JIG_TRACE_KB_ON && prm.trace ? clock64() : 0;
           mbar_wait(&full[stage], phase);
+          if (kPair) JIG_TRACE_KB(4, nkb_mma);  // pair: own stage landed (the relay's wait follows)
           // pfull: CTA-scope acquire.  The odd CTA released its stage at cluster scope
           // after observing its own copies complete; the data is read by the tensor
           // core (async proxy, ordered by tcgen05.fence), not by this thread, and a
@@ -766,7 +781,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             const uint64_t edesc = smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0);
             tc_cp_128x128b_warp<kPair>(e_tmem, edesc);
           }
-          JIG_TRACE_KB(4, nkb_mma);
+          if (!kPair) JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
           if (!C_::kHalves && !dense && steps == kStepsPerBlock && !(prm.dbg & 2)) {
