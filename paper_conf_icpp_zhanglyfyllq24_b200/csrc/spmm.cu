@@ -1431,14 +1431,21 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       thread_local std::vector<U> us;
       us.clear();
       int64_t total = 0;
+      // fixed per-unit cost in k-block equivalents (accumulator drain, pipeline
+      // refill).  Pairs with NT = 256 have a single accumulator buffer, so a
+      // unit's epilogue is not overlapped with the next unit's mainloop: 4
+      // (C2 at P = 256: 41.1 -> 35.3 us; the larger cost also stops the split
+      // pieces whose workspace reduction cost more than the balance they bought,
+      // profiles/r01w_unit_cost.txt).  Developer override JIGSAW_UNIT_COST.
+      const int unit_cost = getenv("JIGSAW_UNIT_COST") ? atoi(getenv("JIGSAW_UNIT_COST")) : (pair && NT == 256 ? 4 : 1);
       for (int i = 0; i < n; ++i) {
         const Format& f = *fs[i0 + i];
         const int ntn = (int)((Ns[i0 + i] + NT - 1) / NT);
         for (int p = 0; p < f.npanels; ++p)
           for (int t = 0; t < ntn; ++t) {  // N tiles of a panel adjacent: they share its A stream
             const int nkb = (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
-            us.push_back({nkb + 1, nkb, ((uint32_t)i << 26) | ((uint32_t)(t * f.npanels + p) << 15)});
-            total += nkb + 1;
+            us.push_back({nkb + unit_cost, nkb, ((uint32_t)i << 26) | ((uint32_t)(t * f.npanels + p) << 15)});
+            total += nkb + unit_cost;
           }
       }
       // JIGSAW_SCHED=loc: locality order (problem, panel, N tile) dealt round-robin,
