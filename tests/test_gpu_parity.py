@@ -190,6 +190,40 @@ def test_spmm_batched_and_streams():
         spmm_check(_host(c), a, b)
 
 
+@pytest.mark.parametrize("M1,K,N,P", [(512, 2048, 256, 128), (2048, 512, 256, 128), (1024, 1536, 512, 256)])
+def test_programmatic_dependent_launch_ordering(M1, K, N, P):
+    """k_spmm is launched with the programmatic-dependent-launch attribute: its
+    prologue (handle-owned A / metadata / gather lists) overlaps the previous
+    kernel, every access to B and C waits on griddepcontrol.wait.  Checked with no
+    host sync anywhere: B written by the kernel right before the call (behind a
+    long matmul), C read by the kernel right before (write-after-read: the clone
+    must see the old contents), C consumed right after, and a chain where the
+    output of one SpMM is the B of the next (single split-K, grouped and pair
+    launches)."""
+    v = 8
+    A1 = synth.vector_sparse(M1, K, v, 0.9, 61)
+    A2 = synth.vector_sparse(384, M1, v, 0.9, 62)
+    Bh = synth.dense_b(K, N, 63)
+    h1 = jig.reorder(_dev(A1), v, panel_rows=P)
+    h2 = jig.reorder(_dev(A2), v)
+    src = _dev(Bh)
+    B = torch.zeros_like(src)
+    C1 = torch.full((M1, N), 7.0, dtype=torch.float16, device="cuda")
+    C2 = torch.empty((384, N), dtype=torch.float16, device="cuda")
+    big = torch.randn(4096, 4096, device="cuda", dtype=torch.float16)
+    torch.cuda.synchronize()
+    _ = big @ big                 # keeps the stream busy so the copy below is still pending
+    B.copy_(src)                  # producer of B, immediately before the SpMM
+    old = C1.clone()              # reader of C, immediately before the SpMM
+    h1.spmm(B, C=C1)
+    h2.spmm(C1, C=C2)             # consumer of C1 as the next B
+    torch.cuda.synchronize()
+    assert bool((old == 7.0).all())
+    C1h = _host(C1)
+    spmm_check(C1h, A1, Bh)
+    spmm_check(_host(C2), A2, C1h)
+
+
 def test_abi_errors_on_gpu():
     A = synth.vector_sparse(128, 64, 4, 0.8, 1)
     h = jig.reorder(_dev(A), 4)
