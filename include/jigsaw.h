@@ -168,6 +168,21 @@ JIGSAW_API jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const 
                                     const int64_t* Ns, void* const* Cs, int count,
                                     jigsaw_stream_t stream);
 
+/* The batch of jigsaw_spmm_batched with every B and C in HOST memory (the
+ * end-to-end path of a batch): Bs_host[i] is K_i x Ns[i] fp16 row-major,
+ * Cs_host[i] M_i x Ns[i] fp16 row-major (overwritten).  The batch is cut into
+ * chunks whose host->device copies, grouped SpMM launches and device->host
+ * copies run on three streams of the handles' device, so the copy engines of
+ * both directions and the SMs work at the same time; pinned host buffers are
+ * needed for the copies to overlap (pageable memory is correct but serial).
+ * Device staging comes from the stream-ordered pool and is returned before the
+ * call returns.  Ordered after prior work on `stream`; synchronous: returns
+ * after every C is in host memory.  Errors as jigsaw_spmm_batched; a failure
+ * in a later chunk leaves earlier Cs written. */
+JIGSAW_API jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* const* Bs_host,
+                                                    const int64_t* Ns, void* const* Cs_host, int count,
+                                                    jigsaw_stream_t stream);
+
 /* Number of kernels the last successful jigsaw_spmm issued per call (for launch
  * accounting in benchmarks); reorder kernels are not counted. */
 JIGSAW_API int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N);

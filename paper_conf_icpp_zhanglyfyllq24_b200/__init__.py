@@ -28,7 +28,7 @@ STATUS = {0: "SUCCESS", 1: "INVALID_VALUE", 2: "UNSUPPORTED", 3: "OUT_OF_MEMORY"
 ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_status",
                "jigsaw_last_error_string", "jigsaw_version", "jigsaw_reorder_ex",
                "jigsaw_reorder_host", "jigsaw_get_info", "jigsaw_export_format",
-               "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_launches_per_call",
+               "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_batched_host", "jigsaw_spmm_launches_per_call",
                "jigsaw_debug_trace"]
 
 
@@ -92,6 +92,8 @@ def lib(build_if_missing: bool = True):
         "jigsaw_spmm_host": (ci, [vp, vp, i64, vp, vp]),
         "jigsaw_spmm_batched": (ci, [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(i64),
                                      ctypes.POINTER(vp), ci, vp]),
+        "jigsaw_spmm_batched_host": (ci, [ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(i64),
+                                          ctypes.POINTER(vp), ci, vp]),
         "jigsaw_spmm_launches_per_call": (ci, [vp, i64]),
         "jigsaw_debug_trace": (ci, [vp, ci]),
     }
@@ -234,6 +236,25 @@ def debug_trace(max_ctas: int = 1024) -> np.ndarray:
     if n < 0:
         raise JigsawError(4, "jigsaw_debug_trace failed")
     return out[:n]
+
+
+def spmm_batched_host(handles, Bs, outs=None, stream=None):
+    """jigsaw_spmm_batched_host: the batch with host B's in and host C's out
+    (pinned arrays, e.g. from torch pin_memory, let the copies overlap)."""
+    n = len(handles)
+    Bs = [np.ascontiguousarray(b).view(np.uint16) if b.dtype == np.float16 else np.ascontiguousarray(b)
+          for b in Bs]
+    if outs is None:
+        outs = [np.empty((h.M, b.shape[1]), dtype=np.uint16) for h, b in zip(handles, Bs)]
+    for h, b, c in zip(handles, Bs, outs):
+        if c.shape != (h.M, b.shape[1]) or not c.flags.c_contiguous or c.itemsize != 2:
+            raise ValueError("each out must be a contiguous M x N 16-bit array")
+    hs = (ctypes.c_void_p * n)(*[h.ptr.value for h in handles])
+    bp = (ctypes.c_void_p * n)(*[b.ctypes.data for b in Bs])
+    cp = (ctypes.c_void_p * n)(*[c.ctypes.data for c in outs])
+    ns = (ctypes.c_int64 * n)(*[b.shape[1] for b in Bs])
+    _raise_if(lib().jigsaw_spmm_batched_host(hs, bp, ns, cp, n, _stream_ptr(stream) if stream is not None else None))
+    return outs
 
 
 def spmm_batched(handles, Bs, Cs, stream=None):

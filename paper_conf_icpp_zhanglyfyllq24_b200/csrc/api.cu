@@ -239,6 +239,150 @@ jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const
   return set_status(JIGSAW_SUCCESS);
 }
 
+// Several independent copies in one submission (cudaMemcpyBatchAsync: one
+// driver call instead of one per product -- per-copy submission cost ~40 us
+// through torch, profiles/r01y_pcie.txt); a plain loop if the batch call fails.
+static cudaError_t copy_batch(std::vector<void*>& dst, std::vector<void*>& src, std::vector<size_t>& sz,
+                              cudaStream_t st) {
+  if (dst.empty()) return cudaSuccess;
+  cudaMemcpyAttributes attr = {};
+  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+  size_t idx = 0, fail = 0;
+  cudaError_t e = cudaMemcpyBatchAsync(dst.data(), src.data(), sz.data(), dst.size(), &attr, &idx, 1, &fail, st);
+  if (e == cudaSuccess) return e;
+  cudaGetLastError();
+  for (size_t i = 0; i < dst.size() && (e = cudaMemcpyAsync(dst[i], src[i], sz[i], cudaMemcpyDefault, st)) == cudaSuccess; ++i) {
+  }
+  return e;
+}
+
+// Helper streams of the host-buffer batch pipeline (created once per device).
+struct HostPipe {
+  cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
+};
+HostPipe g_pipe[64];
+
+jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* const* Bs_host, const int64_t* Ns,
+                                         void* const* Cs_host, int count, jigsaw_stream_t stream) {
+  if (count < 0 || (count > 0 && (!hs || !Bs_host || !Ns || !Cs_host)))
+    return set_status(JIGSAW_ERROR_INVALID_VALUE, "bad batch arguments");
+  for (int i = 0; i < count; ++i) {
+    jigsaw_status_t s = validate_spmm(hs[i], Bs_host[i], Ns[i], Cs_host[i], false);
+    if (s != JIGSAW_SUCCESS) return s;
+    if (i > 0 && hs[i]->f.device != hs[0]->f.device)
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "handles of a batch must live on one device");
+  }
+  if (count == 0) return set_status(JIGSAW_SUCCESS);
+  const int dev = hs[0]->f.device;
+  if (dev < 0 || dev >= 64) return set_status(JIGSAW_ERROR_INTERNAL, "device ordinal out of range");
+  HostPipe& P = g_pipe[dev];
+  if (!P.h2d) {
+    if (cudaStreamCreateWithFlags(&P.h2d, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&P.comp, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&P.d2h, cudaStreamNonBlocking) != cudaSuccess) {
+      cudaGetLastError();
+      P = HostPipe{};
+      return set_status(JIGSAW_ERROR_CUDA, "cudaStreamCreate failed");
+    }
+  }
+  cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
+  // staging for the whole batch (one pool allocation each for B and C)
+  size_t bb = 0, cb = 0;
+  std::vector<size_t> boff(count), coff(count);
+  for (int i = 0; i < count; ++i) {
+    boff[i] = bb;
+    coff[i] = cb;
+    bb += ((size_t)hs[i]->f.K * Ns[i] * 2 + 255) & ~size_t(255);
+    cb += ((size_t)hs[i]->f.M * Ns[i] * 2 + 255) & ~size_t(255);
+  }
+  cudaEvent_t ev0;
+  if (cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming) != cudaSuccess) return cuda_status(cudaGetLastError(), "event");
+  cudaEventRecord(ev0, user);  // ordered after prior work on the caller's stream
+  cudaStreamWaitEvent(P.h2d, ev0, 0);
+  char *dB = nullptr, *dC = nullptr;
+  cudaError_t e = staging_alloc(reinterpret_cast<void**>(&dB), bb, P.h2d);
+  if (e == cudaSuccess) e = staging_alloc(reinterpret_cast<void**>(&dC), cb, P.h2d);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    if (dB) cudaFreeAsync(dB, P.h2d);
+    cudaStreamSynchronize(P.h2d);
+    cudaEventDestroy(ev0);
+    return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "staging allocation failed");
+  }
+  // chunks of ~1/8 of the batch's bytes (at least one product; developer
+  // override JIGSAW_HOST_CHUNKS): copy-in of chunk
+  // k+1 and copy-out of chunk k-1 overlap the grouped launch of chunk k
+  const int nchunks = getenv("JIGSAW_HOST_CHUNKS") ? std::max(1, atoi(getenv("JIGSAW_HOST_CHUNKS"))) : 8;
+  const size_t target = std::max<size_t>((bb + cb) / nchunks, 1);
+  std::vector<const Format*> fs;
+  std::vector<const void*> pb;
+  std::vector<int64_t> pn;
+  std::vector<void*> pc;
+  jigsaw_status_t st = JIGSAW_SUCCESS;
+  std::vector<cudaEvent_t> evs;
+  for (int i0 = 0; i0 < count && st == JIGSAW_SUCCESS;) {
+    int i1 = i0;
+    size_t acc = 0;
+    while (i1 < count && (i1 == i0 || acc < target)) {
+      acc += (size_t)hs[i1]->f.K * Ns[i1] * 2 + (size_t)hs[i1]->f.M * Ns[i1] * 2;
+      ++i1;
+    }
+    std::vector<void*> cd, cs;
+    std::vector<size_t> cz;
+    for (int i = i0; i < i1; ++i) {
+      cd.push_back(dB + boff[i]);
+      cs.push_back(const_cast<void*>(Bs_host[i]));
+      cz.push_back((size_t)hs[i]->f.K * Ns[i] * 2);
+    }
+    if (e == cudaSuccess) e = copy_batch(cd, cs, cz, P.h2d);
+    cudaEvent_t in, done;
+    cudaEventCreateWithFlags(&in, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
+    evs.push_back(in);
+    evs.push_back(done);
+    cudaEventRecord(in, P.h2d);
+    cudaStreamWaitEvent(P.comp, in, 0);
+    fs.clear(); pb.clear(); pn.clear(); pc.clear();
+    for (int i = i0; i < i1; ++i) {
+      fs.push_back(&hs[i]->f);
+      pb.push_back(dB + boff[i]);
+      pn.push_back(Ns[i]);
+      pc.push_back(dC + coff[i]);
+    }
+    if (e == cudaSuccess) st = launch_spmm_grouped(fs.data(), pb.data(), pn.data(), pc.data(), i1 - i0, P.comp);
+    cudaEventRecord(done, P.comp);
+    cudaStreamWaitEvent(P.d2h, done, 0);
+    cd.clear(); cs.clear(); cz.clear();
+    for (int i = i0; i < i1; ++i) {
+      cd.push_back(Cs_host[i]);
+      cs.push_back(dC + coff[i]);
+      cz.push_back((size_t)hs[i]->f.M * Ns[i] * 2);
+    }
+    if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, P.d2h);
+    i0 = i1;
+  }
+  // staging goes back to the pool after the last copy-out
+  cudaEvent_t fin;
+  cudaEventCreateWithFlags(&fin, cudaEventDisableTiming);
+  cudaEventRecord(fin, P.d2h);
+  cudaStreamWaitEvent(P.h2d, fin, 0);
+  cudaFreeAsync(dB, P.h2d);
+  cudaFreeAsync(dC, P.h2d);
+  cudaEventRecord(fin, P.h2d);
+  cudaStreamWaitEvent(user, fin, 0);
+  cudaError_t e2 = cudaStreamSynchronize(P.h2d);
+  cudaError_t e3 = cudaStreamSynchronize(P.comp);
+  cudaError_t e4 = cudaStreamSynchronize(P.d2h);
+  for (cudaEvent_t x : evs) cudaEventDestroy(x);
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(fin);
+  if (st != JIGSAW_SUCCESS) return st;
+  if (e != cudaSuccess) return cuda_status(e, "jigsaw_spmm_batched_host copies");
+  if (e2 != cudaSuccess || e3 != cudaSuccess || e4 != cudaSuccess)
+    return cuda_status(e2 != cudaSuccess ? e2 : e3 != cudaSuccess ? e3 : e4, "jigsaw_spmm_batched_host");
+  return set_status(JIGSAW_SUCCESS);
+}
+
 int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N) {
   (void)h;
   (void)N;

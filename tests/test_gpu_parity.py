@@ -558,3 +558,22 @@ def test_small_panel_formats_bit_exact(P, M, K, v, s, mode):
                        D=g["D"] if mode == 1 else None, rcol=g["rcol"] if mode == 1 else None,
                        dvals=g["dvals"] if mode == 1 else None)
     h.free()
+
+
+def test_spmm_batched_host_pipeline():
+    """jigsaw_spmm_batched_host: host B's in, host C's out, chunks of the batch
+    pipelined over three streams -- every C against the oracle, mixed panel
+    heights (single and pair launches), ragged N, pinned and pageable buffers."""
+    pts = [(512, 2048, 4, 0.9, 256), (2048, 512, 8, 0.8, 200), (384, 700, 8, 0.8, 72), (1024, 1024, 8, 0.9, 512)]
+    mats = [synth.vector_sparse(M, K, v, s, 70 + i) for i, (M, K, v, s, N) in enumerate(pts)]
+    Bs = [synth.dense_b(K, N, 80 + i) for i, (M, K, v, s, N) in enumerate(pts)]
+    hs = [jig.reorder(_dev(a), v, panel_rows=(256 if i == 3 else 128)) for i, (a, (M, K, v, s, N)) in
+          enumerate(zip(mats, pts))]
+    Cs = jig.spmm_batched_host(hs, Bs)                        # pageable
+    for a, b, c in zip(mats, Bs, Cs):
+        spmm_check(c, a, b)
+    pin_B = [torch.from_numpy(b.view(np.int16)).pin_memory().numpy().view(np.uint16) for b in Bs]
+    pin_C = [torch.empty((M, N), dtype=torch.int16).pin_memory().numpy().view(np.uint16) for (M, K, v, s, N) in pts]
+    jig.spmm_batched_host(hs, pin_B, pin_C)                   # pinned, overlapped
+    for a, b, c in zip(mats, Bs, pin_C):
+        spmm_check(c, a, b)
