@@ -6,7 +6,7 @@
 //                    (col_idx_array; R-Q4)
 //   R3 k_main_tiles  one warp per full 16-column tile of S_p: Alg. 1
 //                    + reorder retry -- tiles are independent
-//   R4 k_overflow    one warp per panel: the remainder of S_p and the evicted
+//   R4 k_overflow    one CTA per panel (waves of warps): the remainder of S_p and the evicted
 //                    columns, re-tiled in FIFO order (R-Q12)
 //   R5 k_emit        2:4 compression straight into the device
 //                    layout the SpMM kernel consumes (A image, TMEM metadata
@@ -227,20 +227,29 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
     }
   }
   __syncwarp();
+  // depth-first over up to 4 disjoint blocks, the first block dealt to the lanes
+  // (lane l starts from blocks l, l + 32, ...): a search that must fail -- the
+  // common case once a tile has more than 8 hard columns -- is exhausted 32
+  // lanes at a time instead of by one thread
   int found = 0;
-  if (lane == 0) {
-    const int n = s.nbig, need = __popc(realset) - 8;
-    if (n > kMaxBig) {
-      found = 1;
-    } else {
-      // depth-first over disjoint blocks (<= 4 deep), best excess first
-      int idx[4] = {0, 0, 0, 0};
-      uint32_t used[5] = {0, 0, 0, 0, 0};
-      int exc[5] = {0, 0, 0, 0, 0};
-      int d = 0, budget = 1 << 16;
-      while (d >= 0 && !found) {
+  const int n = s.nbig, need = __popc(realset) - 8;
+  if (n > kMaxBig) {
+    found = 1;
+  } else {
+    int budget = 1 << 14;  // per lane; exceeding it answers "maybe" (exactness kept)
+    for (int i0 = lane; i0 < n && !found; i0 += 32) {
+      const uint32_t b0 = s.big[i0];
+      int idx[3];
+      uint32_t used[4];
+      int exc[4];
+      used[0] = b0;
+      exc[0] = __popc(b0) - 2;
+      if (exc[0] >= need) { found = 1; break; }
+      int d = 0;
+      idx[0] = i0 + 1;
+      while (d >= 0) {
         if (--budget < 0) { found = 1; break; }
-        if (idx[d] >= n || d == 4) {          // level exhausted: backtrack
+        if (idx[d] >= n) {                    // level exhausted: backtrack
           --d;
           if (d >= 0) ++idx[d];
           continue;
@@ -250,11 +259,11 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
         used[d + 1] = used[d] | b;
         exc[d + 1] = exc[d] + __popc(b) - 2;
         if (exc[d + 1] >= need) { found = 1; break; }
-        if (d + 1 < 4) { idx[d + 1] = idx[d] + 1; ++d; } else { ++idx[d]; }
+        if (d + 1 < 3) { idx[d + 1] = idx[d] + 1; ++d; } else { ++idx[d]; }
       }
     }
   }
-  return __shfl_sync(kFull, found, 0) != 0;
+  return __any_sync(kFull, found) != 0;
 }
 
 // Alg. 1 + reorder retry on one tile, executed by one full warp.  On entry
@@ -414,18 +423,34 @@ __global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const RowMask* __r
 // DENSE mode: only the partial last tile of S_p is built here, and the
 // evicted columns of all tiles, in tile and eviction order, form the residual
 // list R_p (left at the front of the panel's queue buffer, count in nres[p]).
-__global__ void __launch_bounds__(32) k_overflow(const RowMask* __restrict__ masks,
-                                                 const int32_t* __restrict__ S,
-                                                 const int32_t* __restrict__ Kp, int64_t K,
-                                                 Scratch sc, int32_t* __restrict__ queue,
-                                                 int64_t qcap, int32_t* __restrict__ T,
-                                                 int* __restrict__ err, int mode,
-                                                 int32_t* __restrict__ nres) {
-  __shared__ TileSmem s;
-  const int p = blockIdx.x, lane = threadIdx.x;
+//
+// One CTA of kR4Warps warps per panel, in waves.  CR1 pops the FIFO one tile at a
+// time, each tile appending its evictions at the back; so every tile whose 16
+// columns are already in the queue when a wave starts sees exactly the columns
+// the sequential algorithm would give it (appends only go behind it).  A wave
+// searches all such tiles in parallel (one warp per tile), then appends their
+// evictions in tile order.  When fewer than 16 columns are queued, every earlier
+// tile is done and the one (partial) tile is popped exactly as in CR1.  The
+// result is bit-identical to the sequential queue (tests compare with the oracle).
+constexpr int kR4Warps = 8;
+__global__ void __launch_bounds__(32 * kR4Warps) k_overflow(const RowMask* __restrict__ masks,
+                                                            const int32_t* __restrict__ S,
+                                                            const int32_t* __restrict__ Kp, int64_t K,
+                                                            Scratch sc, int32_t* __restrict__ queue,
+                                                            int64_t qcap, int32_t* __restrict__ T,
+                                                            int* __restrict__ err, int mode,
+                                                            int32_t* __restrict__ nres) {
+  extern __shared__ __align__(16) uint8_t r4_smem[];
+  TileSmem* sm = reinterpret_cast<TileSmem*>(r4_smem);
+  __shared__ int64_t s_head, s_tail;
+  __shared__ int s_t, s_nw, s_stop;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int p = blockIdx.x;
   const int kp = Kp[p], nfull = kp / 16, rem = kp - 16 * nfull;
   int32_t* q = queue + (int64_t)p * qcap;
   if (mode == 1) {
+    if (warp != 0) return;
+    TileSmem& s = sm[0];
     int t = nfull;
     if (rem > 0) {
       if (lane < 16) {
@@ -453,37 +478,68 @@ __global__ void __launch_bounds__(32) k_overflow(const RowMask* __restrict__ mas
   }
   // FIFO contents after the full tiles: the rest of S_p, then the columns the full
   // tiles evicted, in tile order and eviction order (exactly CR1's sequential queue).
-  for (int i = lane; i < rem; i += 32) q[i] = S[(int64_t)p * K + 16 * nfull + i];
-  int64_t tail = rem;
-  for (int t = 0; t < nfull; ++t) {
-    const int n = sc.tnev[(int64_t)p * sc.cap + t];
-    if (lane < n) q[tail + lane] = sc.tev[((int64_t)p * sc.cap + t) * 16 + lane];
-    tail += n;
-  }
-  __syncwarp();
-  int64_t head = 0;
-  int t = nfull;
-  while (head < tail) {
-    if (t >= sc.cap || tail + 16 > qcap) {
-      if (lane == 0) atomicExch(err, 1);
-      break;
+  if (warp == 0) {
+    for (int i = lane; i < rem; i += 32) q[i] = S[(int64_t)p * K + 16 * nfull + i];
+    int64_t tail = rem;
+    for (int t = 0; t < nfull; ++t) {
+      const int n = sc.tnev[(int64_t)p * sc.cap + t];
+      if (lane < n) q[tail + lane] = sc.tev[((int64_t)p * sc.cap + t) * 16 + lane];
+      tail += n;
     }
-    if (lane < 16) {
-      const int32_t c = head + lane < tail ? q[head + lane] : kPad;
-      s.cols[lane] = c;
-      s.m[lane] = c == kPad ? zero_mask() : masks[(int64_t)p * K + c];
+    if (lane == 0) {
+      s_head = 0;
+      s_tail = tail;
+      s_t = nfull;
+      s_stop = 0;
     }
-    head = min(head + 16, tail);
-    __syncwarp();
-    tile_search(s, lane);
-    store_tile(s, sc, p, t, lane);
-    if (lane < s.nev) q[tail + lane] = s.ev[lane];
-    tail += s.nev;
-    ++t;
-    __syncwarp();
   }
-  if (lane == 0) {
-    T[p] = t;
+  __syncthreads();
+  for (;;) {
+    if (threadIdx.x == 0) {
+      const int64_t avail = s_tail - s_head;
+      int nw = avail >= 16 ? (int)(avail / 16) : (avail > 0 ? 1 : 0);
+      if (nw > 0 && (s_t + nw > sc.cap || s_tail + 16 * (int64_t)nw > qcap)) {
+        atomicExch(err, 1);
+        nw = 0;
+      }
+      s_nw = nw;
+    }
+    __syncthreads();
+    const int nw = s_nw;
+    if (nw == 0) break;
+    const int64_t head = s_head, tail0 = s_tail;
+    const int t0 = s_t;
+    for (int k = warp; k < nw; k += kR4Warps) {
+      TileSmem& s = sm[warp];
+      if (lane < 16) {
+        const int64_t pos = head + 16 * (int64_t)k + lane;
+        const int32_t c = pos < tail0 ? q[pos] : kPad;
+        s.cols[lane] = c;
+        s.m[lane] = c == kPad ? zero_mask() : masks[(int64_t)p * K + c];
+      }
+      __syncwarp();
+      tile_search(s, lane);
+      store_tile(s, sc, p, t0 + k, lane);
+      __syncwarp();
+    }
+    __syncthreads();
+    if (warp == 0) {  // the wave's evictions, in tile order
+      int64_t tail = tail0;
+      for (int k = 0; k < nw; ++k) {
+        const int n = sc.tnev[(int64_t)p * sc.cap + t0 + k];
+        if (lane < n) q[tail + lane] = sc.tev[((int64_t)p * sc.cap + t0 + k) * 16 + lane];
+        tail += n;
+      }
+      if (lane == 0) {
+        s_head = min(head + 16 * (int64_t)nw, tail0);
+        s_tail = tail;
+        s_t = t0 + nw;
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    T[p] = s_t;
     nres[p] = 0;
   }
 }
@@ -709,7 +765,16 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   k_compact<<<npan, 1024, 0, stream>>>(masks, K, S, Kp);
   k_main_tiles<<<dim3((unsigned)((K / 16 + kR3Warps - 1) / kR3Warps), npan), 32 * kR3Warps, 0, stream>>>(
       masks, S, Kp, K, sc);
-  k_overflow<<<npan, 32, 0, stream>>>(masks, S, Kp, K, sc, queue, qcap, T, err, mode, nres);
+  {
+    static bool attr_set[64] = {};
+    if (dev >= 0 && dev < 64 && !attr_set[dev]) {
+      JIG_CU(cudaFuncSetAttribute(k_overflow, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)(kR4Warps * sizeof(TileSmem))), "cudaFuncSetAttribute(k_overflow)");
+      attr_set[dev] = true;
+    }
+  }
+  k_overflow<<<npan, 32 * kR4Warps, kR4Warps * sizeof(TileSmem), stream>>>(masks, S, Kp, K, sc, queue, qcap, T, err,
+                                                                          mode, nres);
   JIG_CU(cudaGetLastError(), "reorder kernels launch");
   JIG_CU(cudaMemcpyAsync(hKp.data(), Kp, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy Kp");
   JIG_CU(cudaMemcpyAsync(hT.data(), T, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy T");
