@@ -143,6 +143,7 @@ struct TileSmem {
   int32_t ev[16];         // evicted columns, in eviction order
   uint8_t perm[16];
   int nev;
+  int stop;               // cover_exists: some lane found a cover (the others stop)
 };
 
 __device__ __forceinline__ bool compat(const TileSmem& s, uint32_t sub) {
@@ -201,7 +202,10 @@ __device__ bool complete_cover(const TileSmem& s, uint32_t used, uint32_t& o1, u
 // sum(|b_i| - 2) >= nreal - 8.  Falls back to "maybe" (true) when the
 // candidate list or the search budget overflows.
 __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
-  if (lane == 0) s.nbig = 0;
+  if (lane == 0) {
+    s.nbig = 0;
+    s.stop = 0;
+  }
   __syncwarp();
   for (int k = lane; k < kNumSubsets; k += 32) {          // 4 real columns
     const uint32_t sub = g_subs[k];
@@ -236,8 +240,9 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
   if (n > kMaxBig) {
     found = 1;
   } else {
-    int budget = 1 << 14;  // per lane; exceeding it answers "maybe" (exactness kept)
-    for (int i0 = lane; i0 < n && !found; i0 += 32) {
+    int budget = 1 << 13;  // per lane; exceeding it answers "maybe" (exactness kept)
+    volatile int* stop = &s.stop;
+    for (int i0 = lane; i0 < n && !found && !*stop; i0 += 32) {
       const uint32_t b0 = s.big[i0];
       int idx[3];
       uint32_t used[4];
@@ -249,6 +254,7 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
       idx[0] = i0 + 1;
       while (d >= 0) {
         if (--budget < 0) { found = 1; break; }
+        if ((budget & 63) == 0 && *stop) break;  // another lane already answered
         if (idx[d] >= n) {                    // level exhausted: backtrack
           --d;
           if (d >= 0) ++idx[d];
@@ -261,6 +267,7 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
         if (exc[d + 1] >= need) { found = 1; break; }
         if (d + 1 < 3) { idx[d + 1] = idx[d] + 1; ++d; } else { ++idx[d]; }
       }
+      if (found) *stop = 1;
     }
   }
   return __any_sync(kFull, found) != 0;

@@ -4,22 +4,31 @@
 // (deepened pipeline: gather indices fetched ahead of the B copies), re-designed
 // for tcgen05:
 //
-//   320 threads, warp-specialised, mbarrier ring of kStages k-blocks
+//   512 threads (16 warps), warp-specialised, mbarrier ring of kStages k-blocks
 //   (k-block = 4 k-steps = 128 logical columns = 8 tiles):
 //     warp 0      A/E producer : cp.async.bulk of the compressed A image (4 KB per
-//                               k-step) and of the TMEM metadata block (2 KB)
-//     warps 6-9   B producers  : warp w gathers the 32 B rows of k-step w with
-//                               16-byte cp.async straight into the SW128 MN-major
-//                               UMMA layout (PAD rows / columns >= N zero-filled)
+//                               k-step) and of the TMEM metadata block (2 KB); a
+//                               second cursor fills the gather-list ring ahead
+//     warps 6-15  B producers  : 8 warps (9 and 13 idle: SM sub-partition 1 is
+//     except 9,13               left to the MMA warp) gather the B rows of the
+//                               k-block with 16-byte cp.async straight into the
+//                               SW128 MN-major UMMA layout (PAD rows / columns
+//                               >= N zero-filled)
 //     warp 1      MMA issuer   : tcgen05.cp metadata -> TMEM, then per k-step one
-//                               tcgen05.mma.sp.kind::f16 M=128 N=NT K=32 (logical)
-//                               into a double-buffered fp32 TMEM accumulator
-//     warps 2-5   epilogue     : tcgen05.ld -> fp16 (RN) -> C rows < M
-//   work unit = (panel of 128 rows, NT columns of C), panels fastest.
-//   Split-K (few units, e.g. the DLMC shapes of BASELINE configs[1]): a cluster
-//   of S CTAs shares one unit, each CTA runs 1/S of the panel's k-blocks, and
-//   the fp32 partial tiles are reduce-scattered through DSMEM with st.async
-//   (owner CTA r sums rows [r*128/S, (r+1)*128/S) and writes them to C).
+//                               tcgen05.mma.sp.kind::f16 (M = 128, or M = 256 on a
+//                               CTA pair) x N = NT x K = 32 (logical) into fp32
+//                               TMEM accumulators; odd CTA of a pair: the relay
+//     warps 2-5   epilogue     : tcgen05.ld -> fp16 (RN) -> C rows < M (and the
+//                               first unit's initial loads at kernel start)
+//   Launched with programmatic stream serialization: everything before
+//   griddepcontrol.wait touches only handle-owned data.
+//   Work unit = (panel, NT columns of C).  Persistent grouped launches (a
+//   dynamic tile scheduler, or a static LPT schedule for CTA pairs) split long
+//   units into k-range pieces reduced by the last piece to finish.  Split-K for
+//   single small products: a cluster of S CTAs shares one unit, each CTA runs
+//   1/S of the panel's k-blocks, and the fp32 partial tiles are reduce-scattered
+//   through DSMEM by bulk copies (owner CTA r sums rows [r*128/S, (r+1)*128/S)
+//   and writes them to C).
 #include <cuda_fp16.h>
 
 #include <algorithm>
