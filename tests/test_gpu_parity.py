@@ -272,6 +272,29 @@ def test_full_size_sampled(M, K, v, s, N):
     spmm_check(C, A, B, rows=rows)
 
 
+@pytest.mark.parametrize("M,P", [(2049 * 128 - 40, 128), (1040 * 256 + 8, 256)])
+def test_parameter_table_capacity_fallbacks(M, P):
+    """Tall matrices past the grouped launch's parameter tables: more panels than
+    the in-parameter panel table holds (1024: the kernel reads the device copy)
+    and, at P = 128, more work units than the host schedule list holds (2048:
+    units are decoded by scanning the problem table).  Format bit-exact on
+    sampled panels, C on sampled rows (incl. the ragged last panel)."""
+    K, v, s, N = 64, 8, 0.9, 64
+    A = synth.vector_sparse(M, K, v, s, 17)
+    B = synth.dense_b(K, N, 17)
+    h = jig.reorder(_dev(A), v, panel_rows=P)
+    g = h.export()
+    npan = (M + P - 1) // P
+    for p in sorted({0, 1500 % npan, npan - 1}):
+        ref = oracle.reorder(A, P=P, panels=(p, p + 1))
+        assert_format_equal(g, ref, panels=(p, p + 1))
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(1)
+    rows = np.sort(np.concatenate([rng.choice(M, size=40, replace=False), np.arange(M - 8, M)]))
+    spmm_check(C, A, B, rows=rows)
+
+
 @pytest.mark.parametrize("force", ["1", "2", "4", "8"])
 @pytest.mark.parametrize("M,K,v,s,N", [(512, 2048, 4, 0.9, 256), (384, 700, 8, 0.8, 200),
                                        (256, 96, 2, 0.95, 64)])
