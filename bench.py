@@ -226,7 +226,7 @@ def run_reference(args):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": desc, "l2": "n/a (CPU)"},
             "cpu_baseline": {"value": val, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, "cpu_model": cpu_model()},
             "e2e": {"value": val, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
     return 0
@@ -252,7 +252,18 @@ def cpu_baseline(points, mats, budget_s=12.0):
     dt = time.perf_counter() - t0
     return {"value": fl / dt / 1e12, "unit": "TFLOP/s", "cores": 1, "kind": "oracle",
             "sample": f"first {rows} rows of each of the {len(points)} matrices, full N "
-                      f"({dt:.1f} s of CPU work)"}
+                      f"({dt:.1f} s of CPU work)", "cpu_model": cpu_model()}
+
+
+def cpu_model() -> str:
+    """Host CPU model (the CPU baseline's hardware)."""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 # ------------------------------------------------------------------ jigsaw arm
