@@ -286,6 +286,9 @@ __device__ void tile_search(TileSmem& s, int lane) {
     for (int i = lane; i < 2048; i += 32) s.bitmap[i] = 0;
     __syncwarp();
     int fr = 0, hmax = 0;
+    // freq counters, per lane: slot j counts in byte (j & 3) of word j >> 2 (<= 57
+    // subsets per lane, no byte overflow); reduced over the warp once, below
+    uint32_t pc0 = 0, pc1 = 0, pc2 = 0, pc3 = 0;
     for (int k0 = 0; k0 < kNumSubsets; k0 += 32) {
       const int k = k0 + lane;
       bool ok = false;
@@ -302,13 +305,31 @@ __device__ void tile_search(TileSmem& s, int lane) {
         if (ok) {
           atomicOr(&s.bitmap[sub >> 5], 1u << (sub & 31));
           hmax = max(hmax, __popc(sub & realset));
+          // nibble -> one count per byte: (n * 0x00204081) & 0x01010101
+          pc0 += ((sub & 0xFu) * 0x00204081u) & 0x01010101u;
+          pc1 += (((sub >> 4) & 0xFu) * 0x00204081u) & 0x01010101u;
+          pc2 += (((sub >> 8) & 0xFu) * 0x00204081u) & 0x01010101u;
+          pc3 += (((sub >> 12) & 0xFu) * 0x00204081u) & 0x01010101u;
         }
       }
-      // freq[j] = number of compatible groups containing slot j
+    }
+    {
+      // freq[j] = number of compatible groups containing slot j: the byte
+      // counters widened to 16-bit halves (<= 455 each) and summed over the warp
+      const uint32_t pw[4] = {pc0, pc1, pc2, pc3};
+      uint32_t tot[8];
 #pragma unroll
-      for (int j = 0; j < 16; ++j) {
-        const unsigned bj = __ballot_sync(kFull, ok && ((sub >> j) & 1u));
-        if (lane == j) fr += __popc(bj);
+      for (int w = 0; w < 4; ++w) {
+        tot[2 * w] = __reduce_add_sync(kFull, pw[w] & 0x00FF00FFu);             // bytes 0, 2
+        tot[2 * w + 1] = __reduce_add_sync(kFull, (pw[w] >> 8) & 0x00FF00FFu);  // bytes 1, 3
+      }
+      if (lane < 16) {
+        const int w = lane >> 2, b = lane & 3;
+        uint32_t t = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+          if (i == 2 * w + (b & 1)) t = tot[i];
+        fr = (int)((t >> (16 * (b >> 1))) & 0xFFFFu);
       }
     }
     for (int o = 16; o; o >>= 1) hmax = max(hmax, __shfl_xor_sync(kFull, hmax, o));
