@@ -446,4 +446,10 @@ __device__ __forceinline__ void st_async_v4(uint32_t raddr, uint32_t a, uint32_t
 // of the stream) have completed and their memory is visible.  A no-op when the
 // launch carries no programmatic dependency.
 __device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// Allow the dependent grid (the next kernel of the stream launched with the
+// programmatic attribute) to be scheduled once every CTA of this grid has
+// issued this or exited.
+__device__ __forceinline__ void griddep_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
 }  // namespace jig

@@ -45,6 +45,9 @@
 #ifndef JIG_RELAY
 #define JIG_RELAY 1  // pair relay: bit 0 fence.proxy.async, bit 1 release.cluster arrive (else relaxed; release: C4 +16 %)
 #endif
+#ifndef JIG_EARLY_TRIGGER
+#define JIG_EARLY_TRIGGER 1  // griddepcontrol.launch_dependents once a CTA has fetched its last unit
+#endif
 #ifndef JIG_HALVES
 #define JIG_HALVES 0  // pair N = 256 as two 128-column halves (see Cfg::kHalves); measured slower
 #endif
@@ -627,6 +630,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           atomicExch(&g_sched[prm.sched][1], 0);
         }
       }
+      // This CTA takes no more units: once every CTA got here (all of them are
+      // resident, so this cannot starve the grid), the next kernel of the stream
+      // may launch and run its prologue on the SMs this grid frees; its B / C /
+      // workspace / scheduler accesses still wait for this grid to complete.
+      if (JIG_EARLY_TRIGGER) griddep_launch_dependents();
     }
   } else if (bprod_index(warp) >= 0) {
     // ------------------------------------------------------------ B producers
