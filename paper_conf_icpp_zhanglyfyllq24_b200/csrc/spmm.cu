@@ -389,6 +389,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   const uint32_t s_last = smem_u32(tmem_slot + 1);  // split piece: this CTA reduces (int flag)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (JIG_EARLY_TRIGGER == 2 && threadIdx.x == 0) griddep_launch_dependents();  // at entry (A/B option)
   const int S = kSplit ? prm.S : 1;
   const int CS = kPair ? 2 : S;  // CTAs per cluster
   const uint32_t rank = (kSplit || kPair) ? cluster_ctarank() : 0;
@@ -634,7 +635,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       // resident, so this cannot starve the grid), the next kernel of the stream
       // may launch and run its prologue on the SMs this grid frees; its B / C /
       // workspace / scheduler accesses still wait for this grid to complete.
-      if (JIG_EARLY_TRIGGER) griddep_launch_dependents();
+      if (JIG_EARLY_TRIGGER == 1) griddep_launch_dependents();
     }
   } else if (bprod_index(warp) >= 0) {
     // ------------------------------------------------------------ B producers
