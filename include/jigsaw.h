@@ -124,7 +124,11 @@ JIGSAW_API jigsaw_handle_t jigsaw_reorder(const void* A, int64_t M, int64_t K, i
  *   N > 0, N % 8 == 0 (TMA needs 16-byte rows).
  * Asynchronous on `stream`; no host synchronisation and no allocation.  The handle
  * is immutable, so calls may run concurrently on several streams.  C must not
- * alias B. */
+ * alias B.  The kernel is launched with programmatic stream serialization: it
+ * may start while the previous kernel of `stream` drains, but reads B and
+ * writes C only after that kernel has completed (stream order is preserved for
+ * B and C); it lets the next programmatic launch on `stream` start once its own
+ * last work unit is scheduled.  JIGSAW_PDL=0 in the environment disables this. */
 JIGSAW_API jigsaw_status_t jigsaw_spmm(jigsaw_handle_t h, const void* B, int64_t N, void* C,
                             jigsaw_stream_t stream);
 
