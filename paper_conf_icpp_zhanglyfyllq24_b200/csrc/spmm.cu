@@ -1014,7 +1014,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         // st.async per lane moved ~15 B/clk)
         const int rpo = 128 / S;                           // rows owned per CTA
         constexpr int kMaxRun = 32;                        // rows of a warp sent by one copy
-        if (warp == 2 && lane == 0) mbar_arrive_expect_tx(recv_full, (uint32_t)(128 * C_::kRecvStride));
+        // the S - 1 peers' slices of this CTA's rows arrive by bulk copy
+        if (warp == 2 && lane == 0) mbar_arrive_expect_tx(recv_full, (uint32_t)((128 - rpo) * C_::kRecvStride));
         const uint32_t stg = smem_u32(sB + q * 32 * C_::kRecvStride);
 #pragma unroll 1
         for (int c0 = 0; c0 < NT; c0 += 32) {
@@ -1033,18 +1034,25 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         }
         fence_proxy_async();  // the staged rows are read by the bulk copy (async proxy)
         __syncwarp();
-        // one copy per owner of the warp's rows (S = 8: 16-row owners, two copies)
+        // one copy per owner of the warp's rows (S = 8: 16-row owners, two runs);
+        // rows this CTA owns itself are moved inside its shared memory by the warp
         const int run = rpo < kMaxRun ? rpo : kMaxRun;
-        if (lane < 32 / run) {
-          const int r0 = q * 32 + lane * run;
+#pragma unroll 1
+        for (int ri = 0; ri < 32 / run; ++ri) {
+          const int r0 = q * 32 + ri * run;
           const uint32_t owner = (uint32_t)(r0 / rpo);
-          bulk_s2cluster(mapa_shared(smem_u32(sRecv + (rank * rpo + r0 % rpo) * C_::kRecvStride), owner),
-                         stg + lane * run * C_::kRecvStride, run * C_::kRecvStride,
-                         mapa_shared(smem_u32(recv_full), owner));
+          const uint32_t src = stg + ri * run * C_::kRecvStride;
+          const uint32_t dst = smem_u32(sRecv + (rank * rpo + r0 % rpo) * C_::kRecvStride);
+          if (owner == rank) {
+            for (int o = lane * 16; o < run * C_::kRecvStride; o += 32 * 16) st_shared_v4u(dst + o, ld_shared_v4u(src + o));
+          } else if (lane == 0) {
+            bulk_s2cluster(mapa_shared(dst, owner), src, run * C_::kRecvStride, mapa_shared(smem_u32(recv_full), owner));
+          }
         }
         // owner: wait for all S partial slices of its rows, sum, convert, store
         if (warp == 2 && lane == 0) JIG_TRACE(7);
         mbar_wait(recv_full, 0);
+        asm volatile("bar.sync 1, 128;" ::: "memory");  // the local slice, copied by all four warps
         if (warp == 2 && lane == 0) JIG_TRACE(8);
         const int t = threadIdx.x - 64;                    // 0..127
         constexpr int C8 = NT / 8;                         // 8-column groups per row
