@@ -239,19 +239,16 @@ jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const
   return set_status(JIGSAW_SUCCESS);
 }
 
-// Several independent copies in one submission (cudaMemcpyBatchAsync: one
-// driver call instead of one per product -- per-copy submission cost ~40 us
-// through torch, profiles/r01y_pcie.txt); a plain loop if the batch call fails.
+// Several independent copies on one stream: one cudaMemcpyAsync per copy.
+// (The one-submission batch-copy call is not used: it faulted the GPU on this
+// pool's boxes, so the per-copy submission cost stays.)
 static cudaError_t copy_batch(std::vector<void*>& dst, std::vector<void*>& src, std::vector<size_t>& sz,
-                              cudaStream_t st) {
-  if (dst.empty()) return cudaSuccess;
-  cudaMemcpyAttributes attr = {};
-  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-  size_t idx = 0, fail = 0;
-  cudaError_t e = cudaMemcpyBatchAsync(dst.data(), src.data(), sz.data(), dst.size(), &attr, &idx, 1, &fail, st);
-  if (e == cudaSuccess) return e;
-  cudaGetLastError();
-  for (size_t i = 0; i < dst.size() && (e = cudaMemcpyAsync(dst[i], src[i], sz[i], cudaMemcpyDefault, st)) == cudaSuccess; ++i) {
+                              cudaMemcpyKind kind, cudaStream_t st) {
+  // No merging of address-adjacent copies: two host buffers can sit back to
+  // back yet belong to separate pinned registrations, and one copy spanning
+  // both is rejected (invalid argument).
+  cudaError_t e = cudaSuccess;
+  for (size_t i = 0; i < dst.size() && (e = cudaMemcpyAsync(dst[i], src[i], sz[i], kind, st)) == cudaSuccess; ++i) {
   }
   return e;
 }
@@ -334,7 +331,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
       cs.push_back(const_cast<void*>(Bs_host[i]));
       cz.push_back((size_t)hs[i]->f.K * Ns[i] * 2);
     }
-    if (e == cudaSuccess) e = copy_batch(cd, cs, cz, P.h2d);
+    if (e == cudaSuccess) e = copy_batch(cd, cs, cz, cudaMemcpyHostToDevice, P.h2d);
     cudaEvent_t in, done;
     cudaEventCreateWithFlags(&in, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
@@ -358,7 +355,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
       cs.push_back(dC + coff[i]);
       cz.push_back((size_t)hs[i]->f.M * Ns[i] * 2);
     }
-    if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, P.d2h);
+    if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, cudaMemcpyDeviceToHost, P.d2h);
     i0 = i1;
   }
   // staging goes back to the pool after the last copy-out

@@ -600,3 +600,32 @@ def test_spmm_batched_host_pipeline():
     jig.spmm_batched_host(hs, pin_B, pin_C)                   # pinned, overlapped
     for a, b, c in zip(mats, Bs, pin_C):
         spmm_check(c, a, b)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("chunks", ["1", "8"])
+def test_spmm_batched_host_packed_buffers(monkeypatch, chunks):
+    """jigsaw_spmm_batched_host with every B in one pinned block and every C in
+    another (views into one registration, back to back; one product with a
+    size that is not a multiple of 256 B), whole batch as one chunk and as
+    several."""
+    pts = [(256, 512, 4, 0.8, 128), (512, 256, 8, 0.9, 64), (384, 520, 8, 0.8, 72), (256, 256, 4, 0.7, 128)]
+    mats = [synth.vector_sparse(M, K, v, s, 90 + i) for i, (M, K, v, s, N) in enumerate(pts)]
+    Bs = [synth.dense_b(K, N, 95 + i) for i, (M, K, v, s, N) in enumerate(pts)]
+    hs = [jig.reorder(_dev(a), v) for a, (M, K, v, s, N) in zip(mats, pts)]
+    nb = sum(K * N for (M, K, v, s, N) in pts)
+    nc = sum(M * N for (M, K, v, s, N) in pts)
+    blkB = torch.empty(nb, dtype=torch.int16).pin_memory().numpy().view(np.uint16)
+    blkC = torch.empty(nc, dtype=torch.int16).pin_memory().numpy().view(np.uint16)
+    vb, vc, ob, oc = [], [], 0, 0
+    for b, (M, K, v, s, N) in zip(Bs, pts):
+        vb.append(blkB[ob:ob + K * N].reshape(K, N))
+        vb[-1][...] = b.view(np.uint16) if b.dtype == np.float16 else b
+        vc.append(blkC[oc:oc + M * N].reshape(M, N))
+        ob += K * N
+        oc += M * N
+    blkC[...] = 0xFFFF
+    monkeypatch.setenv("JIGSAW_HOST_CHUNKS", chunks)        # 1: the whole batch is one chunk
+    jig.spmm_batched_host(hs, vb, vc)
+    for a, b, c in zip(mats, Bs, vc):
+        spmm_check(c, a, b)
