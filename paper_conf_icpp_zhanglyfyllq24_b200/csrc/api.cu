@@ -306,10 +306,11 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
     cudaEventDestroy(ev0);
     return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "staging allocation failed");
   }
-  // chunks of ~1/8 of the batch's bytes (at least one product; developer
-  // override JIGSAW_HOST_CHUNKS): copy-in of chunk
-  // k+1 and copy-out of chunk k-1 overlap the grouped launch of chunk k
-  const int nchunks = getenv("JIGSAW_HOST_CHUNKS") ? std::max(1, atoi(getenv("JIGSAW_HOST_CHUNKS"))) : 8;
+  // chunks of ~1/16 of the batch's bytes (at least one product; developer
+  // override JIGSAW_HOST_CHUNKS): copy-in of chunk k+1 and copy-out of chunk
+  // k-1 overlap the grouped launch of chunk k (16 measured best with one copy
+  // per product and direction, profiles/r01zt_e2e_chunks.txt)
+  const int nchunks = getenv("JIGSAW_HOST_CHUNKS") ? std::max(1, atoi(getenv("JIGSAW_HOST_CHUNKS"))) : 16;
   const size_t target = std::max<size_t>((bb + cb) / nchunks, 1);
   std::vector<const Format*> fs;
   std::vector<const void*> pb;
