@@ -122,8 +122,14 @@ JIGSAW_API jigsaw_handle_t jigsaw_reorder(const void* A, int64_t M, int64_t K, i
  *   B : device pointer, fp16 row-major K x N (ld = N), 16-byte aligned.
  *   C : device pointer, fp16 row-major M x N (ld = N), 16-byte aligned; overwritten.
  *   N > 0, N % 8 == 0 (TMA needs 16-byte rows).
- * Asynchronous on `stream`; no host synchronisation and no allocation.  The handle
- * is immutable, so calls may run concurrently on several streams.  C must not
+ * Asynchronous on `stream`; no host synchronisation and no allocation, except
+ * that the first grouped launch with split units (long units cut into k-range
+ * pieces) on a device grows the library's fp32 partial-tile workspace (one
+ * cudaMalloc + device synchronisation, outside stream capture; inside a capture
+ * such a launch runs whole units instead).  The handle is immutable, so calls may
+ * run concurrently on several streams: each stream gets its own workspace
+ * regions (up to 8 streams per device; beyond that streams share regions and
+ * must not run split launches at the same time).  C must not
  * alias B.  The kernel is launched with programmatic stream serialization: it
  * may start while the previous kernel of `stream` drains, but reads B and
  * writes C only after that kernel has completed (stream order is preserved for

@@ -33,6 +33,9 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <mutex>
+#include <utility>
+#include <vector>
 #include <string>
 #include <type_traits>
 
@@ -1358,44 +1361,61 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   return launch_params(prm, NT, S, grid, f.device, pair, s);
 }
 
-// Device workspace for the fp32 partial tiles of split units: R regions used
-// round-robin by successive launches (so back-to-back or concurrently replayed
-// launches do not share partials), each region = [counters | partial tiles].
-// Grown outside stream capture only; counters are zeroed once at allocation and
+// Device workspace for the fp32 partial tiles of split units, each region =
+// [counters | partial tiles].  The regions come in pairs; every stream that
+// launches split units gets its own pair on first use (kWsPairs streams per
+// device before pairs are shared) and alternates between its two regions, so
+// launches on different streams never share partials, and back-to-back
+// launches on one stream (which may overlap under programmatic dependent
+// launch) do not either.  Assigning a pair allocates nothing, so a capture
+// stream seen for the first time inside a capture still gets one.  The arena
+// grows outside stream capture only; counters are zeroed at allocation and
 // reset by the last piece of every unit.
+constexpr int kWsPairs = 8;
 struct SplitWs {
   char* base = nullptr;
   size_t region = 0;
-  int next = 0;
+  int next_pair = 0;
+  std::vector<std::pair<cudaStream_t, int>> pair_of;  // stream -> pair index
+  int toggle[kWsPairs] = {};
 };
-constexpr int kWsRegions = 4;
 SplitWs g_ws[64];
+std::mutex g_ws_mu;
 
 static bool split_workspace(int dev, size_t tile_bytes, size_t cnt_bytes, cudaStream_t s, float** ws, int** wcnt) {
   if (dev < 0 || dev >= 64) return false;
+  std::lock_guard<std::mutex> lock(g_ws_mu);
   SplitWs& w = g_ws[dev];
   const size_t need = ((cnt_bytes + 255) & ~size_t(255)) + tile_bytes;
   if (need > w.region) {
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return false;
-    if (cudaStreamSynchronize(s) != cudaSuccess) return false;
+    if (cudaDeviceSynchronize() != cudaSuccess) return false;  // every stream's use of the old arena is done
     if (w.base) cudaFree(w.base);
     w.base = nullptr;
     w.region = 0;
     const size_t region = std::max(need, (size_t)8 << 20);
-    if (cudaMalloc(&w.base, region * kWsRegions) != cudaSuccess) {
+    if (cudaMalloc(&w.base, region * 2 * kWsPairs) != cudaSuccess) {
       cudaGetLastError();
       w.base = nullptr;
       return false;
     }
-    if (cudaMemset(w.base, 0, region * kWsRegions) != cudaSuccess) {
+    if (cudaMemset(w.base, 0, region * 2 * kWsPairs) != cudaSuccess) {
       cudaFree(w.base);
       w.base = nullptr;
       return false;
     }
     w.region = region;
   }
-  char* r = w.base + (size_t)(w.next++ % kWsRegions) * w.region;
+  int pi = -1;
+  for (const auto& e : w.pair_of)
+    if (e.first == s) pi = e.second;
+  if (pi < 0) {
+    pi = w.next_pair++ % kWsPairs;
+    w.pair_of.push_back({s, pi});
+  }
+  const int ri = 2 * pi + (w.toggle[pi]++ & 1);
+  char* r = w.base + (size_t)ri * w.region;
   *wcnt = reinterpret_cast<int*>(r);
   *ws = reinterpret_cast<float*>(r + ((cnt_bytes + 255) & ~size_t(255)));
   return true;
