@@ -5,6 +5,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <string>
 
@@ -57,10 +58,12 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 // Stream-ordered staging memory for the host-buffer entry points: a private pool
 // per device that keeps its memory (no release to the OS between calls).
 cudaMemPool_t g_pool[64] = {};
+std::mutex g_lazy_mu;  // guards the lazy creation of the pools and pipeline streams
 cudaError_t staging_alloc(void** p, size_t bytes, cudaStream_t st) {
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) return cudaMallocAsync(p, bytes, st);
+  std::lock_guard<std::mutex> lock(g_lazy_mu);
   if (!g_pool[dev]) {
     cudaMemPoolProps props = {};
     props.allocType = cudaMemAllocationTypePinned;
@@ -273,6 +276,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
   const int dev = hs[0]->f.device;
   if (dev < 0 || dev >= 64) return set_status(JIGSAW_ERROR_INTERNAL, "device ordinal out of range");
   HostPipe& P = g_pipe[dev];
+  std::unique_lock<std::mutex> lazy(g_lazy_mu);
   if (!P.h2d) {
     if (cudaStreamCreateWithFlags(&P.h2d, cudaStreamNonBlocking) != cudaSuccess ||
         cudaStreamCreateWithFlags(&P.comp, cudaStreamNonBlocking) != cudaSuccess ||
@@ -282,6 +286,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
       return set_status(JIGSAW_ERROR_CUDA, "cudaStreamCreate failed");
     }
   }
+  lazy.unlock();
   cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
   // staging for the whole batch (one pool allocation each for B and C)
   size_t bb = 0, cb = 0;

@@ -32,6 +32,7 @@
 #include <cuda_fp16.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <mutex>
 #include <utility>
@@ -1262,7 +1263,7 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
 
 int g_trace_ctas = 0;
 
-int g_sched_next[64] = {0};
+std::atomic<unsigned> g_sched_next[64] = {};  // slot rotation, shared by host threads (unsigned: wraps)
 
 template <class Prm>
 static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, bool pair, cudaStream_t s,
@@ -1283,7 +1284,7 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   prm.nunits = npieces_total >= 0 ? npieces_total : u;
   // (a CTA per unit needs no scheduler: its one unit is known at kernel start)
   if (S == 1 && !pair && grid < prm.nunits && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
-    prm.sched = (g_sched_next[dev]++) % kSchedSlots;
+    prm.sched = (int)(g_sched_next[dev]++ % kSchedSlots);
   constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 8;
   if (pair) {
     if (NT == 256) return launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s);

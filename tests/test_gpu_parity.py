@@ -665,3 +665,42 @@ def test_grouped_split_pieces_two_streams():
     for dC in outs:
         for r, c in zip(refs, dC):
             assert np.array_equal(_host(c).view(np.float16).astype(np.float64), r)
+
+
+def test_host_threads_concurrent_calls():
+    """Four host threads call jigsaw_spmm_batched_host and jigsaw_spmm_batched at
+    once (ctypes releases the GIL, so the calls really overlap in the library:
+    lazily created pools, pipeline streams and workspace assignment under
+    contention); every C against the oracle."""
+    import threading
+    pts = [(256, 512, 4, 0.8, 64), (384, 700, 8, 0.9, 72)]
+    mats = [synth.vector_sparse(M, K, v, s, 700 + i) for i, (M, K, v, s, N) in enumerate(pts)]
+    Bs = [synth.dense_b(K, N, 710 + i) for i, (M, K, v, s, N) in enumerate(pts)]
+    hs = [jig.reorder(_dev(a), v) for a, (M, K, v, s, N) in zip(mats, pts)]
+    dB = [_dev(b) for b in Bs]
+    torch.cuda.synchronize()
+    results, errors = {}, []
+
+    def work(t):
+        try:
+            torch.cuda.set_device(0)
+            if t % 2:
+                results[t] = jig.spmm_batched_host(hs, Bs)
+            else:
+                st = torch.cuda.Stream()
+                dC = [torch.empty((M, N), dtype=torch.float16, device="cuda") for (M, K, v, s, N) in pts]
+                jig.spmm_batched(hs, dB, dC, stream=st)
+                st.synchronize()
+                results[t] = [_host(c) for c in dC]
+        except Exception as e:                  # noqa: BLE001 -- reported below
+            errors.append(repr(e))
+
+    ths = [threading.Thread(target=work, args=(t,)) for t in range(4)]
+    for th in ths:
+        th.start()
+    for th in ths:
+        th.join()
+    assert not errors, errors
+    for t in range(4):
+        for a, b, c in zip(mats, Bs, results[t]):
+            spmm_check(c, a, b)
