@@ -3,29 +3,40 @@
 (BASELINE.json metric) for the Jigsaw hot path on B200.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c2|c1|c3|c4|c5a|c5b|venom]
-                  [--impl jigsaw|reference]
+                  [--impl jigsaw|reference] [--panel-rows 0|128|256] [--no-extra] [--multi]
 
 A STEP is one pass of the SpMM hot path over one batch of synthetic matrices
 with the prepared formats resident in HBM (the paper times the kernel only and
 excludes format conversion): for the default workload (BASELINE
 configs[1], "C2") the batch is the 36 DLMC-transformer-shaped matrices
-512x2048 / 2048x512 x v in {2,4,8} x s in {.50,.70,.80,.90,.95,.98}, N = 256.
-  value   = sum over the batch of 2*M*N*K (dense-equivalent flops) / step time
-  e2e     = the same metric through the C ABI with HOST buffers
-            (jigsaw_spmm_batched_host: the batch's B's host->device, grouped SpMM,
-            C's device->host, every step; chunks overlap on three streams)
-  e2e_full= + the reorder of A from host memory (jigsaw_reorder_host) every step,
-            i.e. every §8(a) row of the hot path
-L2 is flushed (256 MB write) before every timed step; per-step device time is
-taken with CUDA events on the launching stream and summed; multi-GPU: one
-process per GPU (torchrun), weak scaling (each rank its own batch, seeds offset
-by rank), barrier + synchronize around the timed region, max over ranks.
+512x2048 / 2048x512 x v in {2,4,8} x s in {.50,.70,.80,.90,.95,.98}, N = 256,
+issued as ONE jigsaw_spmm_batched call (one grouped k_spmm launch).
+  value    = sum over the batch of 2*M*N*K (dense-equivalent flops) / step time
+  e2e      = the same metric through the C ABI with HOST buffers
+             (jigsaw_spmm_batched_host: the batch's B's host->device, grouped
+             SpMM, C's device->host, every step)
+  e2e_full = + the reorder of A from host memory (jigsaw_reorder_host) every
+             step, i.e. every §8(a) row of the hot path
+  cublas   = the same products as dense fp16 GEMMs in cuBLAS (the paper's
+             baseline): per matrix (cublasGemmEx, best of COMPUTE_16F and
+             COMPUTE_32F, L2 flushed before every call) and as a batch (one
+             cublasGemmStridedBatchedEx per shape group, best of 16F / 32F,
+             timed exactly like the jigsaw step)
+  c4       = (default run) the same measurements for BASELINE configs[3], the
+             compute-bound Llama-shaped batch, with its tensor roofline
+  c5a/c5b  = (N > 1, or --multi) the sharded sweep of configs[4]: 64 DLMC
+             matrices split by matrix (LPT), and 4096^2 N = 16384 split by C
+             columns; C5b's shards are gathered with NCCL after the timed
+             region and checked, and the ranks' format hashes compared
+L2 is flushed (256 MB write) before every timed step, outside the events;
+per-step device time is taken with CUDA events on the launching stream around
+a CUDA-graph replay of the step; multi-GPU: one process per GPU (torchrun),
+barrier + synchronize around the timed region, max over ranks.
 """
 from __future__ import annotations
 
 import argparse
 import json
-import math
 import os
 import subprocess
 import sys
@@ -116,12 +127,21 @@ def point_seed(i: int, rank: int) -> int:
 
 
 def load_peaks():
+    """HBM GB/s and dense bf16 TF/s (MEASURED_PEAKS.json, driver-written), and the
+    measured tcgen05.mma.sp issue-rate peaks (profiles/sparse_mma_peak.json,
+    tools/probe_pair_rate.cu on this pool's B200)."""
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
         d = json.load(open(p))
-        return float(d["hbm_gbs"]), float(d["bf16_tflops"]), "measured"
+        hbm, bf16, src = float(d["hbm_gbs"]), float(d["bf16_tflops"]), "MEASURED_PEAKS.json"
     except Exception:
-        return 6650.0, 1590.0, "fallback (B200_PROFILING.md)"
+        hbm, bf16, src = 6650.0, 1590.0, "fallback (B200_PROFILING.md)"
+    try:
+        sp = json.load(open(os.path.join(ROOT, "profiles", "sparse_mma_peak.json")))
+    except Exception:
+        sp = {"single_m128_n256_tflops": 2 * bf16, "pair_m256_n256_tflops": 2 * bf16,
+              "source": "2 x dense bf16 (no sparse microbenchmark file)"}
+    return hbm, bf16, src, sp
 
 
 # ------------------------------------------------------------------ clocks
@@ -173,15 +193,16 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ roofline terms
-def algorithmic(info: dict, M: int, K: int, N: int, rows_touched: int):
-    """Per-launch algorithmic bytes and executed flops of k_spmm."""
+def algorithmic(info: dict, M: int, K: int, N: int, rows_touched: int, c_bytes_per_elem: int = 2):
+    """Per-launch algorithmic bytes and executed flops of k_spmm:
+    per tile 16P values + 2P metadata + 64 B gather list, the touched B rows once,
+    C once; executed = logical sparse MMA work 2*P*16*N per tile."""
     P = info["panel_rows"]
-    n_tiles = (N + 127) // 128
-    a_bytes = (16 * P + 2 * P + 64) * info["ntiles"]          # values + metadata + gather per tile
-    b_bytes = 2 * N * rows_touched                              # touched B rows, once
-    c_bytes = 2 * M * N
-    exec_flops = 2 * P * 16 * info["ntiles"] * N               # logical sparse MMA work
-    return a_bytes + b_bytes + c_bytes, exec_flops, n_tiles
+    a_bytes = (16 * P + 2 * P + 64) * info["ntiles"]
+    b_bytes = 2 * N * rows_touched
+    c_bytes = c_bytes_per_elem * M * N
+    exec_flops = 2 * P * 16 * info["ntiles"] * N
+    return a_bytes + b_bytes + c_bytes, exec_flops
 
 
 # ------------------------------------------------------------------ reference arm (CPU oracle)
@@ -266,214 +287,110 @@ def cpu_model() -> str:
     return "unknown"
 
 
-# ------------------------------------------------------------------ jigsaw arm
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
-    ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--workload", default="c2")
-    ap.add_argument("--panel-rows", type=int, default=0, choices=[0, 128, 256],
-                    help="reorder panel height: 0 = library auto (256 for M >= 4096), 128 (one CTA "
-                         "per panel) or 256 (CTA pairs)")
-    ap.add_argument("--impl", default="jigsaw", choices=["jigsaw", "reference"])
-    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
-    ap.add_argument("--no-cublas", action="store_true")
-    ap.add_argument("--detail", action="store_true", help="print the per-point table to stderr")
-    args = ap.parse_args()
-    if args.warmup < 3:
-        args.warmup = 3
-    if args.impl == "reference":
-        return run_reference(args)
+# ------------------------------------------------------------------ the jigsaw arm
+class Batch:
+    """One rank's share of a workload, prepared: formats (jigsaw_reorder, untimed,
+    P:263), device B / C, host copies of A / B, and the roofline terms."""
 
-    import torch
-    import torch.distributed as dist
-    import paper_conf_icpp_zhanglyfyllq24_b200 as jig
+    def __init__(self, name, rank, world, panel_rows, dev, torch, jig):
+        self.name = name
+        self.all_points, self.desc, self.scaling = workload(name)
+        jobs = local_jobs(name, self.all_points, rank, world)
+        self.points = [(M, K, v, s, n1 - n0) for (M, K, v, s, N, seed, n0, n1) in jobs]
+        self.jobs = jobs
+        self.mats, self.hs, self.dA, self.dB, self.dC = [], [], [], [], []
+        self.reorder_ms = 0.0
+        self.alg_bytes = self.exec_flops = self.eff_flops = 0
+        for ji, (M, K, v, s, N, seed, n0, n1) in enumerate(jobs):
+            A = make_a(name, ji, M, K, v, s, seed)
+            B = synth.dense_b(K, N, seed)
+            if (n0, n1) != (0, N):
+                B = np.ascontiguousarray(B[:, n0:n1])
+            N = n1 - n0
+            self.mats.append((A, B))
+            a_t = torch.from_numpy(A.view(np.int16)).to(dev).view(torch.float16)
+            h = jig.reorder(a_t, v, panel_rows=panel_rows)
+            info = h.info()
+            self.reorder_ms += info["reorder_ms"]
+            self.hs.append(h)
+            self.dA.append(a_t)
+            self.dB.append(torch.from_numpy(B.view(np.int16)).to(dev).view(torch.float16))
+            self.dC.append(torch.empty((M, N), dtype=torch.float16, device=dev))
+            rows_touched = int(((A & 0x7FFF) != 0).any(axis=0).sum())
+            ab, ef = algorithmic(info, M, K, N, rows_touched)
+            self.alg_bytes += ab
+            self.exec_flops += ef
+            self.eff_flops += 2 * M * N * K
+        self.pair = any(h.info()["panel_rows"] == 256 for h in self.hs)
+        self.panel_rows_used = sorted(set(h.info()["panel_rows"] for h in self.hs))
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    else:
-        torch.cuda.set_device(0)
-    dev = torch.device("cuda", torch.cuda.current_device())
-    stream = torch.cuda.current_stream()
-    hbm, bf16, peak_src = load_peaks()
+    def step(self, jig):
+        jig.spmm_batched(self.hs, self.dB, self.dC)
 
-    all_points, desc, scaling = workload(args.workload)
-    jobs = local_jobs(args.workload, all_points, rank, world)
-    points = [(M, K, v, s, n1 - n0) for (M, K, v, s, N, seed, n0, n1) in jobs]
-    total_eff = sum(2 * M * K * N for (M, K, v, s, N) in all_points) * (world if scaling == "weak" else 1)
-    mats, hs, dB, dC, dA = [], [], [], [], []
-    reorder_ms = 0.0
-    alg_bytes = exec_flops = eff_flops = 0
-    for ji, (M, K, v, s, N, seed, n0, n1) in enumerate(jobs):
-        A = make_a(args.workload, ji, M, K, v, s, seed)
-        B = synth.dense_b(K, N, seed)
-        if (n0, n1) != (0, N):
-            B = np.ascontiguousarray(B[:, n0:n1])
-        N = n1 - n0
-        mats.append((A, B))
-        a_t = torch.from_numpy(A.view(np.int16)).to(dev).view(torch.float16)
-        h = jig.reorder(a_t, v, panel_rows=args.panel_rows)
-        info = h.info()
-        reorder_ms += info["reorder_ms"]
-        hs.append(h)
-        dA.append(a_t)
-        dB.append(torch.from_numpy(B.view(np.int16)).to(dev).view(torch.float16))
-        dC.append(torch.empty((M, N), dtype=torch.float16, device=dev))
-        rows_touched = int(((A & 0x7FFF) != 0).any(axis=0).sum())
-        ab, ef, _ = algorithmic(info, M, K, N, rows_touched)
-        alg_bytes += ab
-        exec_flops += ef
-        eff_flops += 2 * M * N * K
-    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    def free(self):
+        for h in self.hs:
+            h.free()
 
-    def step_eager():
-        # the whole batch in grouped launches (jigsaw_spmm_batched: <= 64 products per kernel)
-        jig.spmm_batched(hs, dB, dC)
 
-    def step_unbatched():
-        for h, b, c in zip(hs, dB, dC):
-            h.spmm(b, C=c)
-
-    # warm up eagerly (first-call attribute setup), then capture the step in a CUDA
-    # graph so that host launch latency stays out of the device timing
-    for _ in range(2):
-        step_eager()
-        step_unbatched()
+def timed_steps(fn, steps, warmup, flush, stream, torch, dist=None, world=1, dev_index=0):
+    """fn captured in a CUDA graph; W warm-up replays, then K replays each preceded
+    by an L2 flush (outside the events), CUDA events on `stream` around each
+    replay, barrier + synchronize on both sides, clocks sampled during the timed
+    region.  Returns (ms per step, max over ranks; clocks)."""
+    fn()
     torch.cuda.synchronize()
-    graph = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(graph):
-        step_eager()
-    graph_unb = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(graph_unb):
-        step_unbatched()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        fn()
     torch.cuda.synchronize()
-    launches = (len(points) + 63) // 64
-
-    def step():
-        graph.replay()
-
-    for _ in range(args.warmup):
+    for _ in range(max(3, warmup)):
         flush.zero_()
-        step()
+        g.replay()
     torch.cuda.synchronize()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(args.steps)]
-    sampler = ClockSampler(dev.index if dev.index is not None else 0)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    sampler = ClockSampler(dev_index)
     sampler.start()
     time.sleep(0.15)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    for k in range(args.steps):
+    for k in range(steps):
         flush.zero_()                     # L2 flush, outside the timed events
         evs[k][0].record(stream)
-        step()
+        g.replay()
         evs[k][1].record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
     total_ms = sum(a.elapsed_time(b) for a, b in evs)
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    total_ms = float(t.item())
-    ms_per_step = total_ms / args.steps
-    value = total_eff / (ms_per_step * 1e-3) / 1e12   # whole job, all ranks
+    from paper_conf_icpp_zhanglyfyllq24_b200 import shard
+    total_ms = shard.max_over_ranks(total_ms, dist=dist if world > 1 else None,
+                                    device=torch.device("cuda", dev_index))
+    del g
+    return total_ms / steps, clocks
 
-    # roofline of the dominant (only) kernel, k_spmm: algorithmic bytes / flops per
-    # launch over the average launch duration of the timed region
-    t_hbm = alg_bytes / (hbm * 1e9)
-    t_tc = exec_flops / (2 * bf16 * 1e12)          # sparse logical peak = 2x dense
-    if t_hbm >= t_tc:
-        roof = {"bound": "hbm", "achieved": alg_bytes / (ms_per_step * 1e-3) / 1e9, "peak": hbm,
-                "unit": "GB/s"}
-    else:
-        roof = {"bound": "tensor", "achieved": exec_flops / (ms_per_step * 1e-3) / 1e12,
-                "peak": 2 * bf16, "unit": "TFLOP/s"}
-    roof["frac"] = roof["achieved"] / roof["peak"]
-    roof["peak_source"] = peak_src
-    roof["traffic"] = None
-    roof["per_launch_us"] = ms_per_step * 1e3 / launches
-    roof["t_roof_us_per_step"] = max(t_hbm, t_tc) * 1e6
-    try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))[args.workload]
-        roof["traffic"] = prof["bytes_per_step"] / launches
-        roof["traffic_unit"] = "bytes per launch"
-        roof["traffic_source"] = prof.get("source")
-    except Exception:
-        pass
 
-    # per-point detail: jigsaw vs cuBLAS (torch.matmul on the dense fp16 A).  Each
-    # call's device time in a stream of back-to-back kernels, L2 flushed before
-    # every call: [graph of R x (flush, call)] - [graph of R x (flush)], / R (median
-    # of reps) -- the event clock here moves in ~2 us steps, too coarse for
-    # single-call events; the difference over R calls resolves ~0.1 us.
-    detail = []
-    cublas_ms = jig_ms = cslt_ms = 0.0
-    # cuSPARSELt (torch._cslt_*) on natively 2:4 inputs (the f4 workload): the
-    # library 2:4 SpMM, which cannot skip all-zero columns
-    cslt_A, cslt_err = None, None
-    if not args.no_cublas and args.workload == "venom":
-        try:
-            cslt_A = [torch._cslt_compress(a) for a in dA]
-            torch._cslt_sparse_mm(cslt_A[0], dB[0])
-            torch.cuda.synchronize()
-        except Exception as e:  # library without an sm_100 build, or API absent
-            cslt_A, cslt_err = None, f"{type(e).__name__}: {str(e).splitlines()[0][:200]}"
-    if not args.no_cublas:
-        reps, R = 7, 8
+def per_call_us(fn, flush, stream, torch, R=8, reps=7):
+    """Device time of one call in a stream of back-to-back kernels, L2 flushed
+    before every call: ([graph of R x (flush, call)] - [graph of R x flush]) / R,
+    median of `reps` (the event clock moves in ~2 us steps; the difference over
+    R calls resolves ~0.1 us)."""
+    def graphed(f):
+        if f is not None:
+            f()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            for _ in range(R):
+                flush.zero_()
+                if f is not None:
+                    f()
+        return g
 
-        def graphed(fn):
-            if fn is not None:
-                fn()
-            torch.cuda.synchronize()
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g):
-                for _ in range(R):
-                    flush.zero_()
-                    if fn is not None:
-                        fn()
-            return g
-
-        def timeit(g):
-            ts = []
-            for _ in range(reps):
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                e0.record(stream)
-                g.replay()
-                e1.record(stream)
-                e1.synchronize()
-                ts.append(e0.elapsed_time(e1))
-            return float(np.median(ts))
-        g_flush = graphed(None)
-        for i, (M, K, v, s, N) in enumerate(points):
-            t0 = timeit(g_flush)
-            tj = (timeit(graphed(lambda: hs[i].spmm(dB[i], C=dC[i]))) - t0) / R
-            Cref = torch.empty_like(dC[i])
-            tc = (timeit(graphed(lambda: torch.matmul(dA[i], dB[i], out=Cref))) - t0) / R
-            cublas_ms += tc
-            jig_ms += tj
-            d = {"M": M, "K": K, "v": v, "s": s, "N": N, "tag": point_tag(args.workload, i, v, s),
-                 "jigsaw_us": tj * 1e3, "cublas_us": tc * 1e3, "speedup": tc / tj,
-                 "eff_tflops": 2 * M * N * K / (tj * 1e-3) / 1e12}
-            if cslt_A is not None and cslt_A[i] is not None:
-                ts = (timeit(graphed(lambda: torch._cslt_sparse_mm(cslt_A[i], dB[i]))) - t0) / R
-                d["cusparselt_us"] = ts * 1e3
-                d["speedup_vs_cusparselt"] = ts / tj
-                cslt_ms += ts
-            detail.append(d)
-    # step-level comparison: the same batch as one CUDA graph of per-matrix cuBLAS
-    # calls, and of per-matrix jigsaw_spmm calls (36 launches), same flush policy
-    def step_ms(g, reps=30):
+    def timeit(g):
         ts = []
         for _ in range(reps):
-            flush.zero_()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
             g.replay()
@@ -481,112 +398,278 @@ def main():
             e1.synchronize()
             ts.append(e0.elapsed_time(e1))
         return float(np.median(ts))
-    outs = [torch.empty_like(c) for c in dC]
+    t0 = timeit(graphed(None))
+    return (timeit(graphed(fn)) - t0) / R * 1e3
 
-    def cublas_step():
-        for a, b, o in zip(dA, dB, outs):
-            torch.matmul(a, b, out=o)
-    cublas_step()
-    torch.cuda.synchronize()
-    g_cub = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(g_cub):
-        cublas_step()
-    cublas_step_ms = step_ms(g_cub)
-    unbatched_step_ms = step_ms(graph_unb)
-    speed = {}
-    speed_cs = {}
-    for d in detail:
-        speed.setdefault(d["tag"], []).append(d["speedup"])
-        if "speedup_vs_cusparselt" in d:
-            speed_cs.setdefault(d["tag"], []).append(d["speedup_vs_cusparselt"])
-    speed_gm = {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(speed.items())}
-    cslt = None
-    if cslt_A is not None:
-        def cslt_step():
-            for a, b, o in zip(cslt_A, dB, outs):
-                o.copy_(torch._cslt_sparse_mm(a, b))
-        cslt_step()
-        torch.cuda.synchronize()
-        g_cs = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(g_cs):
-            cslt_step()
-        cs_ms = step_ms(g_cs)
-        cslt = {"step_ms": cs_ms, "speedup_step": cs_ms / ms_per_step,
-                "speedup_total_time": (cslt_ms / jig_ms) if jig_ms else None,
-                "speedup_geomean_by_point": {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(speed_cs.items())},
-                "how": "torch._cslt_compress / torch._cslt_sparse_mm (cuSPARSELt 2:4 SpMM) on the natively 2:4 A; "
-                       "per matrix like cuBLAS; step = one CUDA graph of the batch (+ a copy into C per matrix)"}
-    elif cslt_err:
-        cslt = {"unavailable": cslt_err}
 
-    # e2e through the C ABI with host buffers (every step: B in, SpMM, C out)
-    pin_B = [torch.from_numpy(B.view(np.int16)).pin_memory().numpy().view(np.uint16) for (_, B) in mats]
+def roofline(b: Batch, ms_per_launch, peaks, traffic_key=None):
+    """Roofline of k_spmm (the only kernel of the step): algorithmic bytes or
+    executed flops per launch over the measured average launch duration; the
+    binding roof is the larger of bytes / HBM and executed flops / the measured
+    tcgen05.mma.sp peak of the variant (CTA pair or single CTA)."""
+    hbm, bf16, src, sp = peaks
+    sp_peak = sp["pair_m256_n256_tflops"] if b.pair else sp["single_m128_n256_tflops"]
+    t_hbm = b.alg_bytes / (hbm * 1e9)
+    t_tc = b.exec_flops / (sp_peak * 1e12)
+    s = ms_per_launch * 1e-3
+    if t_hbm >= t_tc:
+        r = {"bound": "hbm", "achieved": b.alg_bytes / s / 1e9, "peak": hbm, "unit": "GB/s",
+             "peak_source": src}
+    else:
+        r = {"bound": "tensor", "achieved": b.exec_flops / s / 1e12, "peak": sp_peak, "unit": "TFLOP/s",
+             "peak_source": f"measured tcgen05.mma.sp {'pair M256' if b.pair else 'M128'} N256 issue rate "
+                            f"({sp.get('source', '')}); dense bf16 MEASURED_PEAKS x2 would be {2 * bf16:.0f}"}
+    r["frac"] = r["achieved"] / r["peak"]
+    r["traffic"] = None
+    r["alg_bytes_per_launch"] = b.alg_bytes
+    r["exec_flops_per_launch"] = b.exec_flops
+    r["t_roof_us"] = max(t_hbm, t_tc) * 1e6
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))[traffic_key or b.name]
+        r["traffic"] = prof["bytes_per_launch"]
+        r["traffic_unit"] = "bytes per launch"
+        r["traffic_source"] = prof.get("source")
+    except Exception:
+        pass
+    return r
+
+
+def cublas_compare(b: Batch, flush, stream, torch, jig, jig_step_ms, steps, warmup, per_matrix=True):
+    """cuBLAS dense fp16 GEMM on the dense A of every product (the paper's
+    baseline): per matrix best of CUBLAS_COMPUTE_16F / 32F,
+    and the batch as one strided-batched GEMM per shape group (best of 16F / 32F),
+    timed like the jigsaw step."""
+    from tools import cublas_ref
+    out = {}
+    outs = [torch.empty((M, N), dtype=torch.float16, device=c.device) for c, (M, K, v, s, N) in
+            zip(b.dC, b.points)]
+    groups = {}
+    for i, (M, K, v, s, N) in enumerate(b.points):
+        groups.setdefault((M, K, N), []).append(i)
+    stk = {}
+    for key, idx in groups.items():
+        M, K, N = key
+        stk[key] = (torch.stack([b.dA[i] for i in idx]), torch.stack([b.dB[i] for i in idx]),
+                    torch.empty((len(idx), M, N), dtype=torch.float16, device=b.dA[0].device))
+    batched = {}
+    for comp in ("16F", "32F"):
+        def step(comp=comp):
+            for A3, B3, C3 in stk.values():
+                cublas_ref.gemm_strided_batched(A3, B3, C3, comp)
+        batched[comp], _ = timed_steps(step, steps, warmup, flush, stream, torch)
+    best = min(batched, key=batched.get)
+    out["batched_step_ms"] = batched[best]
+    out["batched_compute"] = best
+    out["batched_step_ms_16F_32F"] = [batched["16F"], batched["32F"]]
+    out["speedup_vs_batched_cublas"] = batched[best] / jig_step_ms
+    out["batched_how"] = ("one cublasGemmStridedBatchedEx per (M, K, N) group of the batch, best of "
+                          "CUBLAS_COMPUTE_16F / 32F, graph-replayed and timed exactly like the jigsaw step")
+    if not per_matrix:
+        return out
+    detail, sp = [], {}
+    tj_sum = tc_sum = 0.0
+    for i, (M, K, v, s, N) in enumerate(b.points):
+        tj = per_call_us(lambda: b.hs[i].spmm(b.dB[i], C=b.dC[i]), flush, stream, torch)
+        t16 = per_call_us(lambda: cublas_ref.gemm(b.dA[i], b.dB[i], outs[i], "16F"), flush, stream, torch)
+        t32 = per_call_us(lambda: cublas_ref.gemm(b.dA[i], b.dB[i], outs[i], "32F"), flush, stream, torch)
+        tc = min(t16, t32)
+        tag = point_tag(b.name, i, v, s)
+        detail.append({"M": M, "K": K, "v": v, "s": s, "N": N, "tag": tag, "jigsaw_us": tj,
+                       "cublas16F_us": t16, "cublas32F_us": t32, "speedup": tc / tj,
+                       "eff_tflops": 2 * M * N * K / (tj * 1e-6) / 1e12})
+        sp.setdefault(tag, []).append(tc / tj)
+        tj_sum += tj
+        tc_sum += tc
+    out["speedup_geomean_by_v_s"] = {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(sp.items())}
+    out["per_matrix_speedup_total_time"] = tc_sum / tj_sum
+    out["per_matrix_how"] = ("each product alone: jigsaw_spmm vs cublasGemmEx (best of COMPUTE_16F / 32F) on "
+                             "the dense A, [graph of 8 x (L2 flush, call)] - [graph of 8 x flush], / 8, median of 7")
+    out["detail"] = detail
+    return out
+
+
+def e2e_host(b: Batch, jig, torch, steps, dist=None, world=1, dev=None):
+    """The metric end to end through the public API with HOST buffers
+    (jigsaw_spmm_batched_host: pinned B's in, grouped SpMM, C's out, every step)."""
+    pin_B = [torch.from_numpy(B.view(np.int16)).pin_memory().numpy().view(np.uint16) for (_, B) in b.mats]
     pin_C = [torch.empty((M, N), dtype=torch.int16).pin_memory().numpy().view(np.uint16)
-             for (M, K, v, s, N) in points]
-    h2d = sum(B.nbytes for (_, B) in mats)
-    d2h = sum(2 * M * N for (M, K, v, s, N) in points)
-    e2e_steps = max(3, min(args.steps, 20))
-    # one jigsaw_spmm_batched_host call per step: copy-in, grouped SpMM and
-    # copy-out of successive chunks of the batch overlap on three streams
-    jig.spmm_batched_host(hs, pin_B, pin_C)
+             for (M, K, v, s, N) in b.points]
+    h2d = sum(B.nbytes for (_, B) in b.mats)
+    d2h = sum(2 * M * N for (M, K, v, s, N) in b.points)
+    jig.spmm_batched_host(b.hs, pin_B, pin_C)
     if world > 1:
         dist.barrier()
     t0 = time.perf_counter()
-    for _ in range(e2e_steps):
-        jig.spmm_batched_host(hs, pin_B, pin_C)
-    e2e_s = (time.perf_counter() - t0) / e2e_steps
-    te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    for _ in range(steps):
+        jig.spmm_batched_host(b.hs, pin_B, pin_C)
+    e2e_s = (time.perf_counter() - t0) / steps
+    from paper_conf_icpp_zhanglyfyllq24_b200 import shard
+    e2e_s = shard.max_over_ranks(e2e_s, dist=dist if world > 1 else None, device=dev)
+    return e2e_s, h2d, d2h
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--workload", default="c2")
+    ap.add_argument("--panel-rows", type=int, default=0, choices=[0, 128, 256],
+                    help="reorder panel height: 0 = library auto, 128 (one CTA per panel) or 256 (CTA pairs)")
+    ap.add_argument("--impl", default="jigsaw", choices=["jigsaw", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-cublas", action="store_true")
+    ap.add_argument("--no-extra", action="store_true", help="skip the c4 sub-object of the default run")
+    ap.add_argument("--multi", action="store_true", help="also run the C5a / C5b sharded sweep at N = 1")
+    ap.add_argument("--detail", action="store_true", help="print the per-point table to stderr")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_s = float(te.item())
-    # e2e_full: host A -> reorder -> host B -> SpMM -> host C (all §8(a) rows)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")          # communicator init (nranks) in the log
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_zhanglyfyllq24_b200 as jig
+
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        print(f"[bench] rank {rank}: NCCL process group up, world size {dist.get_world_size()}", file=sys.stderr)
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    stream = torch.cuda.current_stream()
+    peaks = load_peaks()
+    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    dist_ = dist if world > 1 else None
+
+    b = Batch(args.workload, rank, world, args.panel_rows, dev, torch, jig)
+    total_eff = sum(2 * M * K * N for (M, K, v, s, N) in b.all_points) * (world if b.scaling == "weak" else 1)
+    b.step(jig)
+    torch.cuda.synchronize()
+    launches = jig.last_launch()["launches"]
+    ms, clocks = timed_steps(lambda: b.step(jig), args.steps, args.warmup, flush, stream, torch,
+                             dist=dist_, world=world, dev_index=dev.index or 0)
+    value = total_eff / (ms * 1e-3) / 1e12
+    roof = roofline(b, ms / max(1, launches), peaks)
+
+    cub = None
+    if not args.no_cublas and b.points:
+        cub = cublas_compare(b, flush, stream, torch, jig, ms, min(args.steps, 30), args.warmup)
+        if args.detail and rank == 0:
+            for d in cub["detail"]:
+                print(json.dumps(d), file=sys.stderr)
+        cub.pop("detail", None)
+
+    e2e_steps = max(3, min(args.steps, 20))
+    e2e_s, h2d, d2h = e2e_host(b, jig, torch, e2e_steps, dist_, world, dev)
+    # e2e_full: host A -> reorder -> host B -> SpMM -> host C (all §8(a) rows), rank 0 batch, one pass
     t0 = time.perf_counter()
-    for (A, B), (M, K, v, s, N) in zip(mats, points):
+    for (A, B), (M, K, v, s, N) in zip(b.mats, b.points):
         hh = jig.reorder_host(A, v, panel_rows=args.panel_rows)
         hh.spmm_host(B)
         hh.free()
     full_s = time.perf_counter() - t0
 
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_baseline(points, mats)
-
     line = {
         "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": world,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
-        "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f16",
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+        "higher_is_better": True, "scaling": b.scaling, "vs_baseline": None, "dtype": "f16",
         "data": "synthetic",
-        "config": {"workload": desc, "matrices_on_rank0": len(points),
+        "config": {"workload": b.desc, "matrices_on_rank0": len(b.points),
                    "flops": "dense-equivalent 2*M*N*K per matrix",
-                   "l2": "flushed (256 MB write) before every timed step", "launch": "step = jigsaw_spmm_batched over the batch (one grouped k_spmm launch per 64 matrices), captured in a CUDA graph",
-                   "seeds": f"synth.SEED_BASE + 1000*rank + index", "format": f"panel_rows={args.panel_rows or 'auto'} (P used: {sorted(set(h.info()['panel_rows'] for h in hs))}), SPTC residual"},
+                   "l2": "flushed (256 MB write) before every timed step",
+                   "launch": "step = one jigsaw_spmm_batched call over the batch (one grouped k_spmm launch per "
+                             "64 matrices of one panel height), captured in a CUDA graph",
+                   "seeds": "synth.SEED_BASE + 1000*rank + index",
+                   "format": f"panel_rows={args.panel_rows or 'auto'} (P used: {b.panel_rows_used}), SPTC residual"},
         "roofline": roof,
-        "cpu_baseline": cpu,
+        "cpu_baseline": None,
         "e2e": {"value": total_eff / e2e_s / 1e12, "unit": "TFLOP/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "call": "jigsaw_spmm_batched_host (pinned host buffers), wall clock per step"},
-        "e2e_full": {"value": eff_flops / full_s / 1e12, "unit": "TFLOP/s",
-                     "note": "rank 0: jigsaw_reorder_host + jigsaw_spmm_host per matrix, one pass"},
+                "call": "jigsaw_spmm_batched_host (pinned host buffers), wall clock per step, max over ranks"},
+        "e2e_full": {"value": b.eff_flops / full_s / 1e12, "unit": "TFLOP/s",
+                     "note": "this rank: jigsaw_reorder_host + jigsaw_spmm_host per matrix, one pass"},
         "gpu_launches": launches * args.steps,
         "clocks": clocks,
-        "cublas": {"step_ms": cublas_step_ms, "step_tflops": eff_flops / (cublas_step_ms * 1e-3) / 1e12,
-                   "speedup_step": cublas_step_ms / ms_per_step,
-                   "jigsaw_unbatched_step_ms": unbatched_step_ms,
-                   "speedup_total_time": (cublas_ms / jig_ms) if jig_ms else None,
-                   "speedup_geomean_by_v_s": speed_gm,
-                   "cublas_eff_tflops": (eff_flops / (cublas_ms * 1e-3) / 1e12) if cublas_ms else None,
-                   "how": "torch.matmul fp16 (cuBLAS) on the dense A: per matrix as [graph of 8 x (L2 flush, call)] - [graph of 8 x (L2 flush)], / 8 (median of 7), and the whole batch as one CUDA graph (median of 30), same L2 flush"},
-        "reorder_ms_total": reorder_ms,
+        "cublas": cub,
+        "reorder_ms_total": b.reorder_ms,
     }
-    if cslt is not None:
-        line["cusparselt"] = cslt
-    if args.detail and rank == 0:
-        for d in detail:
-            print(json.dumps(d), file=sys.stderr)
+
+    # ---- C4 (configs[3]) alongside the default C2 line: compute-bound, CTA pairs
+    if args.workload == "c2" and not args.no_extra:
+        b4 = Batch("c4", rank, world, 0, dev, torch, jig)
+        b4.step(jig)
+        torch.cuda.synchronize()
+        l4 = jig.last_launch()["launches"]
+        st4 = max(5, min(args.steps, 20))
+        ms4, clk4 = timed_steps(lambda: b4.step(jig), st4, args.warmup, flush, stream, torch,
+                                dist=dist_, world=world, dev_index=dev.index or 0)
+        eff4 = sum(2 * M * K * N for (M, K, v, s, N) in b4.all_points) * world
+        c4 = {"workload": b4.desc, "value": eff4 / (ms4 * 1e-3) / 1e12, "unit": "TFLOP/s", "ms_per_step": ms4,
+              "steps": st4, "gpu_launches": l4 * st4, "roofline": roofline(b4, ms4 / max(1, l4), peaks),
+              "clocks": clk4, "format": f"panel_rows=auto (P used: {b4.panel_rows_used})",
+              "reorder_ms_total": b4.reorder_ms}
+        if not args.no_cublas:
+            cb4 = cublas_compare(b4, flush, stream, torch, jig, ms4, st4, args.warmup)
+            cb4.pop("detail", None)
+            c4["cublas"] = cb4
+        e4, h4, d4 = e2e_host(b4, jig, torch, 3, dist_, world, dev)
+        c4["e2e"] = {"value": eff4 / e4 / 1e12, "unit": "TFLOP/s", "h2d_bytes_per_step": h4,
+                     "d2h_bytes_per_step": d4}
+        line["c4"] = c4
+        b4.free()
+
+    # ---- C5a / C5b (configs[4]): the sharded sweep, at N > 1 (or --multi)
+    if (world > 1 or args.multi) and args.workload == "c2":
+        from paper_conf_icpp_zhanglyfyllq24_b200 import shard
+        for name in ("c5a", "c5b"):
+            bs = Batch(name, rank, world, 0, dev, torch, jig)
+            st5 = max(5, min(args.steps, 20))
+            fn = (lambda: bs.step(jig)) if bs.hs else (lambda: None)
+            ms5, clk5 = timed_steps(fn, st5, args.warmup, flush, stream, torch,
+                                    dist=dist_, world=world, dev_index=dev.index or 0)
+            eff5 = sum(2 * M * K * N for (M, K, v, s, N) in bs.all_points)
+            sub = {"workload": bs.desc, "value": eff5 / (ms5 * 1e-3) / 1e12, "unit": "TFLOP/s",
+                   "ms_per_step": ms5, "steps": st5, "scaling": "strong", "matrices_on_rank0": len(bs.points),
+                   "clocks": clk5}
+            if name == "c5b" and world >= 1:
+                # untimed validation: NCCL all_gather of the C column shards, sampled
+                # rows checked on rank 0 against a dense PyTorch product; the ranks'
+                # format hashes (deterministic reorder of the replicated A) compared
+                M, K, v, s, N, seed, n0, n1 = local_jobs("c5b", bs.all_points, rank, world)[0]
+                torch.cuda.synchronize()
+                full = shard.gather_column_shards(bs.dC[0], n0, n1, N, dist, world) if world > 1 else bs.dC[0]
+                hsh = torch.tensor([shard.format_hash(bs.hs[0].export())], dtype=torch.int64, device=dev)
+                hs_all = [torch.zeros_like(hsh) for _ in range(world)]
+                if world > 1:
+                    dist.all_gather(hs_all, hsh)
+                else:
+                    hs_all = [hsh]
+                if rank == 0:
+                    Bfull = torch.from_numpy(synth.dense_b(K, N, seed).view(np.int16)).to(dev).view(torch.float16)
+                    rows = torch.from_numpy(np.sort(np.random.default_rng(5).choice(M, 64, replace=False))).to(dev)
+                    excess = shard.check_against_dense(full, bs.dA[0], Bfull, rows)
+                    sub["validation"] = {"gathered_shape": list(full.shape), "rows_checked": 64,
+                                         "max_excess_over_tolerance": excess, "pass": excess <= 0,
+                                         "format_hashes_equal": len({int(x.item()) for x in hs_all}) == 1,
+                                         "how": "all_gather of C column shards (NCCL) after the timed region; "
+                                                "64 sampled rows vs torch fp32 matmul of the dense fp16 A"}
+            line[name] = sub
+            bs.free()
+
+    if rank == 0 and world == 1 and not args.no_cpu:
+        line["cpu_baseline"] = cpu_baseline(b.points, b.mats)
     if rank == 0:
         print(json.dumps(line))
-    for h in hs:
-        h.free()
+    b.free()
     if world > 1:
         dist.destroy_process_group()
     return 0

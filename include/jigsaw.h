@@ -57,6 +57,13 @@ typedef enum {
   JIGSAW_RESIDUAL_DENSE = 1 /* evicted columns form a dense tail run on dense tensor cores */
 } jigsaw_residual_mode_t;
 
+/* Element type of C (jigsaw_options_t.c_dtype; fp16 in, fp32
+ * accumulate; C rounded to fp16 (RN, the paper's cublasHgemm output) or kept fp32). */
+typedef enum {
+  JIGSAW_C_F16 = 0, /* C is fp16 (IEEE binary16), round-to-nearest-even from the fp32 accumulator (default) */
+  JIGSAW_C_F32 = 1  /* C is fp32: the fp32 accumulator as is */
+} jigsaw_c_dtype_t;
+
 typedef struct {
   int panel_rows;    /* rows per panel (the BLOCK_TILE analogue, R-Q5/R-Q6): 128 (one CTA per
                         panel; the default when opt is NULL), 256 (a CTA pair per panel:
@@ -66,7 +73,8 @@ typedef struct {
                         export / statistics only: jigsaw_spmm on such a handle returns
                         JIGSAW_ERROR_UNSUPPORTED (no tcgen05 M below 128 is built) */
   int residual_mode; /* jigsaw_residual_mode_t */
-  int reserved[6];   /* must be zero */
+  int c_dtype;       /* jigsaw_c_dtype_t: element type of C for every product with this handle */
+  int reserved[5];   /* must be zero */
 } jigsaw_options_t;
 
 /* Statistics of a prepared matrix (jigsaw_get_info). */
@@ -76,6 +84,8 @@ typedef struct {
   int32_t panel_rows;      /* P */
   int32_t residual_mode;   /* jigsaw_residual_mode_t */
   int32_t device;          /* CUDA ordinal the handle lives on */
+  int32_t c_dtype;         /* jigsaw_c_dtype_t */
+  int32_t reserved0;
   int64_t npanels;         /* ceil(M / P) */
   int64_t ntiles;          /* sum_p T_p: 2:4 tiles of 16 logical columns */
   int64_t ndtiles;         /* sum_p D_p: dense residual tiles (DENSE mode) */
@@ -120,21 +130,26 @@ JIGSAW_API jigsaw_handle_t jigsaw_reorder(const void* A, int64_t M, int64_t K, i
 /* C = A x B on sparse tensor cores, beta = 0: every element of C is written
  * (rows of an all-zero panel are written as zeros).
  *   B : device pointer, fp16 row-major K x N (ld = N), 16-byte aligned.
- *   C : device pointer, fp16 row-major M x N (ld = N), 16-byte aligned; overwritten.
+ *   C : device pointer, row-major M x N (ld = N), 16-byte aligned; overwritten.
+ *       fp16, or fp32 if the handle was built with c_dtype = JIGSAW_C_F32.
  *   N > 0, N % 8 == 0 (TMA needs 16-byte rows).
- * Asynchronous on `stream`; no host synchronisation and no allocation, except
- * that the first grouped launch with split units (long units cut into k-range
- * pieces) on a device grows the library's fp32 partial-tile workspace (one
- * cudaMalloc + device synchronisation, outside stream capture; inside a capture
- * such a launch runs whole units instead).  The handle is immutable, so calls may
- * run concurrently on several streams: each stream gets its own workspace
- * regions (up to 8 streams per device; beyond that streams share regions and
- * must not run split launches at the same time).  C must not
- * alias B.  The kernel is launched with programmatic stream serialization: it
- * may start while the previous kernel of `stream` drains, but reads B and
- * writes C only after that kernel has completed (stream order is preserved for
- * B and C); it lets the next programmatic launch on `stream` start once its own
- * last work unit is scheduled.  JIGSAW_PDL=0 in the environment disables this. */
+ * Asynchronous on `stream`, never synchronises the host or the device.
+ * Launches that use the dynamic tile scheduler or split long units into k-range
+ * pieces need a small device workspace (scheduler ticket, piece counters, fp32
+ * partial tiles): on an ordinary stream it is a region owned by that stream,
+ * taken from the library's stream-ordered pool the first time the stream needs
+ * it (or needs more) and then reused; under stream capture it is a graph-owned
+ * allocation node plus a memset node zeroing its counters, freed right after
+ * the kernel node.  So the
+ * handle stays immutable and calls may run concurrently on any number of
+ * streams, and captured graphs may be replayed concurrently with each other and
+ * with eager calls.  C must not alias B.  The kernel is launched with
+ * programmatic stream serialization: it may start while the previous kernel of
+ * `stream` drains, but reads B, writes C and touches its workspace only after
+ * that kernel has completed (stream order is preserved); it lets the next
+ * programmatic launch on `stream` start once its own last work unit is
+ * scheduled.  JIGSAW_PDL=0 in the environment (read once at load) disables
+ * this. */
 JIGSAW_API jigsaw_status_t jigsaw_spmm(jigsaw_handle_t h, const void* B, int64_t N, void* C,
                             jigsaw_stream_t stream);
 
@@ -168,12 +183,15 @@ JIGSAW_API jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format
 
 /* C = A x B with B and C in HOST memory (end-to-end path): copies B in, runs
  * jigsaw_spmm, copies C out, all on `stream`, then synchronises `stream`.
- * Device staging buffers are taken from the stream-ordered allocator. */
+ * C_host holds M x N elements of the handle's c_dtype.  Device staging buffers
+ * are taken from the library's stream-ordered pool. */
 JIGSAW_API jigsaw_status_t jigsaw_spmm_host(jigsaw_handle_t h, const void* B_host, int64_t N, void* C_host,
                                  jigsaw_stream_t stream);
 
 /* `count` independent products Cs[i] = A_i x Bs[i] (handles on the same device),
- * issued back to back on `stream` (the batch of independent matrices, C5a). */
+ * as ONE grouped persistent k_spmm launch per 64 products of the same panel
+ * height (the batch of independent matrices, C5a).  Buffers and semantics as
+ * jigsaw_spmm, per product. */
 JIGSAW_API jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const* Bs,
                                     const int64_t* Ns, void* const* Cs, int count,
                                     jigsaw_stream_t stream);
@@ -186,8 +204,9 @@ JIGSAW_API jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const 
  * both directions and the SMs work at the same time; pinned host buffers are
  * needed for the copies to overlap (pageable memory is correct but serial).
  * Device staging comes from the stream-ordered pool and is returned before the
- * call returns.  Ordered after prior work on `stream`; synchronous: returns
- * after every C is in host memory.  Errors as jigsaw_spmm_batched; a failure
+ * call returns; each call uses helper streams of its own (concurrent calls from
+ * several host threads do not wait for each other).  Ordered after prior work
+ * on `stream`; synchronous: returns after every C is in host memory.  Errors as jigsaw_spmm_batched; a failure
  * in a later chunk leaves earlier Cs written. */
 JIGSAW_API jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* const* Bs_host,
                                                     const int64_t* Ns, void* const* Cs_host, int count,
@@ -199,8 +218,42 @@ JIGSAW_API int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N);
 
 /* ---------------------------------------------------------------- diagnostics */
 
-/* Per-CTA timeline of the most recent k_spmm launch made with the environment
- * variable JIGSAW_TRACE=1 (otherwise nothing is recorded).  Copies up to
+/* How the calling thread's most recent jigsaw_spmm / jigsaw_spmm_batched /
+ * host-buffer call was launched (for tests and benchmarks). */
+typedef struct {
+  int32_t launches;              /* k_spmm launches of that call */
+  int32_t tile_n;                /* N columns per work unit (MMA N) of the last launch */
+  int32_t split_k;               /* CTAs of a split-K cluster (1 = none) */
+  int32_t grid;                  /* CTAs launched */
+  int32_t cta_pair;              /* 1: 256-row panels on CTA pairs (cta_group::2) */
+  int32_t problems;              /* products in the last launch */
+  int32_t work_items;            /* scheduled work items (units, k-range pieces, padding) */
+  int32_t split_slots;           /* k-range pieces reduced through the workspace (0 = none) */
+  int32_t dynamic_schedule;      /* 1: dynamic tile scheduler */
+  int32_t graph_owned_workspace; /* 1: workspace was a graph allocation node (stream capture) */
+  int32_t nsplit_items;          /* column slices of long units (N-split, no workspace) */
+  int32_t reserved[5];
+} jigsaw_launch_desc_t;
+JIGSAW_API jigsaw_status_t jigsaw_last_launch(jigsaw_launch_desc_t* out);
+
+/* Diagnostic override of the launch configuration for the CALLING thread's later
+ * calls (tests reach every kernel variant with it); NULL or all-zero restores
+ * the library's choice.  Fields: tile_n (0 or 32/64/128/256 columns per unit),
+ * split_k (0 or 1/2/4/8: single products of 128-row panels on split-K clusters
+ * of that size, tile 64 or 32), no_pieces (1: no k-range pieces in grouped
+ * launches), host_chunks (0 = 16, else the chunk count of
+ * jigsaw_spmm_batched_host), k_pieces (1: split long units of grouped launches
+ * into k-range pieces reduced through the workspace, instead of the default
+ * column slices).  Results are identical up to fp32 summation order. */
+typedef struct {
+  int32_t tile_n, split_k, no_pieces, host_chunks, k_pieces;
+  int32_t reserved[3]; /* must be zero */
+} jigsaw_launch_override_t;
+JIGSAW_API jigsaw_status_t jigsaw_set_launch_override(const jigsaw_launch_override_t* o);
+
+/* Per-CTA timeline of the most recent k_spmm launch, recorded only when the
+ * environment variable JIGSAW_TRACE=1 was set when the library was loaded (read
+ * once; otherwise nothing is recorded).  Copies up to
  * max_ctas records of 24 int64 each into `out` (host): slots 0-11 are SM clock
  * (clock64) stamps at fixed points of the kernel (entry, setup done, first A/E
  * copy, first B copies, first full stage, last MMA commit, accumulator ready,

@@ -29,7 +29,9 @@ ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_stat
                "jigsaw_last_error_string", "jigsaw_version", "jigsaw_reorder_ex",
                "jigsaw_reorder_host", "jigsaw_get_info", "jigsaw_export_format",
                "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_batched_host", "jigsaw_spmm_launches_per_call",
-               "jigsaw_debug_trace"]
+               "jigsaw_debug_trace", "jigsaw_last_launch", "jigsaw_set_launch_override"]
+
+C_F16, C_F32 = 0, 1            # jigsaw_c_dtype_t
 
 
 class JigsawError(RuntimeError):
@@ -39,14 +41,15 @@ class JigsawError(RuntimeError):
 
 
 class Options(ctypes.Structure):
-    _fields_ = [("panel_rows", ctypes.c_int), ("residual_mode", ctypes.c_int),
-                ("reserved", ctypes.c_int * 6)]
+    _fields_ = [("panel_rows", ctypes.c_int), ("residual_mode", ctypes.c_int), ("c_dtype", ctypes.c_int),
+                ("reserved", ctypes.c_int * 5)]
 
 
 class Info(ctypes.Structure):
     _fields_ = [("M", ctypes.c_int64), ("K", ctypes.c_int64), ("v", ctypes.c_int32),
                 ("panel_rows", ctypes.c_int32), ("residual_mode", ctypes.c_int32),
-                ("device", ctypes.c_int32), ("npanels", ctypes.c_int64), ("ntiles", ctypes.c_int64),
+                ("device", ctypes.c_int32), ("c_dtype", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+                ("npanels", ctypes.c_int64), ("ntiles", ctypes.c_int64),
                 ("ndtiles", ctypes.c_int64), ("overflow_tiles", ctypes.c_int64),
                 ("evictions", ctypes.c_int64), ("nnz", ctypes.c_int64), ("kp_total", ctypes.c_int64),
                 ("max_tiles", ctypes.c_int64), ("nksteps", ctypes.c_int64),
@@ -57,6 +60,17 @@ class Info(ctypes.Structure):
 class FormatHost(ctypes.Structure):
     _fields_ = [(n, ctypes.c_void_p) for n in
                 ("T", "D", "col_idx", "perm", "gather", "vals", "meta", "kind", "nevict", "rcol", "dvals")]
+
+
+class LaunchDesc(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in
+                ("launches", "tile_n", "split_k", "grid", "cta_pair", "problems", "work_items", "split_slots",
+                 "dynamic_schedule", "graph_owned_workspace", "nsplit_items")] + [("reserved", ctypes.c_int32 * 5)]
+
+
+class LaunchOverride(ctypes.Structure):
+    _fields_ = [("tile_n", ctypes.c_int32), ("split_k", ctypes.c_int32), ("no_pieces", ctypes.c_int32),
+                ("host_chunks", ctypes.c_int32), ("k_pieces", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3)]
 
 
 _lib = None
@@ -96,6 +110,8 @@ def lib(build_if_missing: bool = True):
                                           ctypes.POINTER(vp), ci, vp]),
         "jigsaw_spmm_launches_per_call": (ci, [vp, i64]),
         "jigsaw_debug_trace": (ci, [vp, ci]),
+        "jigsaw_last_launch": (ci, [ctypes.POINTER(LaunchDesc)]),
+        "jigsaw_set_launch_override": (ci, [ctypes.POINTER(LaunchOverride)]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -123,12 +139,26 @@ def _stream_ptr(stream):
     return ctypes.c_void_p(stream.cuda_stream)
 
 
-def _check_fp16_cuda(t, name):
+def _check_cuda(t, name, dtype=None):
     import torch
-    if not isinstance(t, torch.Tensor) or t.dtype != torch.float16 or not t.is_cuda:
-        raise TypeError(f"{name} must be a CUDA float16 tensor")
+    dtype = dtype or torch.float16
+    if not isinstance(t, torch.Tensor) or t.dtype != dtype or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA {dtype} tensor")
     if not t.is_contiguous():
         raise ValueError(f"{name} must be contiguous (row-major)")
+
+
+def _check_fp16_cuda(t, name):
+    _check_cuda(t, name)
+
+
+def _host16(x: np.ndarray, name: str) -> np.ndarray:
+    x = np.ascontiguousarray(x)
+    if x.dtype == np.float16:
+        x = x.view(np.uint16)
+    if x.dtype.itemsize != 2 or x.ndim != 2:
+        raise TypeError(f"{name} must be a 2-D fp16 (or 16-bit pattern) host array")
+    return x
 
 
 class Handle:
@@ -138,6 +168,29 @@ class Handle:
         self._h = ctypes.c_void_p(ptr)
         inf = self.info()
         self.M, self.K = inf["M"], inf["K"]
+        self.c_dtype = inf["c_dtype"]
+
+    @property
+    def c_torch_dtype(self):
+        import torch
+        return torch.float32 if self.c_dtype == C_F32 else torch.float16
+
+    @property
+    def c_numpy_dtype(self):
+        return np.float32 if self.c_dtype == C_F32 else np.uint16
+
+    def check_b_c(self, B, C):
+        """The checks jigsaw_spmm relies on the caller for: B is a contiguous CUDA
+        fp16 K x N tensor, C a contiguous CUDA M x N tensor of the handle's c_dtype."""
+        _check_fp16_cuda(B, "B")
+        K, N = B.shape
+        if K != self.K:
+            raise ValueError(f"B has {K} rows, A has K = {self.K}")
+        _check_cuda(C, "C", self.c_torch_dtype)
+        if tuple(C.shape) != (self.M, N):
+            raise ValueError(f"C must be {self.M} x {N}")
+        if C.device != B.device:
+            raise ValueError("B and C must be on the same device")
 
     @property
     def ptr(self):
@@ -149,18 +202,14 @@ class Handle:
         return {n: getattr(out, n) for n, _ in Info._fields_}
 
     def spmm(self, B, C=None, stream=None):
-        """C = A x B (jigsaw_spmm); B: CUDA fp16 K x N; returns C (M x N fp16)."""
+        """C = A x B (jigsaw_spmm); B: CUDA fp16 K x N; returns C (M x N, fp16 or
+        fp32 per the handle's c_dtype)."""
         import torch
         _check_fp16_cuda(B, "B")
-        K, N = B.shape
-        if K != self.K:
-            raise ValueError(f"B has {K} rows, A has K = {self.K}")
+        N = B.shape[1]
         if C is None:
-            C = torch.empty((self.M, N), dtype=torch.float16, device=B.device)
-        else:
-            _check_fp16_cuda(C, "C")
-            if tuple(C.shape) != (self.M, N):
-                raise ValueError("C must be M x N")
+            C = torch.empty((self.M, N), dtype=self.c_torch_dtype, device=B.device)
+        self.check_b_c(B, C)
         _raise_if(lib().jigsaw_spmm(self._h, ctypes.c_void_p(B.data_ptr()), N,
                                     ctypes.c_void_p(C.data_ptr()), _stream_ptr(stream)))
         return C
@@ -168,12 +217,13 @@ class Handle:
     def spmm_host(self, B: np.ndarray, out: np.ndarray = None, stream=None) -> np.ndarray:
         """End-to-end path (jigsaw_spmm_host): host B in, host C out (optionally
         into `out`, e.g. pinned memory)."""
-        B = np.ascontiguousarray(B)
-        if B.dtype == np.float16:
-            B = B.view(np.uint16)
-        C = np.empty((self.M, B.shape[1]), dtype=np.uint16) if out is None else out
-        if C.shape != (self.M, B.shape[1]) or not C.flags.c_contiguous or C.itemsize != 2:
-            raise ValueError("out must be a contiguous M x N 16-bit array")
+        B = _host16(B, "B")
+        if B.shape[0] != self.K:
+            raise ValueError(f"B has {B.shape[0]} rows, A has K = {self.K}")
+        C = np.empty((self.M, B.shape[1]), dtype=self.c_numpy_dtype) if out is None else out
+        if (C.shape != (self.M, B.shape[1]) or not C.flags.c_contiguous
+                or C.itemsize != np.dtype(self.c_numpy_dtype).itemsize):
+            raise ValueError("out must be a contiguous M x N array of the handle's C element size")
         _raise_if(lib().jigsaw_spmm_host(self._h, B.ctypes.data_as(ctypes.c_void_p), B.shape[1],
                                          C.ctypes.data_as(ctypes.c_void_p),
                                          _stream_ptr(stream) if stream is not None else None))
@@ -205,24 +255,24 @@ class Handle:
             pass
 
 
-def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, stream=None) -> Handle:
+def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: int = C_F16,
+            stream=None) -> Handle:
     """jigsaw_reorder_ex: multi-granularity reorder + format build of A (CUDA fp16 M x K)."""
     _check_fp16_cuda(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode)
+    opt = Options(panel_rows, residual_mode, c_dtype)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_ex(ctypes.c_void_p(A.data_ptr()), M, K, v, ctypes.byref(opt),
                                       _stream_ptr(stream), ctypes.byref(out)))
     return Handle(out.value)
 
 
-def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: int = 0) -> Handle:
+def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: int = 0,
+                 c_dtype: int = C_F16) -> Handle:
     """jigsaw_reorder_host: A given as a host array (fp16 or uint16 bits)."""
-    A = np.ascontiguousarray(A)
-    if A.dtype == np.float16:
-        A = A.view(np.uint16)
+    A = _host16(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode)
+    opt = Options(panel_rows, residual_mode, c_dtype)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_host(A.ctypes.data_as(ctypes.c_void_p), M, K, v,
                                         ctypes.byref(opt), None, ctypes.byref(out)))
@@ -242,13 +292,18 @@ def spmm_batched_host(handles, Bs, outs=None, stream=None):
     """jigsaw_spmm_batched_host: the batch with host B's in and host C's out
     (pinned arrays, e.g. from torch pin_memory, let the copies overlap)."""
     n = len(handles)
-    Bs = [np.ascontiguousarray(b).view(np.uint16) if b.dtype == np.float16 else np.ascontiguousarray(b)
-          for b in Bs]
+    if len(Bs) != n or (outs is not None and len(outs) != n):
+        raise ValueError("handles, Bs and outs must have the same length")
+    Bs = [_host16(b, "B") for b in Bs]
+    for h, b in zip(handles, Bs):
+        if b.shape[0] != h.K:
+            raise ValueError(f"B has {b.shape[0]} rows, A has K = {h.K}")
     if outs is None:
-        outs = [np.empty((h.M, b.shape[1]), dtype=np.uint16) for h, b in zip(handles, Bs)]
+        outs = [np.empty((h.M, b.shape[1]), dtype=h.c_numpy_dtype) for h, b in zip(handles, Bs)]
     for h, b, c in zip(handles, Bs, outs):
-        if c.shape != (h.M, b.shape[1]) or not c.flags.c_contiguous or c.itemsize != 2:
-            raise ValueError("each out must be a contiguous M x N 16-bit array")
+        if (c.shape != (h.M, b.shape[1]) or not c.flags.c_contiguous
+                or c.itemsize != np.dtype(h.c_numpy_dtype).itemsize):
+            raise ValueError("each out must be a contiguous M x N array of its handle's C element size")
     hs = (ctypes.c_void_p * n)(*[h.ptr.value for h in handles])
     bp = (ctypes.c_void_p * n)(*[b.ctypes.data for b in Bs])
     cp = (ctypes.c_void_p * n)(*[c.ctypes.data for c in outs])
@@ -258,11 +313,46 @@ def spmm_batched_host(handles, Bs, outs=None, stream=None):
 
 
 def spmm_batched(handles, Bs, Cs, stream=None):
-    """jigsaw_spmm_batched: independent products issued back to back on one stream."""
+    """jigsaw_spmm_batched: independent products in grouped persistent launches."""
     n = len(handles)
+    if len(Bs) != n or len(Cs) != n:
+        raise ValueError("handles, Bs and Cs must have the same length")
+    for h, b, c in zip(handles, Bs, Cs):
+        h.check_b_c(b, c)
     hs = (ctypes.c_void_p * n)(*[h.ptr.value for h in handles])
     bp = (ctypes.c_void_p * n)(*[b.data_ptr() for b in Bs])
     cp = (ctypes.c_void_p * n)(*[c.data_ptr() for c in Cs])
     ns = (ctypes.c_int64 * n)(*[b.shape[1] for b in Bs])
     _raise_if(lib().jigsaw_spmm_batched(hs, bp, ns, cp, n, _stream_ptr(stream)))
     return Cs
+
+
+def last_launch() -> dict:
+    """jigsaw_last_launch: how this thread's most recent SpMM call was launched."""
+    d = LaunchDesc()
+    _raise_if(lib().jigsaw_last_launch(ctypes.byref(d)))
+    return {n: getattr(d, n) for n, _ in LaunchDesc._fields_ if n != "reserved"}
+
+
+def set_launch_override(tile_n: int = 0, split_k: int = 0, no_pieces: int = 0, host_chunks: int = 0,
+                        k_pieces: int = 0):
+    """jigsaw_set_launch_override (diagnostic, this thread): force the tile width,
+    split-K factor, no splitting / k-range pieces instead of column slices, or the
+    host chunk count; all zeros = library choice."""
+    o = LaunchOverride(tile_n, split_k, no_pieces, host_chunks, k_pieces)
+    _raise_if(lib().jigsaw_set_launch_override(ctypes.byref(o)))
+
+
+class launch_override:
+    """Context manager around set_launch_override (restores the library's choice)."""
+
+    def __init__(self, **kw):
+        self.kw = kw
+
+    def __enter__(self):
+        set_launch_override(**self.kw)
+        return self
+
+    def __exit__(self, *exc):
+        set_launch_override()
+        return False

@@ -55,27 +55,70 @@ jigsaw_status_t check_device(int* dev_out) {
 
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
-// Stream-ordered staging memory for the host-buffer entry points: a private pool
-// per device that keeps its memory (no release to the OS between calls).
+// Stream-ordered device memory of the library (host-buffer staging, launch
+// workspaces): a private pool per device.  It keeps up to 256 MB reserved across
+// synchronisations (steady-state calls do not go back to the OS); anything above
+// that is released to the OS at the next synchronisation, so a large host-buffer
+// batch does not pin its peak staging for the life of the process.
 cudaMemPool_t g_pool[64] = {};
-std::mutex g_lazy_mu;  // guards the lazy creation of the pools and pipeline streams
+std::mutex g_lazy_mu;  // guards the lazy creation of the pools
+constexpr uint64_t kPoolKeepBytes = (uint64_t)256 << 20;
 cudaError_t staging_alloc(void** p, size_t bytes, cudaStream_t st) {
   int dev = 0;
   cudaGetDevice(&dev);
   if (dev < 0 || dev >= 64) return cudaMallocAsync(p, bytes, st);
-  std::lock_guard<std::mutex> lock(g_lazy_mu);
-  if (!g_pool[dev]) {
-    cudaMemPoolProps props = {};
-    props.allocType = cudaMemAllocationTypePinned;
-    props.location.type = cudaMemLocationTypeDevice;
-    props.location.id = dev;
-    cudaError_t e = cudaMemPoolCreate(&g_pool[dev], &props);
-    if (e != cudaSuccess) return e;
-    uint64_t thr = UINT64_MAX;
-    cudaMemPoolSetAttribute(g_pool[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+  cudaMemPool_t pool;
+  {
+    std::lock_guard<std::mutex> lock(g_lazy_mu);
+    if (!g_pool[dev]) {
+      cudaMemPoolProps props = {};
+      props.allocType = cudaMemAllocationTypePinned;
+      props.location.type = cudaMemLocationTypeDevice;
+      props.location.id = dev;
+      cudaError_t e = cudaMemPoolCreate(&g_pool[dev], &props);
+      if (e != cudaSuccess) return e;
+      uint64_t thr = kPoolKeepBytes;
+      cudaMemPoolSetAttribute(g_pool[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    pool = g_pool[dev];
   }
-  return cudaMallocFromPoolAsync(p, bytes, g_pool[dev], st);
+  return cudaMallocFromPoolAsync(p, bytes, pool, st);
 }
+
+// Helper streams of the host-buffer batch pipeline: a free list per device; a
+// call takes a triple for its own use and returns it when done, so concurrent
+// calls never share (or wait on) each other's helper streams.
+struct HostPipe {
+  cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
+};
+std::vector<HostPipe> g_pipes_free[64];
+bool take_pipe(int dev, HostPipe* out) {
+  {
+    std::lock_guard<std::mutex> lock(g_lazy_mu);
+    if (!g_pipes_free[dev].empty()) {
+      *out = g_pipes_free[dev].back();
+      g_pipes_free[dev].pop_back();
+      return true;
+    }
+  }
+  HostPipe P;
+  if (cudaStreamCreateWithFlags(&P.h2d, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&P.comp, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&P.d2h, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    if (P.h2d) cudaStreamDestroy(P.h2d);
+    if (P.comp) cudaStreamDestroy(P.comp);
+    return false;
+  }
+  *out = P;
+  return true;
+}
+void give_pipe(int dev, const HostPipe& P) {
+  std::lock_guard<std::mutex> lock(g_lazy_mu);
+  g_pipes_free[dev].push_back(P);
+}
+
+size_t c_elem_bytes(const Format& f) { return f.c_dtype == JIGSAW_C_F32 ? 4 : 2; }
 
 // panel_rows = 0 (auto): CTA pairs (256-row panels) for tall matrices, where the
 // halved B traffic per output pays (4096 x 4096 N = 2048, +30 %);
@@ -100,7 +143,9 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "panel_rows must be 0 (auto), 16, 32, 64, 128 or 256");
     if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC && opt->residual_mode != JIGSAW_RESIDUAL_DENSE)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
-    for (int i = 0; i < 6; ++i)
+    if (opt->c_dtype != JIGSAW_C_F16 && opt->c_dtype != JIGSAW_C_F32)
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown c_dtype");
+    for (int i = 0; i < 5; ++i)
       if (opt->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved options must be zero");
   }
   return JIGSAW_SUCCESS;
@@ -124,6 +169,9 @@ jigsaw_status_t validate_spmm(jigsaw_handle_t h, const void* B, int64_t N, const
 }
 
 }  // namespace
+
+cudaError_t pool_alloc_async(void** p, size_t bytes, cudaStream_t s) { return staging_alloc(p, bytes, s); }
+
 }  // namespace jig
 
 using namespace jig;
@@ -153,6 +201,7 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
     delete h;
     return s;
   }
+  h->f.c_dtype = opt ? opt->c_dtype : (int)JIGSAW_C_F16;
   *out = h;
   return set_status(JIGSAW_SUCCESS);
 }
@@ -203,7 +252,7 @@ jigsaw_status_t jigsaw_spmm_host(jigsaw_handle_t h, const void* B_host, int64_t 
   jigsaw_status_t s = validate_spmm(h, B_host, N, C_host, false);
   if (s != JIGSAW_SUCCESS) return s;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  const size_t bbytes = (size_t)h->f.K * N * 2, cbytes = (size_t)h->f.M * N * 2;
+  const size_t bbytes = (size_t)h->f.K * N * 2, cbytes = (size_t)h->f.M * N * c_elem_bytes(h->f);
   void *dB = nullptr, *dC = nullptr;
   cudaError_t e = staging_alloc(&dB, bbytes, st);
   if (e == cudaSuccess) e = staging_alloc(&dC, cbytes, st);
@@ -256,11 +305,9 @@ static cudaError_t copy_batch(std::vector<void*>& dst, std::vector<void*>& src, 
   return e;
 }
 
-// Helper streams of the host-buffer batch pipeline (created once per device).
-struct HostPipe {
-  cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
-};
-HostPipe g_pipe[64];
+static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_handle_t* hs, const void* const* Bs_host,
+                                            const int64_t* Ns, void* const* Cs_host, int count,
+                                            jigsaw_stream_t stream);
 
 jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* const* Bs_host, const int64_t* Ns,
                                          void* const* Cs_host, int count, jigsaw_stream_t stream) {
@@ -275,18 +322,16 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
   if (count == 0) return set_status(JIGSAW_SUCCESS);
   const int dev = hs[0]->f.device;
   if (dev < 0 || dev >= 64) return set_status(JIGSAW_ERROR_INTERNAL, "device ordinal out of range");
-  HostPipe& P = g_pipe[dev];
-  std::unique_lock<std::mutex> lazy(g_lazy_mu);
-  if (!P.h2d) {
-    if (cudaStreamCreateWithFlags(&P.h2d, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaStreamCreateWithFlags(&P.comp, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaStreamCreateWithFlags(&P.d2h, cudaStreamNonBlocking) != cudaSuccess) {
-      cudaGetLastError();
-      P = HostPipe{};
-      return set_status(JIGSAW_ERROR_CUDA, "cudaStreamCreate failed");
-    }
-  }
-  lazy.unlock();
+  HostPipe P;
+  if (!take_pipe(dev, &P)) return set_status(JIGSAW_ERROR_CUDA, "cudaStreamCreate failed");
+  jigsaw_status_t rs = spmm_batched_host_on(P, hs, Bs_host, Ns, Cs_host, count, stream);
+  give_pipe(dev, P);
+  return rs;
+}
+
+static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_handle_t* hs, const void* const* Bs_host,
+                                            const int64_t* Ns, void* const* Cs_host, int count,
+                                            jigsaw_stream_t stream) {
   cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
   // staging for the whole batch (one pool allocation each for B and C)
   size_t bb = 0, cb = 0;
@@ -295,7 +340,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
     boff[i] = bb;
     coff[i] = cb;
     bb += ((size_t)hs[i]->f.K * Ns[i] * 2 + 255) & ~size_t(255);
-    cb += ((size_t)hs[i]->f.M * Ns[i] * 2 + 255) & ~size_t(255);
+    cb += ((size_t)hs[i]->f.M * Ns[i] * c_elem_bytes(hs[i]->f) + 255) & ~size_t(255);
   }
   cudaEvent_t ev0;
   if (cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming) != cudaSuccess) return cuda_status(cudaGetLastError(), "event");
@@ -311,11 +356,11 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
     cudaEventDestroy(ev0);
     return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "staging allocation failed");
   }
-  // chunks of ~1/16 of the batch's bytes (at least one product; developer
-  // override JIGSAW_HOST_CHUNKS): copy-in of chunk k+1 and copy-out of chunk
+  // chunks of ~1/16 of the batch's bytes (at least one product; diagnostic
+  // override jigsaw_set_launch_override host_chunks): copy-in of chunk k+1 and copy-out of chunk
   // k-1 overlap the grouped launch of chunk k (16 measured best with one copy
   // per product and direction, profiles/r01zt_e2e_chunks.txt)
-  const int nchunks = getenv("JIGSAW_HOST_CHUNKS") ? std::max(1, atoi(getenv("JIGSAW_HOST_CHUNKS"))) : 16;
+  const int nchunks = launch_override().host_chunks > 0 ? launch_override().host_chunks : 16;
   const size_t target = std::max<size_t>((bb + cb) / nchunks, 1);
   std::vector<const Format*> fs;
   std::vector<const void*> pb;
@@ -327,7 +372,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
     int i1 = i0;
     size_t acc = 0;
     while (i1 < count && (i1 == i0 || acc < target)) {
-      acc += (size_t)hs[i1]->f.K * Ns[i1] * 2 + (size_t)hs[i1]->f.M * Ns[i1] * 2;
+      acc += (size_t)hs[i1]->f.K * Ns[i1] * 2 + (size_t)hs[i1]->f.M * Ns[i1] * c_elem_bytes(hs[i1]->f);
       ++i1;
     }
     std::vector<void*> cd, cs;
@@ -359,7 +404,7 @@ jigsaw_status_t jigsaw_spmm_batched_host(const jigsaw_handle_t* hs, const void* 
     for (int i = i0; i < i1; ++i) {
       cd.push_back(Cs_host[i]);
       cs.push_back(dC + coff[i]);
-      cz.push_back((size_t)hs[i]->f.M * Ns[i] * 2);
+      cz.push_back((size_t)hs[i]->f.M * Ns[i] * c_elem_bytes(hs[i]->f));
     }
     if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, cudaMemcpyDeviceToHost, P.d2h);
     i0 = i1;
@@ -392,6 +437,32 @@ int jigsaw_spmm_launches_per_call(jigsaw_handle_t h, int64_t N) {
   return 1;  // jigsaw_spmm: one k_spmm launch; jigsaw_spmm_batched: one per 64 products
 }
 
+jigsaw_status_t jigsaw_last_launch(jigsaw_launch_desc_t* out) {
+  if (!out) return set_status(JIGSAW_ERROR_INVALID_VALUE, "NULL argument");
+  *out = last_launch();
+  return set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_status_t jigsaw_set_launch_override(const jigsaw_launch_override_t* o) {
+  LaunchOverride v;
+  if (o) {
+    for (int i = 0; i < 3; ++i)
+      if (o->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved fields must be zero");
+    if (!(o->tile_n == 0 || o->tile_n == 32 || o->tile_n == 64 || o->tile_n == 128 || o->tile_n == 256))
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "tile_n must be 0, 32, 64, 128 or 256");
+    if (!(o->split_k == 0 || o->split_k == 1 || o->split_k == 2 || o->split_k == 4 || o->split_k == 8))
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "split_k must be 0, 1, 2, 4 or 8");
+    if (o->host_chunks < 0) return set_status(JIGSAW_ERROR_INVALID_VALUE, "host_chunks must be >= 0");
+    v.tile_n = o->tile_n;
+    v.split_k = o->split_k;
+    v.no_pieces = o->no_pieces ? 1 : 0;
+    v.host_chunks = o->host_chunks;
+    v.k_pieces = o->k_pieces ? 1 : 0;
+  }
+  launch_override() = v;
+  return set_status(JIGSAW_SUCCESS);
+}
+
 int jigsaw_debug_trace(int64_t* out, int max_ctas) {
   if (!out || max_ctas == 0) return 0;
   return debug_trace_read(reinterpret_cast<long long*>(out), max_ctas);
@@ -419,6 +490,7 @@ jigsaw_status_t jigsaw_get_info(jigsaw_handle_t h, jigsaw_info_t* out) {
   out->panel_rows = f.P;
   out->residual_mode = f.mode;
   out->device = f.device;
+  out->c_dtype = f.c_dtype;
   out->npanels = f.npanels;
   out->ntiles = f.ntiles;
   out->ndtiles = f.ndtiles;

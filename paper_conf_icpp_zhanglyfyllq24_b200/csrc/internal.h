@@ -24,6 +24,7 @@ constexpr int kPad = -1;
 struct Format {
   int64_t M = 0, K = 0;
   int v = 0, P = kPanelRows, mode = 0, device = 0;
+  int c_dtype = JIGSAW_C_F16;  // element type of C written by jigsaw_spmm (jigsaw_options_t.c_dtype)
   int64_t npanels = 0, ntiles = 0, nksteps = 0, nkblocks = 0, ndtiles = 0;
   // host copies of per-panel counts / offsets
   std::vector<int32_t> T, D, tile_off, ks_off, kb_off;
@@ -54,6 +55,20 @@ struct Format {
 // status plumbing (api.cu)
 jigsaw_status_t set_status(jigsaw_status_t s, const std::string& msg = "");
 jigsaw_status_t cuda_status(cudaError_t e, const char* what);
+// stream-ordered allocation from the library's private pool of the current
+// device (api.cu); under stream capture it becomes a graph allocation node
+cudaError_t pool_alloc_async(void** p, size_t bytes, cudaStream_t s);
+
+// Diagnostic launch override (jigsaw_set_launch_override), per host thread.
+struct LaunchOverride {
+  int tile_n = 0;       // 0 = library choice; 32 / 64 / 128 / 256
+  int split_k = 0;      // 0 = library choice; 1 / 2 / 4 / 8 (single products, NT 64 or 32)
+  int no_pieces = 0;    // 1: grouped launches never cut units into k-range pieces
+  int host_chunks = 0;  // 0 = default; > 0: chunks of jigsaw_spmm_batched_host
+  int k_pieces = 0;     // 1: split long units by k-range pieces (workspace) instead of N slices
+};
+LaunchOverride& launch_override();
+jigsaw_launch_desc_t& last_launch();  // this thread's most recent jigsaw_spmm* call
 
 // reorder.cu: builds *f from device A (M x K fp16) on `stream`; synchronous.
 jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,

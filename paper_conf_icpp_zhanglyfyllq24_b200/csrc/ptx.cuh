@@ -1,5 +1,5 @@
-// ptx.cuh -- thin inline-PTX wrappers for sm_100a: mbarrier, bulk / tensor TMA
-// (incl. tile::gather4), tcgen05 (alloc, cp, mma, mma.sp, commit, ld).
+// ptx.cuh -- thin inline-PTX wrappers for sm_100a: mbarrier, bulk TMA, cp.async,
+// tcgen05 (alloc, cp, mma, mma.sp, commit, ld), clusters, programmatic launch.
 // Product code (libjigsaw.so).  Layout notes are in DESIGN.md §5.
 #pragma once
 #include <cstdint>
@@ -28,24 +28,6 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 }
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-// Non-blocking probe of phase `parity` (true once it has completed).
-__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred P1;\n\t"
-      "mbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
-      "selp.u32 %0, 1, 0, P1;\n\t}"
-      : "=r"(ok)
-      : "r"(smem_u32(bar)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-// Wait with back-off: for warps that wait long (the epilogue waits a whole
-// mainloop) so their polling does not take issue slots from the producer and
-// MMA warps on the same SM sub-partition.
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, uint32_t ns) {
-  while (!mbar_test(bar, parity)) __nanosleep(ns);
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   asm volatile(
@@ -101,27 +83,6 @@ __device__ __forceinline__ void bulk_s2cluster(uint32_t rdst, uint32_t src, uint
                "r"(src), "r"(bytes), "r"(rbar)
                : "memory");
 }
-// Four rows (r0..r3) x one box of columns starting at c0 of a 2-D tensor map.
-__device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, int32_t c0, int32_t r0,
-                                            int32_t r1, int32_t r2, int32_t r3, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
-      "l"(map), "r"(c0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int32_t c0, int32_t c1,
-                                            uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_u32(dst)),
-      "l"(map), "r"(c0), "r"(c1), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ void prefetch_tmap(const CUtensorMap* map) {
-  asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
-}
-
 // ---------------------------------------------------------------- tcgen05
 template <uint32_t kCols>
 __device__ __forceinline__ void tmem_alloc(uint32_t* dst_smem) {  // whole warp
@@ -139,16 +100,6 @@ __device__ __forceinline__ void tc_fence_before() {
 }
 __device__ __forceinline__ void tc_fence_after() {
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-}
-// All prior async tcgen05 ops of this thread arrive on `bar` once complete.
-__device__ __forceinline__ void tc_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
-                   smem_u32(bar))
-               : "memory");
-}
-// SMEM (128 rows x 16 B, K-major no-swizzle core matrices) -> TMEM lanes 0..127, 4 columns.
-__device__ __forceinline__ void tc_cp_128x128b(uint32_t taddr, uint64_t sdesc) {
-  asm volatile("tcgen05.cp.cta_group::1.128x128b [%0], %1;" ::"r"(taddr), "l"(sdesc) : "memory");
 }
 // D[tmem] (+)= A[smem, 2:4 compressed] . B[smem], metadata at [tmem_e].
 __device__ __forceinline__ void tc_mma_sp_f16(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
@@ -201,17 +152,6 @@ __device__ __forceinline__ void tmem_alloc_pair(uint32_t* dst_smem) {  // whole 
 template <uint32_t kCols>
 __device__ __forceinline__ void tmem_dealloc_pair(uint32_t taddr) {  // whole warp, both CTAs
   asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "n"(kCols));
-}
-// Completion of this thread's prior pair MMAs arrives on `bar` (same offset) in both CTAs.
-__device__ __forceinline__ void tc_commit_pair(uint64_t* bar) {
-  asm volatile(
-      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
-          smem_u32(bar)),
-      "h"((uint16_t)3)
-      : "memory");
-}
-__device__ __forceinline__ void tc_cp_128x128b_pair(uint32_t taddr, uint64_t sdesc) {
-  asm volatile("tcgen05.cp.cta_group::2.128x128b [%0], %1;" ::"r"(taddr), "l"(sdesc) : "memory");
 }
 __device__ __forceinline__ void tc_mma_sp_f16_pair(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
                                                    uint32_t e_tmem, uint32_t idesc, uint32_t accumulate) {
@@ -289,39 +229,6 @@ __device__ __forceinline__ void tc_mma_sp_f16_x4_warp(uint32_t d_tmem, uint64_t 
         : "memory");
   }
 }
-template <bool kPairT>
-__device__ __forceinline__ void tc_mma_sp_f16_x4(uint32_t d_tmem, uint64_t adesc0, uint64_t bdesc0, uint32_t astep,
-                                                 uint32_t bstep, uint32_t e_tmem, uint32_t idesc0, uint32_t acc0) {
-  if constexpr (kPairT) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t.reg .b64 a1, a2, a3, b1, b2, b3, as, bs;\n\t.reg .b32 e2, i1;\n\t"
-        "cvt.u64.u32 as, %3;\n\tcvt.u64.u32 bs, %4;\n\t"
-        "add.s64 a1, %1, as;\n\tadd.s64 a2, a1, as;\n\tadd.s64 a3, a2, as;\n\t"
-        "add.s64 b1, %2, bs;\n\tadd.s64 b2, b1, bs;\n\tadd.s64 b3, b2, bs;\n\t"
-        "add.u32 e2, %5, 2;\n\tor.b32 i1, %6, 1;\n\t"
-        "setp.ne.b32 p, %7, 0;\n\t"
-        "tcgen05.mma.sp.cta_group::2.kind::f16 [%0], %1, %2, [%5], %6, p;\n\t"
-        "tcgen05.mma.sp.cta_group::2.kind::f16 [%0], a1, b1, [%5], i1, 1;\n\t"
-        "tcgen05.mma.sp.cta_group::2.kind::f16 [%0], a2, b2, [e2], %6, 1;\n\t"
-        "tcgen05.mma.sp.cta_group::2.kind::f16 [%0], a3, b3, [e2], i1, 1;\n\t}" ::"r"(d_tmem),
-        "l"(adesc0), "l"(bdesc0), "r"(astep), "r"(bstep), "r"(e_tmem), "r"(idesc0), "r"(acc0)
-        : "memory");
-  } else {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t.reg .b64 a1, a2, a3, b1, b2, b3, as, bs;\n\t.reg .b32 e2, i1;\n\t"
-        "cvt.u64.u32 as, %3;\n\tcvt.u64.u32 bs, %4;\n\t"
-        "add.s64 a1, %1, as;\n\tadd.s64 a2, a1, as;\n\tadd.s64 a3, a2, as;\n\t"
-        "add.s64 b1, %2, bs;\n\tadd.s64 b2, b1, bs;\n\tadd.s64 b3, b2, bs;\n\t"
-        "add.u32 e2, %5, 2;\n\tor.b32 i1, %6, 1;\n\t"
-        "setp.ne.b32 p, %7, 0;\n\t"
-        "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], %1, %2, [%5], %6, p;\n\t"
-        "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], a1, b1, [%5], i1, 1;\n\t"
-        "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], a2, b2, [e2], %6, 1;\n\t"
-        "tcgen05.mma.sp.cta_group::1.kind::f16 [%0], a3, b3, [e2], i1, 1;\n\t}" ::"r"(d_tmem),
-        "l"(adesc0), "l"(bdesc0), "r"(astep), "r"(bstep), "r"(e_tmem), "r"(idesc0), "r"(acc0)
-        : "memory");
-  }
-}
 __device__ __forceinline__ void tc_mma_f16_pair(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
                                                 uint32_t idesc, uint32_t accumulate) {
   asm volatile(
@@ -358,12 +265,6 @@ __host__ __device__ constexpr uint32_t idesc_f16(int M, int N, int a_mn, int b_m
 
 namespace jig {
 // ---------------------------------------------------------------- cp.async (LDGSTS)
-// 16-byte global -> shared copy; src_bytes = 0 writes 16 zero bytes (zero fill).
-__device__ __forceinline__ void cp_async_16(void* dst, const void* src, uint32_t src_bytes) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
-               "r"(src_bytes)
-               : "memory");
-}
 // 16-byte cp.async to a shared::cta address; `zero` = write zeros, read nothing
 // (ignore-src predicate: maps to the LDGSTS ZFILL predicate, no size arithmetic).
 __device__ __forceinline__ void cp_async_16_zfill(uint32_t dst, const void* src, bool zero) {
@@ -388,9 +289,6 @@ __device__ __forceinline__ uint32_t cluster_ctarank() {
 // outstanding global stores to be performed (the release form does).
 __device__ __forceinline__ void cluster_sync_relaxed() {
   asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void cluster_sync_all() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 // Split cluster barrier: arrive now, wait (acquire) later, only where needed.
 __device__ __forceinline__ void cluster_arrive_relaxed() {
@@ -419,6 +317,23 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t rbar) {
 __device__ __forceinline__ void mbar_arrive_cluster_relaxed(uint32_t rbar) {
   asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(rbar) : "memory");
 }
+// Non-blocking probe (acquire, cluster scope) of phase `parity` of a local
+// mbarrier that remote CTAs arrive on: true once that phase has completed.
+__device__ __forceinline__ bool mbar_test_cluster(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\t"
+      "mbarrier.test_wait.parity.acquire.cluster.shared::cta.b64 P1, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, P1;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// 32-bit store to the shared memory of a CTA of the cluster (shared::cluster address).
+__device__ __forceinline__ void st_cluster_s32(uint32_t raddr, int32_t v) {
+  asm volatile("st.shared::cluster.b32 [%0], %1;" ::"r"(raddr), "r"(v) : "memory");
+}
 // Wait (acquire, cluster scope) for phase `parity` of a local mbarrier that remote CTAs arrive on.
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
   asm volatile(
@@ -431,16 +346,6 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
       "r"(parity)
       : "memory");
 }
-// 16-byte asynchronous store into (possibly remote) shared memory of the cluster,
-// completing 16 transaction bytes on the mbarrier at `rbar` (same CTA as `raddr`).
-__device__ __forceinline__ void st_async_v4(uint32_t raddr, uint32_t a, uint32_t b, uint32_t c, uint32_t d,
-                                            uint32_t rbar) {
-  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
-                   raddr),
-               "r"(a), "r"(b), "r"(c), "r"(d), "r"(rbar)
-               : "memory");
-}
-
 // ---------------------------------------------------------------- programmatic dependent launch
 // Block this thread until the grids this launch depends on (the previous kernels
 // of the stream) have completed and their memory is visible.  A no-op when the

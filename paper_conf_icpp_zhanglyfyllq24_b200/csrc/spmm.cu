@@ -39,6 +39,7 @@
 #include <vector>
 #include <string>
 #include <type_traits>
+#include <unordered_map>
 
 #include "internal.h"
 #include "ptx.cuh"
@@ -52,8 +53,8 @@
 #ifndef JIG_EARLY_TRIGGER
 #define JIG_EARLY_TRIGGER 1  // griddepcontrol.launch_dependents once a CTA has fetched its last unit
 #endif
-#ifndef JIG_HALVES
-#define JIG_HALVES 0  // pair N = 256 as two 128-column halves (see Cfg::kHalves); measured slower
+#ifndef JIG_DEV
+#define JIG_DEV 0  // developer build (-DJIG_DEV=1): timing-only JIGSAW_DBG modes and schedule experiments
 #endif
 
 namespace jig {
@@ -101,12 +102,11 @@ struct Cfg {
   static constexpr int kStageB = kChunks * kChunkB;
   static constexpr int kStages = kPair ? (NT == 256 ? 4 : 6) : NT == 256 ? 2 : NT == 128 ? 4 : 5;
   static constexpr int kAccCols = NT;
-  // kHalves (pair, N = 256): the accumulator is two 128-column halves taken from
-  // a ring of three half-buffers, each MMA k-step issued as two N = 128 MMAs, so
-  // the next unit starts as soon as the epilogue has drained one half.
-  static constexpr bool kHalves = JIG_HALVES && kPair && NT == 256;
-  static constexpr int kAccBufs = kHalves ? 3 : NT == 256 ? 1 : 2;   // TMEM: 512 columns total
-  static constexpr int kEColBase = kHalves ? 3 * 128 : kAccBufs * NT;
+  // TMEM (512 columns): double-buffered fp32 accumulators, one for NT = 256
+  // (two half-width accumulators issued as N = 128 MMAs measured slower in
+  // round 1); then 4 metadata columns per stage
+  static constexpr int kAccBufs = NT == 256 ? 1 : 2;
+  static constexpr int kEColBase = kAccBufs * NT;
   static constexpr uint32_t kTmemCols = kAccBufs * NT + 4 * kStages <= 256 ? 256 : 512;
   static constexpr int kRecvStride = NT * 4 + 16;          // bytes per received row (padded)
   static constexpr int kRecvBytes = kSplit ? 128 * kRecvStride : 0;
@@ -126,7 +126,7 @@ struct Cfg {
   static constexpr int kGS = (2 * kStages + kBGroups - 1) / kBGroups * kBGroups;
   static constexpr int kGAhead = kStages;
   static constexpr size_t kSmem =
-      1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 512;
+      1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 1024;
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
@@ -137,13 +137,14 @@ struct Problem {
   const int32_t* G;
   const int4* pin;  // per panel {k-steps, first k-step, first E block, 0} (device)
   const __half* B;
-  __half* C;
+  void* C;  // fp16 or fp32 (c32) row-major M x N
   int64_t M, N, K;
   int64_t planeA, planeE;  // bytes between the A / E planes of the two 128-row halves (P = 256)
   int64_t boff;  // offset of this problem's B in the concatenation of all B's (L2 prefetch)
   int npanels;
   int unit0;  // first global work unit of this problem
   int pin0;   // offset of this problem's panels in ParamsT::pin (if use_pin)
+  int c32;    // 1: C is fp32 (jigsaw_options_t.c_dtype), else fp16
 };
 // Kernel parameters: a problem table and the panel table, kept in parameter space
 // (read with LDC, no dependent global load at kernel start).  Two sizes: a
@@ -173,10 +174,14 @@ struct ParamsT {
   // a unit split into `pieces` k-ranges (split-K inside the persistent launch)
   // reduces its fp32 partials through `ws` (slots pslot .. pslot + pieces - 1)
   uint32_t ulist[MAXU];
-  float* ws;        // partial tiles: [slot][rank][NT / 32][warp 4][8][lane 32][4] fp32
-  int* wcnt;        // per split unit and CTA rank: pieces finished (reset by the last)
+  // Per-launch workspace (a region owned by the launching stream, or a graph-owned
+  // allocation under stream capture; spmm.cu acquire_workspace): counters that
+  // are zero at launch start and left zero, and the fp32 partial tiles of split units
+  float* ws;       // partial tiles: [slot][rank][NT / 32][warp 4][8][lane 32][4] fp32
+  int* wcnt;       // per split unit and CTA rank: pieces finished (reset by the last piece)
+  int* sched_ctr;  // dynamic tile scheduler: [next ticket, CTAs done fetching] (reset by the last CTA)
   int nprob, nunits, S, use_pin, use_ulist;
-  int sched;  // >= 0: dynamic tile scheduler on counter slot `sched`; -1: static round-robin
+  int dyn;    // 1: dynamic tile scheduler on sched_ctr; 0: static (round-robin / host schedule)
   int trace;  // 1: record a per-CTA timeline into g_trace (JIGSAW_TRACE=1)
   int prefetch;  // 1: prefetch each unit's gather lists / metadata into L2 at unit start
   int dbg;       // developer timing experiments (JIGSAW_DBG, results invalid): 1 skip tcgen05.cp, 2 skip MMAs,
@@ -224,10 +229,12 @@ struct Work {
   const uint8_t* Eimg;
   const int32_t* G;
   const __half* B;
-  __half* C;
+  void* C;
+  int c32;
   int64_t M, N, K;
   int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
   int piece, npieces, pslot;  // split-K piece of a grouped launch (npieces = 1: whole unit)
+  int ncols;                  // C columns of this unit (NT, or NT / nsplit for an N-split unit)
   bool valid;                 // false: padding entry of a static per-slot schedule
   int64_t ks0, kb0;  // first k-step / E block of the panel
   int64_t row0;      // first C row written by this CTA
@@ -242,6 +249,9 @@ struct Work {
   __device__ __forceinline__ int64_t gks(int kb) const { return ks0 + (int64_t)kb * kStepsPerBlock; }
 };
 constexpr uint32_t kNoWork = 0xFFFFFFFFu;  // schedule padding
+// Schedule code with partial-slot field kNSplit: an N-split unit, piece `piece`
+// of `pieces` column slices of width NT / pieces (full k-range, no workspace).
+constexpr uint32_t kNSplit = 0x1FFu;
 // `hint` = problem index of this thread's previous unit: units are visited in
 // increasing order, so the scan is amortised O(1) instead of O(problems).
 // kPair: `rank` selects this CTA's 128-row half of the 256-row panel (its A / E
@@ -259,6 +269,7 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
       w.G = prm.pr[0].G;
       w.B = prm.pr[0].B;
       w.C = prm.pr[0].C;
+      w.c32 = prm.pr[0].c32;
       w.M = prm.pr[0].M;
       w.N = prm.pr[0].N;
       w.K = prm.pr[0].K;
@@ -274,6 +285,7 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
       w.piece = 0;
       w.npieces = 1;
       w.pslot = 0;
+      w.ncols = NT;
       w.row0 = (int64_t)w.p * kPanelRows;
       return w;
     }
@@ -301,12 +313,21 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.G = prm.pr[i].G;
   w.B = prm.pr[i].B;
   w.C = prm.pr[i].C;
+  w.c32 = prm.pr[i].c32;
   w.M = prm.pr[i].M;
   w.N = prm.pr[i].N;
   w.K = prm.pr[i].K;
   const int np = prm.pr[i].npanels;
   w.p = lu % np;
   w.n0 = (lu / np) * NT;
+  w.ncols = NT;
+  if (pslot == (int)kNSplit) {  // column slice `piece` of the N tile, whole k-range
+    w.ncols = NT / npieces;
+    w.n0 += piece * w.ncols;
+    piece = 0;
+    npieces = 1;
+    pslot = 0;
+  }
   // panel table from parameter space (no dependent global load at kernel start)
   const int4 pi = prm.use_pin ? prm.pin[prm.pr[i].pin0 + w.p] : prm.pr[i].pin[w.p];
   w.nks = pi.x;
@@ -337,10 +358,19 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
 }
 
 // Dynamic tile scheduler (persistent launches): CTA b starts with unit b, then
-// takes gridDim.x + atomicAdd(counter); the counter slot is reset by the last CTA
-// to finish, so launches (and CUDA-graph replays) need no host-side memset.
-constexpr int kSchedSlots = 64, kSD = 4;  // counter slots per device, unit-ring depth
-__device__ int g_sched[kSchedSlots][2];   // [next unit, CTAs done]
+// takes gridDim.x + atomicAdd(ticket).  The counters live in the launch's
+// workspace (zero when the launch starts: see acquire_workspace) and are reset
+// to zero by the last CTA to stop fetching, so the next launch that uses the
+// same workspace (the next one on the stream) finds them zero.  (%gridid cannot
+// tag launches instead: CUDA-graph replays reuse the value fixed at
+// instantiation, tools/gridid_probe.cu.)
+constexpr int kSD = 4;  // unit-ring depth
+// CTA pairs under the dynamic scheduler: the even CTA takes the tickets and
+// forwards every unit id, in order, through a kMB-deep mailbox in the odd CTA's
+// shared memory (remote store + release arrive on the odd CTA's mfull; the odd
+// CTA frees the slot with a release arrive on the even CTA's mempty), so both
+// CTAs of the pair run the same unit sequence.
+constexpr int kMB = 16;
 
 // Unit-ring consumer: the A/E producer publishes each unit id (or -1 = done)
 // into a kSD-deep ring in shared memory; every consumer warp reads the same
@@ -388,8 +418,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint64_t* rfull = recv_full + 1;   // unit ring (dynamic scheduler)
   uint64_t* rempty = rfull + kSD;
   uint64_t* pfull = rempty + kSD;    // kPair, even CTA: the odd CTA's stage has landed
-  volatile int* ring = reinterpret_cast<volatile int*>(pfull + C_::kStages);
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pfull + C_::kStages) + kSD;
+  uint64_t* mfull = pfull + C_::kStages;  // kPair + dynamic, odd CTA: mailbox slot written by the even CTA
+  uint64_t* mempty = mfull + kMB;         // kPair + dynamic, even CTA: mailbox slot read by the odd CTA
+  volatile int* ring = reinterpret_cast<volatile int*>(mempty + kMB);
+  int* mbox = const_cast<int*>(ring) + kSD;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(mbox + kMB);
   const uint32_t s_last = smem_u32(tmem_slot + 1);  // split piece: this CTA reduces (int flag)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -398,7 +431,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   const int CS = kPair ? 2 : S;  // CTAs per cluster
   const uint32_t rank = (kSplit || kPair) ? cluster_ctarank() : 0;
   const int cluster_id = blockIdx.x / CS, nclusters = gridDim.x / CS;
-  const bool dyn = !kSplit && !kPair && prm.sched >= 0;
+  const bool dyn = !kSplit && prm.dyn;
   if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
     g_trace[blockIdx.x * kTraceSlots + 15] = gtimer();
     g_trace[blockIdx.x * kTraceSlots + 14] = smid();
@@ -430,7 +463,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   // are contiguous in shared memory: full, empty, gfull, gempty, tfull, tempty,
   // recv_full, rfull, rempty, pfull.
   if (warp == 0) {
-    constexpr int nb = 3 * C_::kStages + 2 * C_::kGS + 7 + 2 * kSD;
+    constexpr int nb = 3 * C_::kStages + 2 * C_::kGS + 7 + 2 * kSD + 2 * kMB;
     for (int i = lane; i < nb; i += 32) {
       int k = i;
       uint32_t cnt;
@@ -442,8 +475,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       else if ((k -= 3) < 3) cnt = kPair ? 8 : 4;          // tempty: epilogue warps (of both CTAs of a pair)
       else if ((k -= 3) < 1) cnt = 1;                      // recv_full
       else if ((k -= 1) < kSD) cnt = 1;                    // rfull
-      else if ((k -= kSD) < kSD) cnt = kBProdWarps + 1 + 4;  // rempty: B-producer warps + MMA + epilogue warps
-      else cnt = 1;                                        // pfull
+      else if ((k -= kSD) < kSD) cnt = kBProdWarps + 1 + 4;  // rempty: B-producer warps + MMA / relay + epilogue warps
+      else cnt = 1;                                        // pfull, mfull, mempty
       mbar_init(full + i, cnt);
     }
     fence_barrier_init();
@@ -522,16 +555,22 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     }
   }
 
+  if constexpr (kPair) {  // the unit mailbox is remote: the peer's barriers must be initialised
+    if (warp == 0 && dyn) {
+      cluster_wait();
+      cl_waited = true;
+    }
+  }
   if (warp == 0) {
     // ------------------------------------------------------------ A / E producer
     if (lane == 0) {
-      // the dynamic scheduler's counters are shared with the previous launch
+      // the dynamic scheduler's ticket is shared with the previous launch on the stream
       if (dyn) griddep_wait();
       // state after the parallel initial fill: stages 0..nA0-1 and gather slots
       // 0..nG0-1 hold the first unit's first k-blocks
       int stage = nA0 % C_::kStages, hint = 0, nkb_issued = nA0, rslot = 0;
       uint32_t phase = nA0 == C_::kStages ? 1u : 0u, rph = 0;
-      int* ctr = dyn ? &g_sched[prm.sched][0] : nullptr;
+      int* const ctr = prm.sched_ctr;
       // Unit sequence of this CTA (static stride or dynamic scheduler), fetched
       // into a small queue shared by two cursors over the same (unit, k-block)
       // sequence: the gather-list cursor runs kGAhead k-blocks ahead of the A/E
@@ -540,11 +579,38 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       constexpr int kQ = 16;
       int uq[kQ];
       int qn = 0, mq = 0, next_un = cluster_id;
-      auto fetch = [&]() {
-        const int un = next_un < prm.nunits ? next_un : -1;
-        if (un >= 0) next_un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : un + nclusters;
+      // Queues the CTA's next unit (-1 = none left).  Pairs under the dynamic
+      // scheduler: the even CTA forwards each unit to the odd CTA's mailbox, the
+      // odd CTA reads it from there.  Non-blocking calls (the gather cursor) give
+      // up when the mailbox slot is not ready, so only the A/E cursor -- which
+      // has issued every k-block of the units before -- ever waits on the peer.
+      auto fetch = [&](bool block) -> bool {
+        int un;
+        if (kPair && dyn) {
+          const int slot = qn % kMB;
+          const uint32_t ph = (uint32_t)(qn / kMB) & 1u;
+          if (rank == 0) {
+            if (!block && !mbar_test_cluster(&mempty[slot], ph ^ 1)) return false;
+            mbar_wait_cluster(&mempty[slot], ph ^ 1);
+            un = next_un < prm.nunits ? next_un : -1;
+            // forward first: the release arrive would otherwise wait for the
+            // ticket atomic below (the next ticket is only needed at the next fetch)
+            st_cluster_s32(mapa_shared(smem_u32(mbox + slot), 1), un);
+            mbar_arrive_cluster(mapa_shared(smem_u32(&mfull[slot]), 1));
+            if (un >= 0) next_un = nclusters + atomicAdd(ctr, 1);
+          } else {
+            if (!block && !mbar_test_cluster(&mfull[slot], ph)) return false;
+            mbar_wait_cluster(&mfull[slot], ph);
+            un = ld_shared_s32(smem_u32(mbox + slot));
+            mbar_arrive_cluster(mapa_shared(smem_u32(&mempty[slot]), 0));
+          }
+        } else {
+          un = next_un < prm.nunits ? next_un : -1;
+          if (un >= 0) next_un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : un + nclusters;
+        }
         uq[qn % kQ] = un;
         ++qn;
+        return true;
       };
       // gather-list cursor
       int gq = 0, ghint = 0, gkb = 0, gkbe = 0, gslot = nG0 % C_::kGS;
@@ -553,7 +619,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       bool gend = false;
       Work gwk = w0;
       if (nG0 > 0) {  // the gather cursor continues inside the first unit
-        fetch();
+        fetch(true);
         gq = 1;
         gkb = w0.kb_lo + nG0;
         gkbe = w0.kb_hi;
@@ -563,7 +629,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (gkb >= gkbe) {  // next unit with work
             if (gq == qn) {
               if (qn - mq >= kQ) return;  // queue full: the A/E cursor catches up first
-              fetch();
+              if (!fetch(false)) return;  // pair mailbox not ready: the A/E cursor goes on
             }
             const int u = uq[gq % kQ];
             if (u < 0) {
@@ -588,7 +654,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       };
       int64_t mi = nA0;  // k-blocks issued by the A/E cursor
       for (;;) {
-        if (mq == qn) fetch();
+        if (mq == qn) fetch(true);
         if (mq == 0) JIG_TRACE(16);
         const int u = uq[mq % kQ];
         ++mq;
@@ -614,7 +680,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           const bool dense = wk.dense(kb);
           const int64_t gks = wk.gks(kb);
           mbar_wait(&empty[stage], phase ^ 1);
-          if (prm.dbg & 16) {  // timing only: no A / metadata loads
+          if (JIG_DEV && (prm.dbg & 16)) {  // timing only: no A / metadata loads
             mbar_arrive(&full[stage]);
           } else {
             mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
@@ -628,11 +694,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
-      if (dyn) {  // the last CTA to finish fetching resets the counter slot
+      if (dyn && rank == 0) {  // the last CTA to stop fetching resets the ticket for the next launch
         __threadfence();
-        if (atomicAdd(&g_sched[prm.sched][1], 1) == (int)gridDim.x - 1) {
-          atomicExch(&g_sched[prm.sched][0], 0);
-          atomicExch(&g_sched[prm.sched][1], 0);
+        if (atomicAdd(ctr + 1, 1) == nclusters - 1) {
+          atomicExch(ctr, 0);
+          atomicExch(ctr + 1, 0);
         }
       }
       // This CTA takes no more units: once every CTA got here (all of them are
@@ -669,10 +735,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       // is then SHFL (row index) + IMAD.WIDE (address) + ISETP (bound) + LDGSTS
       // per 16 bytes: the B producers are issue-bound (a few extra instructions
       // per copy measured -25 % on C4).
-      const int col = wk.n0 + (kPair ? (int)rank * C_::kNTL : 0) + 8 * c;
+      // CTA r of a pair stages columns [r * ncols / 2, (r + 1) * ncols / 2) of the
+      // unit; lanes whose 16-byte chunk lies beyond the unit's width (an N-split
+      // unit narrower than NT) zero-fill it without reading (the MMA reads only
+      // ncols columns) -- the same ignore-src path as columns past N, so the hot
+      // loop carries no extra predicate
+      const int wl = kPair ? wk.ncols / 2 : wk.ncols;   // columns staged by this CTA
+      const int col = wk.n0 + (kPair ? (int)rank * wl : 0) + 8 * c;
       const char* const colbase = reinterpret_cast<const char*>(wk.B) + (int64_t)col * 2;
       const uint32_t ldb_bytes = (uint32_t)wk.N * 2u;
-      const uint32_t kbound = col < wk.N && !(prm.dbg & 8) ? (uint32_t)wk.K : 0u;  // dbg 8: no B reads
+      const uint32_t kbound = col < wk.N && 8 * c < wl && !(JIG_DEV && (prm.dbg & 8)) ? (uint32_t)wk.K : 0u;
       const uint32_t hsw = (uint32_t)((c & 7) ^ (lane / LPR));  // SW128 chunk of this lane, row phase 0
       int kb = wk.kb_lo + (int)((grp - j % C_::kBGroups + C_::kBGroups) % C_::kBGroups);
       j += kb - wk.kb_lo;
@@ -722,11 +794,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     // The even CTA issues the pair's MMAs; it may read this CTA's stage only once
     // this CTA's A/E bulk copies and B cp.async have landed: relay full -> pfull.
     if (lane == 0) {
-      int stage = 0, hint = 0, nrel = 0;
-      uint32_t phase = 0;
+      int stage = 0, hint = 0, nrel = 0, rslot = 0;
+      uint32_t phase = 0, rph = 0;
       const uint32_t rpfull = mapa_shared(smem_u32(pfull), 0);
-      for (int us = cluster_id; us < prm.nunits; us += nclusters) {
-        const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
+      for (int us = cluster_id;; us += nclusters) {
+        const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, false, lane) : (us < prm.nunits ? us : -1);
+        if (u < 0) break;
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
         if (!wk.valid) continue;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           mbar_wait(&full[stage], phase);
@@ -752,13 +826,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const bool issuer = lane == 0;
       const uint32_t tbase_u = __shfl_sync(kFullMask, tbase, 0);
       constexpr int MM = kPair ? 256 : 128;
-      const uint32_t idesc0 = idesc_f16(MM, NT, 0, 1, 1, 0);
-      const uint32_t idesc1 = idesc_f16(MM, NT, 0, 1, 1, 1);
-      const uint32_t idesc_dense = idesc_f16(MM, NT, 0, 1, 0, 0);
-      constexpr int NH = C_::kHalves ? 128 : NT;   // N of one MMA instruction
-      const uint32_t hdesc0 = idesc_f16(MM, NH, 0, 1, 1, 0);
-      const uint32_t hdesc1 = idesc_f16(MM, NH, 0, 1, 1, 1);
-      const uint32_t hdesc_dense = idesc_f16(MM, NH, 0, 1, 0, 0);
       int stage = 0, hint = 0, nkb_mma = 0, rslot = 0;
       uint32_t phase = 0, rph = 0;
       int it = 0;
@@ -771,18 +838,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         if (!wk.valid) continue;
         const int kb_lo = wk.kb_lo, kb_hi = wk.kb_hi;
         if (kb_lo == kb_hi) continue;
-        // accumulator buffer(s) of this unit; kHalves: half-uses 2it, 2it+1 of the 3-ring
-        const int a = C_::kHalves ? (2 * it) % 3 : it % C_::kAccBufs;
-        const int a1 = (2 * it + 1) % 3;
-        const uint32_t use = C_::kHalves ? (uint32_t)((2 * it) / 3) : (uint32_t)(it / C_::kAccBufs);
-        const uint32_t use1 = (uint32_t)((2 * it + 1) / 3);
+        // MMA N = the unit's width (NT, or a column slice of an N-split unit)
+        const uint32_t idesc0 = idesc_f16(MM, wk.ncols, 0, 1, 1, 0);
+        const uint32_t idesc1 = idesc0 | 1u;  // metadata selector id2 = 1
+        const uint32_t idesc_dense = idesc_f16(MM, wk.ncols, 0, 1, 0, 0);
+        const int a = it % C_::kAccBufs;  // accumulator buffer of this unit
+        const uint32_t use = (uint32_t)(it / C_::kAccBufs);
         if (kPair)
           mbar_wait_cluster(&tempty[a], (use & 1) ^ 1);
         else
           mbar_wait(&tempty[a], (use & 1) ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tbase_u + (C_::kHalves ? a * 128 : a * C_::kAccCols);
-        const uint32_t d_tmem1 = tbase_u + a1 * 128;
+        const uint32_t d_tmem = tbase_u + a * C_::kAccCols;
         for (int kb = kb_lo; kb < kb_hi; ++kb) {
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
@@ -799,43 +866,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
           const uint32_t e_tmem = tbase_u + C_::kEColBase + 4 * stage;
-          if (!dense && !(prm.dbg & 1)) {
+          if (!dense && !(JIG_DEV && (prm.dbg & 1))) {
             const uint64_t edesc = smem_desc(smem_u32(sE + stage * kStageE), 16, 128, 0);
             tc_cp_128x128b_warp<kPair>(e_tmem, edesc);
           }
           if (!kPair) JIG_TRACE_KB(4, nkb_mma);
           const uint32_t a_base = smem_u32(sA + stage * kStageA);
           const uint32_t b_base = smem_u32(sB + stage * C_::kStageB);
-          if (!C_::kHalves && !dense && steps == kStepsPerBlock && !(prm.dbg & 2)) {
+          if (!dense && steps == kStepsPerBlock && !(JIG_DEV && (prm.dbg & 2))) {
             // full sparse k-block: one asm block for the 4 MMAs (descriptors stepped in PTX)
             tc_mma_sp_f16_x4_warp<kPair>(d_tmem, smem_desc(a_base, 128, 256, 0),
                                          smem_desc(b_base, kChunkB, 1024, 2), kKStepBytesA >> 4,
                                          (32 * 128) >> 4, e_tmem, idesc0, kb != kb_lo);
           } else
-          for (int s = 0; s < (prm.dbg & 2 ? 0 : steps); ++s) {
+          for (int s = 0; s < (JIG_DEV && (prm.dbg & 2) ? 0 : steps); ++s) {
             const uint64_t adesc = smem_desc(a_base + s * kKStepBytesA, 128, 256, 0);
             const uint64_t bdesc = smem_desc(b_base + s * 32 * 128, kChunkB, 1024, 2);
             const uint32_t acc = (kb != kb_lo) || (s != 0);
-            if constexpr (C_::kHalves) {
-              // low half: SW128 chunk 0 of each CTA (unit columns [0,64) and [128,192));
-              // high half: chunk 1 (unit columns [64,128) and [192,256))
-              const uint64_t bdesc1 = smem_desc(b_base + kChunkB + s * 32 * 128, kChunkB, 1024, 2);
-              if (dense) {
-                if (issuer) tc_mma_f16_pair(d_tmem, adesc, bdesc, hdesc_dense, acc);
-              } else {
-                if (issuer) tc_mma_sp_f16_pair(d_tmem, adesc, bdesc, e_tmem + (s & 2), (s & 1) ? hdesc1 : hdesc0, acc);
-              }
-              if (kb == kb_lo && s == 0) {  // the high half-buffer: drained by the previous epilogue?
-                mbar_wait_cluster(&tempty[a1], (use1 & 1) ^ 1);
-                tc_fence_after();
-              }
-              if (issuer) {
-                if (dense)
-                  tc_mma_f16_pair(d_tmem1, adesc, bdesc1, hdesc_dense, acc);
-                else
-                  tc_mma_sp_f16_pair(d_tmem1, adesc, bdesc1, e_tmem + (s & 2), (s & 1) ? hdesc1 : hdesc0, acc);
-              }
-            } else if constexpr (kPair) {
+            if constexpr (kPair) {
               if (issuer) {
                 if (dense)
                   tc_mma_f16_pair(d_tmem, adesc, bdesc, idesc_dense, acc);
@@ -858,7 +906,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
         tc_commit_warp<kPair>(&tfull[a]);
-        if constexpr (C_::kHalves) tc_commit_warp<kPair>(&tfull[a1]);
         JIG_TRACE(5);
         ++it;
       }
@@ -881,31 +928,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       if (!wk.valid) continue;
       const int p = wk.p, n0 = wk.n0;
       const int64_t M = wk.M, N = wk.N;
-      __half* const Cm = wk.C;
+      void* const Cm = wk.C;
+      const bool c32 = wk.c32 != 0;
       const bool has_acc = wk.kb_hi > wk.kb_lo;
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
-      const int a = C_::kHalves ? (2 * it) % 3 : it % C_::kAccBufs;
-      const int a1 = (2 * it + 1) % 3;                   // kHalves: the high half-buffer
+      const int a = it % C_::kAccBufs;
+      const int ncols = wk.ncols;                        // C columns of this unit
       if (has_acc) {
-        mbar_wait(&tfull[a], (uint32_t)(C_::kHalves ? (2 * it) / 3 : it / C_::kAccBufs) & 1);
-        if constexpr (C_::kHalves) mbar_wait(&tfull[a1], (uint32_t)((2 * it + 1) / 3) & 1);
+        mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
         tc_fence_after();
       }
-      // 32-column chunk k of the unit: its TMEM column and its C column offset.
-      // kHalves: chunks 0-3 are the low half-buffer = unit columns [0,64) ++ [128,192),
-      // chunks 4-7 the high one = [64,128) ++ [192,256) (B is split across the pair
-      // by 64-column SW128 chunks, see the MMA issuer)
-      auto tcol = [&](int k) -> uint32_t {
-        if constexpr (C_::kHalves) return (uint32_t)((k < 4 ? a : a1) * 128 + 32 * (k & 3));
-        return (uint32_t)(a * C_::kAccCols + 32 * k);
-      };
-      auto ucol = [&](int k) -> int {
-        if constexpr (C_::kHalves) {
-          const int j = k >> 2, cc = 32 * (k & 3);
-          return cc < 64 ? 64 * j + cc : 128 + 64 * j + (cc - 64);
-        }
-        return 32 * k;
-      };
+      // 32-column chunk k of the unit: its TMEM column and its C column offset
+      auto tcol = [&](int k) -> uint32_t { return (uint32_t)(a * C_::kAccCols + 32 * k); };
+      auto ucol = [&](int k) -> int { return 32 * k; };
       auto release = [&](int buf) {  // this warp is done reading accumulator buffer `buf`
         tc_fence_before();
         __syncwarp();
@@ -916,7 +951,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             mbar_arrive(&tempty[buf]);
         }
       };
-      bool released_lo = false;
       if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
       if constexpr (!kSplit) {
         const uint32_t stg = smem_u32(sC + q * (32 * 64));
@@ -929,7 +963,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           constexpr size_t kTile = (size_t)128 * NT;  // floats per partial tile
           float* part = prm.ws + ((size_t)(wk.pslot + wk.piece) * CS + rank) * kTile;
 #pragma unroll 1
-          for (int c0 = 0; c0 < NT; c0 += 32) {
+          for (int c0 = 0; c0 < ncols; c0 += 32) {
             uint32_t v[32];
             if (has_acc) {
               tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + tcol(c0 / 32), v);
@@ -951,22 +985,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             int* cnt = prm.wcnt + wk.pslot * CS + rank;
             const int done = atomicAdd(cnt, 1);
             st_shared_s32(s_last, done == npc - 1);
-            if (done == npc - 1) atomicExch(cnt, 0);  // ready for the next launch
+            if (done == npc - 1) atomicExch(cnt, 0);  // zero again for the next launch
           }
           asm volatile("bar.sync 1, 128;" ::: "memory");
           write_c = ld_shared_s32(s_last) != 0;
           if (write_c) __threadfence();
         }
 #pragma unroll 1
-        for (int c0 = 0; write_c && c0 < NT; c0 += 32) {
+        for (int c0 = 0; write_c && c0 < ncols; c0 += 32) {
           uint32_t v[32];
           if (has_acc) {
             tc_ld_32x32b_x32(tbase + ((uint32_t)(q * 32) << 16) + tcol(c0 / 32), v);
             tc_wait_ld();
-            if (C_::kHalves && npc == 1 && c0 == 96) {  // low half drained: the next unit may start
-              release(a);
-              released_lo = true;
-            }
           } else {
 #pragma unroll
             for (int j = 0; j < 32; ++j) v[j] = 0;     // all-zero panel (R-Q21)
@@ -987,28 +1017,51 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
               }
             }
           }
-          // fp16 (RN), transposed through shared memory so that each store
-          // instruction writes 8 rows x 64 contiguous bytes (4 lanes per row)
-          // instead of 32 rows x 16 bytes; 16-byte chunks swizzled by (row >> 1) & 3
+          // Transposed through shared memory so that each store instruction
+          // writes 8 rows x 64 contiguous bytes (4 lanes per row) instead of 32
+          // rows x 16 bytes; 16-byte chunks swizzled by (row >> 1) & 3.
+          // fp16 C (RN): the 32 columns are one 64-byte row segment; fp32 C
+          // (c_dtype = 1): two 16-column halves of 64 bytes each.
+          if (!c32) {
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            uint4 pk;
-            pk.x = pack_h2(__uint_as_float(v[8 * j + 0]), __uint_as_float(v[8 * j + 1]));
-            pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
-            pk.z = pack_h2(__uint_as_float(v[8 * j + 4]), __uint_as_float(v[8 * j + 5]));
-            pk.w = pack_h2(__uint_as_float(v[8 * j + 6]), __uint_as_float(v[8 * j + 7]));
-            st_shared_v4u(stg + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4), pk);
-          }
-          __syncwarp();
+            for (int j = 0; j < 4; ++j) {
+              uint4 pk;
+              pk.x = pack_h2(__uint_as_float(v[8 * j + 0]), __uint_as_float(v[8 * j + 1]));
+              pk.y = pack_h2(__uint_as_float(v[8 * j + 2]), __uint_as_float(v[8 * j + 3]));
+              pk.z = pack_h2(__uint_as_float(v[8 * j + 4]), __uint_as_float(v[8 * j + 5]));
+              pk.w = pack_h2(__uint_as_float(v[8 * j + 6]), __uint_as_float(v[8 * j + 7]));
+              st_shared_v4u(stg + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4), pk);
+            }
+            __syncwarp();
 #pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const int rr = 8 * i + (lane >> 2), c = lane & 3;
-            const int64_t grow = wk.row0 + q * 32 + rr;
-            const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
-            const int col = n0 + ucol(c0 / 32) + 8 * c;
-            if (grow < M && col < N) *reinterpret_cast<uint4*>(Cm + grow * N + col) = pk;
+            for (int i = 0; i < 4; ++i) {
+              const int rr = 8 * i + (lane >> 2), c = lane & 3;
+              const int64_t grow = wk.row0 + q * 32 + rr;
+              const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
+              const int col = n0 + ucol(c0 / 32) + 8 * c;
+              if (grow < M && col < N) *reinterpret_cast<uint4*>(static_cast<__half*>(Cm) + grow * N + col) = pk;
+            }
+            __syncwarp();
+          } else {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+#pragma unroll
+              for (int j = 0; j < 4; ++j)
+                st_shared_v4u(stg + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4),
+                              make_uint4(v[16 * h + 4 * j], v[16 * h + 4 * j + 1], v[16 * h + 4 * j + 2],
+                                         v[16 * h + 4 * j + 3]));
+              __syncwarp();
+#pragma unroll
+              for (int i = 0; i < 4; ++i) {
+                const int rr = 8 * i + (lane >> 2), c = lane & 3;
+                const int64_t grow = wk.row0 + q * 32 + rr;
+                const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
+                const int col = n0 + ucol(c0 / 32) + 16 * h + 4 * c;
+                if (grow < M && col < N) *reinterpret_cast<uint4*>(static_cast<float*>(Cm) + grow * N + col) = pk;
+              }
+              __syncwarp();
+            }
           }
-          __syncwarp();
         }
       } else {
         // reduce-scatter of the fp32 partial tile through DSMEM: each warp stages
@@ -1072,19 +1125,24 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           const int64_t row = (int64_t)p * 128 + rank * rpo + i;
           const int64_t colg = n0 + c8 * 8;
           if (row < M && colg < N) {
-            uint4 pk;
-            pk.x = pack_h2(acc[0], acc[1]);
-            pk.y = pack_h2(acc[2], acc[3]);
-            pk.z = pack_h2(acc[4], acc[5]);
-            pk.w = pack_h2(acc[6], acc[7]);
-            *reinterpret_cast<uint4*>(Cm + row * N + colg) = pk;
+            if (c32) {
+              float4* dst = reinterpret_cast<float4*>(static_cast<float*>(Cm) + row * N + colg);
+              dst[0] = make_float4(acc[0], acc[1], acc[2], acc[3]);
+              dst[1] = make_float4(acc[4], acc[5], acc[6], acc[7]);
+            } else {
+              uint4 pk;
+              pk.x = pack_h2(acc[0], acc[1]);
+              pk.y = pack_h2(acc[2], acc[3]);
+              pk.z = pack_h2(acc[4], acc[5]);
+              pk.w = pack_h2(acc[6], acc[7]);
+              *reinterpret_cast<uint4*>(static_cast<__half*>(Cm) + row * N + colg) = pk;
+            }
           }
         }
       }
       if (warp == 2 && lane == 0) JIG_TRACE(9);
       if (has_acc) {
-        if (!released_lo) release(a);
-        if constexpr (C_::kHalves) release(a1);
+        release(a);
         ++it;
       }
     }
@@ -1117,25 +1175,62 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 
 int g_num_sms[64] = {0};
 
-// JIGSAW_PDL=0 launches without the programmatic-dependency attribute (A/B only).
-bool spmm_pdl_enabled() {
-  static const bool on = !(getenv("JIGSAW_PDL") && atoi(getenv("JIGSAW_PDL")) == 0);
-  return on;
+// Environment read ONCE per process (library load): JIGSAW_PDL=0 launches
+// without the programmatic-dependency attribute, JIGSAW_TRACE=1 records the
+// per-CTA timeline of jigsaw_debug_trace.  Developer builds (-DJIG_DEV=1) also
+// read the schedule / timing experiments below; product builds compile them
+// out (the constants are the product defaults).
+struct Knobs {
+  bool pdl = true, trace = false;
+  int dbg = 0;               // JIGSAW_DBG (timing only, results invalid)
+  bool no_prefetch = false;  // JIGSAW_NO_PREFETCH: no per-unit metadata prefetch into L2
+  bool static_sched = false; // JIGSAW_STATIC_SCHEDULE: no dynamic tile scheduler
+  int unit_cost = -1;        // JIGSAW_UNIT_COST: per-unit cost in k-block equivalents
+  bool sched_loc = false;    // JIGSAW_SCHED=loc: locality order, no cost sort, no pieces
+  bool debug_sched = false;  // JIGSAW_DEBUG_SCHED: print the pair schedule balance
+  int64_t group_bpf = 0;     // JIGSAW_GROUP_BPF (MB): L2 prefetch of all B's of a grouped launch
+  bool bpf = false;          // JIGSAW_BPF: L2 prefetch of B for single products
+  bool no_ctab = false;      // JIGSAW_NO_CTAB: no host-decoded first units
+  bool pair_dyn = false;     // JIGSAW_PAIR_DYN: dynamic scheduler for CTA pairs (measured slower than static LPT)
+  int split_pct = 125;       // JIGSAW_SPLIT_PCT: split a unit into pieces above this % of the per-slot load
+};
+const Knobs& knobs() {
+  static const Knobs k = [] {
+    Knobs r;
+    auto env = [](const char* n) -> const char* { return getenv(n); };
+    r.pdl = !(env("JIGSAW_PDL") && atoi(env("JIGSAW_PDL")) == 0);
+    r.trace = env("JIGSAW_TRACE") && env("JIGSAW_TRACE")[0] == '1';
+#if JIG_DEV
+    r.dbg = env("JIGSAW_DBG") ? atoi(env("JIGSAW_DBG")) : 0;
+    r.no_prefetch = env("JIGSAW_NO_PREFETCH") != nullptr;
+    r.static_sched = env("JIGSAW_STATIC_SCHEDULE") != nullptr;
+    r.unit_cost = env("JIGSAW_UNIT_COST") ? atoi(env("JIGSAW_UNIT_COST")) : -1;
+    r.sched_loc = env("JIGSAW_SCHED") && std::string(env("JIGSAW_SCHED")) == "loc";
+    r.debug_sched = env("JIGSAW_DEBUG_SCHED") != nullptr;
+    r.group_bpf = env("JIGSAW_GROUP_BPF") ? atoll(env("JIGSAW_GROUP_BPF")) : 0;
+    r.bpf = env("JIGSAW_BPF") != nullptr;
+    r.no_ctab = env("JIGSAW_NO_CTAB") != nullptr;
+    r.pair_dyn = env("JIGSAW_PAIR_DYN") != nullptr;
+    r.split_pct = env("JIGSAW_SPLIT_PCT") ? atoi(env("JIGSAW_SPLIT_PCT")) : 125;
+#endif
+    return r;
+  }();
+  return k;
 }
-bool g_attr_set[64][16] = {};  // [device][variant]
+std::atomic<bool> g_attr_set[64][16] = {};  // [device][variant]
 
 template <int NT, bool kSplit, bool kPair, class Prm>
 jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
   using C_ = Cfg<NT, kSplit, kPair>;
   auto kern = k_spmm<NT, kSplit, kPair, Prm>;
-  if (dev >= 0 && dev < 64 && !g_attr_set[dev][vid]) {
+  if (dev >= 0 && dev < 64 && !g_attr_set[dev][vid].load(std::memory_order_acquire)) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::kSmem);
     if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(k_spmm)");
     if (kSplit) {
       e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
       if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(cluster)");
     }
-    g_attr_set[dev][vid] = true;
+    g_attr_set[dev][vid].store(true, std::memory_order_release);
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
@@ -1151,17 +1246,26 @@ jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid
   // of the stream drains.  The prologue (barrier init, TMEM allocation, the
   // first k-blocks' compressed A / metadata / gather lists -- handle-owned,
   // immutable) runs before griddepcontrol.wait; every access to B, C and the
-  // shared workspaces / scheduler counters comes after it.
+  // launch workspace (counters, partial tiles) comes after it.
   attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = spmm_pdl_enabled() ? 2 : 1;
+  cfg.numAttrs = knobs().pdl ? 2 : 1;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, prm);
   if (e != cudaSuccess) return cuda_status(e, "k_spmm launch");
   return JIGSAW_SUCCESS;
 }
 
 }  // namespace
+
+LaunchOverride& launch_override() {
+  thread_local LaunchOverride o;
+  return o;
+}
+jigsaw_launch_desc_t& last_launch() {
+  thread_local jigsaw_launch_desc_t d = {};
+  return d;
+}
 
 int spmm_num_sms() {
   int dev = 0;
@@ -1176,8 +1280,8 @@ int spmm_num_sms() {
 // S = 1/2/4 CTAs by the cost model below.  256-row panels (CTA pairs): NT = 256
 // when there is a unit for every pair, else NT = 128; grid = 2 x pairs.
 void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* grid) {
+  const int force = launch_override().tile_n;
   if (f.P == kPairPanelRows) {
-    const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
     const int64_t u256 = f.npanels * ((N + 255) / 256);
     *NT = ((u256 >= sms / 2 && force != 128) || force == 256) ? 256 : 128;
     *S = 1;
@@ -1186,7 +1290,6 @@ void choose_config(const Format& f, int64_t N, int sms, int* NT, int* S, int* gr
     return;
   }
   const int64_t u256 = f.npanels * ((N + 255) / 256), u128 = f.npanels * ((N + 127) / 128);
-  const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
   int64_t kbs = 0;
   for (int64_t p = 0; p < f.npanels; ++p) kbs += (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
   const bool long_units = kbs >= 24 * f.npanels;  // NT = 256 runs a 2-stage ring: needs long units
@@ -1253,7 +1356,8 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
   P.G = f.d_G;
   P.pin = f.d_pin;
   P.B = reinterpret_cast<const __half*>(dB);
-  P.C = reinterpret_cast<__half*>(dC);
+  P.C = dC;
+  P.c32 = f.c_dtype == JIGSAW_C_F32 ? 1 : 0;
   P.M = f.M;
   P.N = N;
   P.K = f.K;
@@ -1263,18 +1367,92 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
 
 int g_trace_ctas = 0;
 
-std::atomic<unsigned> g_sched_next[64] = {};  // slot rotation, shared by host threads (unsigned: wraps)
+// ---------------------------------------------------------------- launch workspace
+// A launch that uses the dynamic tile scheduler or k-range pieces needs a small
+// device workspace: [ticket (256 B) | piece counters (512 slots x 2 ranks x 4 B) |
+// fp32 partial tiles].  The counters must be zero when a launch starts; each
+// launch leaves them zero (reset by the last CTA / last piece).  A workspace is
+// owned by exactly one launch at a time:
+//   * eager launches: one region per stream (keyed by cudaStreamGetId, which is
+//     unique for the life of the process), used only by launches on that
+//     stream; consecutive launches of a stream share it because every workspace
+//     access of a launch comes after griddepcontrol.wait (the previous kernel of
+//     the stream has completed and left the counters zero).  A region is taken
+//     from the library's stream-ordered pool on that stream and its counters
+//     zeroed on that stream; it grows by a new allocation and a stream-ordered
+//     free of the old region on the same stream -- no host or device
+//     synchronisation, no free of memory another stream may still use.
+//   * launches captured into a CUDA graph: a graph-owned allocation
+//     (cudaMallocFromPoolAsync during capture = an allocation node), a memset
+//     node zeroing its counters, and a free node right after the kernel node:
+//     every replay zeroes its own workspace, and graph replays never share one
+//     with any other launch (a graph exec never runs concurrently with itself).
+constexpr size_t kWsTicket = 256, kWsHead = kWsTicket + 512 * 2 * 4;
+struct StreamRegion {
+  char* base = nullptr;
+  size_t size = 0;
+};
+std::mutex g_ws_mu;
+std::unordered_map<unsigned long long, StreamRegion> g_ws[64];
+
+struct Workspace {
+  char* base = nullptr;
+  bool graph_owned = false;
+};
+
+static jigsaw_status_t acquire_workspace(int dev, size_t bytes, cudaStream_t s, Workspace* w) {
+  if (dev < 0 || dev >= 64) return set_status(JIGSAW_ERROR_INTERNAL, "device ordinal out of range");
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaError_t e = cudaStreamIsCapturing(s, &cs);
+  if (e != cudaSuccess) return cuda_status(e, "cudaStreamIsCapturing");
+  void* p = nullptr;
+  if (cs != cudaStreamCaptureStatusNone) {
+    e = pool_alloc_async(&p, bytes, s);
+    if (e != cudaSuccess) return cuda_status(e, "workspace allocation node (stream capture)");
+    e = cudaMemsetAsync(p, 0, kWsHead, s);
+    if (e != cudaSuccess) return cuda_status(e, "workspace memset node (stream capture)");
+    w->base = static_cast<char*>(p);
+    w->graph_owned = true;
+    return JIGSAW_SUCCESS;
+  }
+  unsigned long long id = 0;
+  e = cudaStreamGetId(s, &id);
+  if (e != cudaSuccess) return cuda_status(e, "cudaStreamGetId");
+  std::lock_guard<std::mutex> lock(g_ws_mu);
+  StreamRegion& r = g_ws[dev][id];
+  if (r.size < bytes) {
+    const size_t sz = std::max<size_t>({bytes, (size_t)4 << 20, 2 * r.size});
+    e = pool_alloc_async(&p, sz, s);
+    if (e != cudaSuccess) return cuda_status(e, "workspace allocation");
+    e = cudaMemsetAsync(p, 0, kWsHead, s);
+    if (e != cudaSuccess) return cuda_status(e, "workspace counters");
+    if (r.base) cudaFreeAsync(r.base, s);  // after every earlier launch of this stream
+    r.base = static_cast<char*>(p);
+    r.size = sz;
+  }
+  w->base = r.base;
+  w->graph_owned = false;
+  return JIGSAW_SUCCESS;
+}
 
 template <class Prm>
+static void set_workspace(Prm& prm, const Workspace& w) {
+  prm.sched_ctr = reinterpret_cast<int*>(w.base);
+  prm.wcnt = w.base ? reinterpret_cast<int*>(w.base + kWsTicket) : nullptr;
+  prm.ws = w.base ? reinterpret_cast<float*>(w.base + kWsHead) : nullptr;
+}
+
+// Launches k_spmm for the parameter block.  `pslots` split-piece slots of
+// `tile_bytes` each need workspace; the dynamic scheduler is used when a
+// single-CTA launch has more units than CTAs.
+template <class Prm>
 static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, bool pair, cudaStream_t s,
-                                     int npieces_total = -1) {
+                                     int npieces_total = -1, int pslots = 0, size_t tile_bytes = 0) {
   prm.S = S;
-  // persistent launches use the dynamic scheduler on a rotating counter slot
-  prm.sched = -1;
-  prm.prefetch = getenv("JIGSAW_NO_PREFETCH") ? 0 : 1;
-  prm.dbg = getenv("JIGSAW_DBG") ? atoi(getenv("JIGSAW_DBG")) : 0;
-  const char* tr = getenv("JIGSAW_TRACE");
-  prm.trace = (tr && tr[0] == '1') ? 1 : 0;
+  prm.prefetch = knobs().no_prefetch ? 0 : 1;
+
+  prm.dbg = JIG_DEV ? knobs().dbg : 0;
+  prm.trace = knobs().trace ? 1 : 0;
   if (prm.trace) g_trace_ctas = std::min(grid, kTraceCTAs);
   int u = 0;
   for (int i = 0; i < prm.nprob; ++i) {
@@ -1283,39 +1461,67 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   }
   prm.nunits = npieces_total >= 0 ? npieces_total : u;
   // (a CTA per unit needs no scheduler: its one unit is known at kernel start)
-  if (S == 1 && !pair && grid < prm.nunits && dev >= 0 && dev < 64 && !getenv("JIGSAW_STATIC_SCHEDULE"))
-    prm.sched = (int)(g_sched_next[dev]++ % kSchedSlots);
+  // CTA pairs: static greedy-LPT schedule (the dynamic one, with the even CTA
+  // forwarding tickets through a mailbox, measured 8-20 % slower on C2 / C4:
+  // units fetched ahead of time unbalance the tail); single CTAs: dynamic
+  prm.dyn = (S == 1 && (pair ? grid / 2 : grid) < prm.nunits && !knobs().static_sched &&
+             (!pair || knobs().pair_dyn)) ? 1 : 0;
+  Workspace w;
+  if (prm.dyn || pslots > 0) {
+    jigsaw_status_t st = acquire_workspace(dev, kWsHead + (size_t)pslots * tile_bytes, s, &w);
+    if (st != JIGSAW_SUCCESS) return st;
+  }
+  set_workspace(prm, w);
+  jigsaw_launch_desc_t& d = last_launch();
+  d.tile_n = NT;
+  d.split_k = S;
+  d.grid = grid;
+  d.cta_pair = pair ? 1 : 0;
+  d.problems = prm.nprob;
+  d.work_items = prm.nunits;
+  d.split_slots = pslots;
+  d.dynamic_schedule = prm.dyn;
+  d.graph_owned_workspace = w.graph_owned ? 1 : 0;
+  d.launches += 1;
   constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 8;
-  if (pair) {
-    if (NT == 256) return launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s);
-    return launch_variant<128, false, true>(prm, grid, 2, dev, vb + 4, s);
+  jigsaw_status_t st;
+  if (pair)
+    st = NT == 256 ? launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s)
+                   : launch_variant<128, false, true>(prm, grid, 2, dev, vb + 4, s);
+  else if (NT == 256)
+    st = launch_variant<256, false, false>(prm, grid, 1, dev, vb + 3, s);
+  else if (NT == 128)
+    st = launch_variant<128, false, false>(prm, grid, 1, dev, vb + 0, s);
+  else if (NT == 32 && S == 1)
+    st = launch_variant<32, false, false>(prm, grid, 1, dev, vb + 6, s);
+  else if (S == 1)
+    st = launch_variant<64, false, false>(prm, grid, 1, dev, vb + 1, s);
+  else if constexpr (std::is_same<Prm, ParamsOne>::value)
+    st = NT == 32 ? launch_variant<32, true, false>(prm, grid, S, dev, vb + 7, s)
+                  : launch_variant<64, true, false>(prm, grid, S, dev, vb + 2, s);
+  else
+    st = set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
+  if (w.graph_owned) {
+    cudaError_t e = cudaFreeAsync(w.base, s);  // free node right after the kernel node
+    if (st == JIGSAW_SUCCESS && e != cudaSuccess) st = cuda_status(e, "workspace free node");
   }
-  if (NT == 256) return launch_variant<256, false, false>(prm, grid, 1, dev, vb + 3, s);
-  if (NT == 128) return launch_variant<128, false, false>(prm, grid, 1, dev, vb + 0, s);
-  if (NT == 32 && S == 1) return launch_variant<32, false, false>(prm, grid, 1, dev, vb + 6, s);
-  if (S == 1) return launch_variant<64, false, false>(prm, grid, 1, dev, vb + 1, s);
-  if constexpr (std::is_same<Prm, ParamsOne>::value) {
-    if (NT == 32) return launch_variant<32, true, false>(prm, grid, S, dev, vb + 7, s);
-    return launch_variant<64, true, false>(prm, grid, S, dev, vb + 2, s);
-  }
-  return set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
+  return st;
 }
 
 static jigsaw_status_t launch_group(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
                                     void* const* Cs, int count, cudaStream_t s);
 
 jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC, cudaStream_t s) {
+  last_launch() = jigsaw_launch_desc_t{};
   thread_local ParamsOne prm;  // host-side scratch for the parameter block
   prm.nprob = 1;
-  prm.ws = nullptr;
-  prm.wcnt = nullptr;
   prm.use_pin = 1;
   prm.use_ulist = 0;
   fill_problem(prm, 0, f, dB, N, dC);
   int NT = 128, S = 1, grid = 1;
   choose_config(f, N, spmm_num_sms(), &NT, &S, &grid);
   const bool pair = f.P == kPairPanelRows;
-  const char* force_split = getenv("JIGSAW_FORCE_SPLIT");
+  const int force_split = launch_override().split_k;
   if (pair || (S == 1 && NT >= 128 && !force_split)) {
     // large products: the grouped persistent path (cost-ordered schedule, long
     // units split into pieces; CTA pairs are only scheduled there)
@@ -1325,18 +1531,15 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
   prm.use_ctab = 0;
   prm.bpf_bytes = 0;
   prm.bpf_chunk = 0;
-  if (const char* e = force_split) {  // test hook: force split S (NT = 64, or 32 with JIGSAW_FORCE_NT=32)
-    const int fs = atoi(e);
-    if (fs == 1 || fs == 2 || fs == 4 || fs == 8) {
-      const char* fn = getenv("JIGSAW_FORCE_NT");
-      NT = (fn && atoi(fn) == 32) ? 32 : 64;
-      S = fs;
-      const int64_t un = f.npanels * ((N + NT - 1) / NT);
-      grid = S > 1 ? (int)(un * S) : (int)std::min<int64_t>(un, spmm_num_sms());
-    }
+  if (force_split == 1 || force_split == 2 || force_split == 4 || force_split == 8) {
+    // diagnostic override: split-K S over a cluster (NT = 64, or 32 with tile_n = 32)
+    NT = launch_override().tile_n == 32 ? 32 : 64;
+    S = force_split;
+    const int64_t un = f.npanels * ((N + NT - 1) / NT);
+    grid = S > 1 ? (int)(un * S) : (int)std::min<int64_t>(un, spmm_num_sms());
   }
   // host-decoded first unit of every CTA (see ParamsT::ctab)
-  if (grid <= ParamsOne::kMaxCta && !getenv("JIGSAW_NO_CTAB")) {
+  if (grid <= ParamsOne::kMaxCta && !knobs().no_ctab) {
     const int64_t nkb_units = f.npanels * ((N + NT - 1) / NT);
     for (int c = 0; c < grid; ++c) {
       const int u = S > 1 ? c / S : c, r = S > 1 ? c % S : 0;
@@ -1354,72 +1557,13 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
     prm.use_ctab = 1;
   }
   // small B: prefetch it into L2 at kernel start, spread over the CTAs
+  // (developer option: measured 0.1-0.2 us slower)
   const int64_t bbytes = f.K * N * 2;
-  if (bbytes <= ((int64_t)16 << 20) && getenv("JIGSAW_BPF")) {  // opt-in: measured 0.1-0.2 us slower
+  if (bbytes <= ((int64_t)16 << 20) && knobs().bpf) {
     prm.bpf_bytes = bbytes;
     prm.bpf_chunk = ((bbytes + grid - 1) / grid + 255) & ~int64_t(255);
   }
   return launch_params(prm, NT, S, grid, f.device, pair, s);
-}
-
-// Device workspace for the fp32 partial tiles of split units, each region =
-// [counters | partial tiles].  The regions come in pairs; every stream that
-// launches split units gets its own pair on first use (kWsPairs streams per
-// device before pairs are shared) and alternates between its two regions, so
-// launches on different streams never share partials, and back-to-back
-// launches on one stream (which may overlap under programmatic dependent
-// launch) do not either.  Assigning a pair allocates nothing, so a capture
-// stream seen for the first time inside a capture still gets one.  The arena
-// grows outside stream capture only; counters are zeroed at allocation and
-// reset by the last piece of every unit.
-constexpr int kWsPairs = 8;
-struct SplitWs {
-  char* base = nullptr;
-  size_t region = 0;
-  int next_pair = 0;
-  std::vector<std::pair<cudaStream_t, int>> pair_of;  // stream -> pair index
-  int toggle[kWsPairs] = {};
-};
-SplitWs g_ws[64];
-std::mutex g_ws_mu;
-
-static bool split_workspace(int dev, size_t tile_bytes, size_t cnt_bytes, cudaStream_t s, float** ws, int** wcnt) {
-  if (dev < 0 || dev >= 64) return false;
-  std::lock_guard<std::mutex> lock(g_ws_mu);
-  SplitWs& w = g_ws[dev];
-  const size_t need = ((cnt_bytes + 255) & ~size_t(255)) + tile_bytes;
-  if (need > w.region) {
-    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return false;
-    if (cudaDeviceSynchronize() != cudaSuccess) return false;  // every stream's use of the old arena is done
-    if (w.base) cudaFree(w.base);
-    w.base = nullptr;
-    w.region = 0;
-    const size_t region = std::max(need, (size_t)8 << 20);
-    if (cudaMalloc(&w.base, region * 2 * kWsPairs) != cudaSuccess) {
-      cudaGetLastError();
-      w.base = nullptr;
-      return false;
-    }
-    if (cudaMemset(w.base, 0, region * 2 * kWsPairs) != cudaSuccess) {
-      cudaFree(w.base);
-      w.base = nullptr;
-      return false;
-    }
-    w.region = region;
-  }
-  int pi = -1;
-  for (const auto& e : w.pair_of)
-    if (e.first == s) pi = e.second;
-  if (pi < 0) {
-    pi = w.next_pair++ % kWsPairs;
-    w.pair_of.push_back({s, pi});
-  }
-  const int ri = 2 * pi + (w.toggle[pi]++ & 1);
-  char* r = w.base + (size_t)ri * w.region;
-  *wcnt = reinterpret_cast<int*>(r);
-  *ws = reinterpret_cast<float*>(r + ((cnt_bytes + 255) & ~size_t(255)));
-  return true;
 }
 
 // Grouped launch: many independent products in ONE persistent kernel (units of
@@ -1431,6 +1575,7 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
   thread_local ParamsGroup prm;
   const int sms = spmm_num_sms();
   const bool pair = count > 0 && fs[0]->P == kPairPanelRows;
+  const Knobs& kn = knobs();
   for (int i0 = 0; i0 < count; i0 += kMaxProblems) {
     const int n = std::min(kMaxProblems, count - i0);
     prm.nprob = n;
@@ -1451,7 +1596,7 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       for (int64_t p = 0; p < f.npanels; ++p) kbs += (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
       npan += f.npanels;
     }
-    const int force = getenv("JIGSAW_FORCE_NT") ? atoi(getenv("JIGSAW_FORCE_NT")) : 0;
+    const int force = launch_override().tile_n;
     int NT;
     if (pair) {
       NT = ((u256 >= sms / 2 && force != 128) || force == 256) ? 256 : 128;
@@ -1470,11 +1615,10 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
     // per-slot average is split into up to 8 k-range pieces (split-K inside the
     // persistent launch) so one long panel does not set the makespan.
     prm.use_ulist = 0;
-    prm.ws = nullptr;
-    prm.wcnt = nullptr;
-    int npieces_total = -1;
+    int npieces_total = -1, pslots = 0, nsplit_items = 0;
+    const size_t tile = (size_t)128 * NT * sizeof(float) * (pair ? 2 : 1);
     if (units <= ParamsGroup::kMaxUnits) {
-      struct U { int cost; int nkb; uint32_t code; };
+      struct U { int cost; int nkb; uint32_t code; int n0; int64_t N; };
       thread_local std::vector<U> us;
       us.clear();
       int64_t total = 0;
@@ -1483,30 +1627,53 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       // unit's epilogue is not overlapped with the next unit's mainloop: 4
       // (C2 at P = 256: 41.1 -> 35.3 us; the larger cost also stops the split
       // pieces whose workspace reduction cost more than the balance they bought,
-      // profiles/r01w_unit_cost.txt).  Developer override JIGSAW_UNIT_COST.
-      const int unit_cost = getenv("JIGSAW_UNIT_COST") ? atoi(getenv("JIGSAW_UNIT_COST")) : (pair && NT == 256 ? 4 : 1);
+      // profiles/r01w_unit_cost.txt).
+      const int unit_cost = kn.unit_cost >= 0 ? kn.unit_cost : (pair && NT == 256 ? 4 : 1);
       for (int i = 0; i < n; ++i) {
         const Format& f = *fs[i0 + i];
         const int ntn = (int)((Ns[i0 + i] + NT - 1) / NT);
         for (int p = 0; p < f.npanels; ++p)
           for (int t = 0; t < ntn; ++t) {  // N tiles of a panel adjacent: they share its A stream
             const int nkb = (f.pin[p].x + 3) / 4 + (f.pin[p].w + 3) / 4;
-            us.push_back({nkb + unit_cost, nkb, ((uint32_t)i << 26) | ((uint32_t)(t * f.npanels + p) << 15)});
+            us.push_back({nkb + unit_cost, nkb, ((uint32_t)i << 26) | ((uint32_t)(t * f.npanels + p) << 15), t * NT,
+                          Ns[i0 + i]});
             total += nkb + unit_cost;
           }
       }
-      // JIGSAW_SCHED=loc: locality order (problem, panel, N tile) dealt round-robin,
-      // no cost sort and no split pieces (developer experiment)
-      const bool loc = getenv("JIGSAW_SCHED") && std::string(getenv("JIGSAW_SCHED")) == "loc";
+      const bool loc = kn.sched_loc;  // developer experiment: locality order, no cost sort, no pieces
       const int64_t target = std::max<int64_t>(4, (total + slots_max - 1) / slots_max);
-      const bool allow_split = !getenv("JIGSAW_NO_PIECES") && !loc;
+      const bool allow_split = !launch_override().no_pieces && !loc;
       thread_local std::vector<std::pair<int, uint32_t>> order;
       order.clear();
-      int pslots = 0;
       if (!loc) std::stable_sort(us.begin(), us.end(), [](const U& a, const U& b) { return a.cost > b.cost; });
+      // Bytes a CTA ingests per k-block: compressed A + metadata, and the B rows
+      // of its NT_L columns (the cost of a column slice scales only the B part).
+      const double kb_a = kStepsPerBlock * kKStepBytesA + kEBlockBytes;
+      const double kb_b = 128.0 * 2 * (pair ? NT / 2 : NT);
+      const int ns_max = pair ? NT / 64 : NT / 32;  // narrowest slice: 32 B columns per CTA
       for (const U& x : us) {
         int np = 1;
-        if (allow_split && x.cost > target + target / 4 && x.nkb >= 8) {
+        const bool too_long = allow_split && (int64_t)x.cost * 100 > target * kn.split_pct;
+        if (too_long && ns_max >= 2 && !launch_override().k_pieces &&
+            (int64_t)order.size() + ns_max <= ParamsGroup::kMaxUnits) {
+          // N-split: column slices of the N tile over the whole k-range (each
+          // re-reads the unit's compressed A, none needs a partial-tile
+          // workspace or a reduction); the fewest slices that bring the unit
+          // to the per-slot load
+          int ns = 2;
+          auto slice_cost = [&](int n) {
+            return (int)(x.nkb * (kb_a + kb_b / n) / (kb_a + kb_b)) + unit_cost;
+          };
+          while (ns < ns_max && slice_cost(ns) > target) ns *= 2;
+          const int w = NT / ns;
+          for (int h = 0; h < ns; ++h)
+            if (x.n0 + h * w < x.N) {
+              order.push_back({-slice_cost(ns), x.code | ((uint32_t)h << 12) | ((uint32_t)(ns - 1) << 9) | kNSplit});
+              ++nsplit_items;
+            }
+          continue;
+        }
+        if (too_long && x.nkb >= 8) {
           np = (int)std::min<int64_t>({8, (x.cost + target - 1) / target, x.nkb / 4});
           if (pslots + np > 511 || (int64_t)order.size() + np > ParamsGroup::kMaxUnits) np = 1;
         }
@@ -1519,21 +1686,14 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
           order.push_back({-x.cost, x.code});
         }
       }
-      if (pslots > 0) {
-        const size_t tile = (size_t)128 * NT * sizeof(float) * (pair ? 2 : 1);
-        if (!split_workspace(fs[i0]->device, (size_t)pslots * tile, 2 * 512 * sizeof(int), s, &prm.ws, &prm.wcnt)) {
-          // no workspace (e.g. first use inside a stream capture): run whole units
-          order.clear();
-          for (const U& x : us) order.push_back({-x.cost, x.code});
-          pslots = 0;
-        }
-      }
       if (!loc)
         std::stable_sort(order.begin(), order.end(),
                          [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
       const int nslots = (int)std::min<int64_t>(slots_max, (int64_t)order.size());
       npieces_total = (int)order.size();
-      if (!pair) {
+      if (!pair || kn.pair_dyn) {
+        // cost order, handed out by the dynamic scheduler (CTA pairs, developer
+        // option: the even CTA takes the tickets and forwards them to its peer)
         for (size_t k = 0; k < order.size(); ++k) prm.ulist[k] = order[k].second;
       } else {
         // static schedule: greedy LPT (each piece, longest first, to the least
@@ -1561,7 +1721,7 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
           maxlen = std::max(maxlen, q[h.second].size());
           std::push_heap(heap.begin(), heap.end(), cmp);
         }
-        if (getenv("JIGSAW_DEBUG_SCHED")) {
+        if (JIG_DEV && kn.debug_sched) {
           int64_t lo = INT64_MAX, hi = 0;
           for (const auto& h : heap) lo = std::min(lo, h.first), hi = std::max(hi, h.first);
           fprintf(stderr, "[jigsaw] pair schedule: %zu pieces (%d split slots) on %d pairs, load min %lld max %lld "
@@ -1585,18 +1745,18 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
     }
     const int grid = pair ? 2 * slots : slots;
     // all B's of the launch small enough to sit in L2 next to the A stream:
-    // prefetch them at kernel start (JIGSAW_GROUP_BPF = cap in MB, 0 disables)
-    {
+    // prefetch them at kernel start (developer option; measured slower for C2,
+    // 44.7 vs 41.0 us)
+    if (kn.group_bpf > 0) {
       int64_t bsum = 0;
       for (int i = 0; i < n; ++i) bsum += fs[i0 + i]->K * Ns[i0 + i] * 2;
-      const char* e = getenv("JIGSAW_GROUP_BPF");
-      const int64_t cap = (int64_t)(e ? atoll(e) : 0) << 20;  // measured slower for C2 (44.7 vs 41.0 us): off
-      if (cap > 0 && bsum <= cap) {
+      if (bsum <= (kn.group_bpf << 20)) {
         prm.bpf_bytes = bsum;
         prm.bpf_chunk = ((bsum + grid - 1) / grid + 255) & ~int64_t(255);
       }
     }
-    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, pair, s, npieces_total);
+    jigsaw_status_t st = launch_params(prm, NT, 1, grid, fs[i0]->device, pair, s, npieces_total, pslots, tile);
+    last_launch().nsplit_items = nsplit_items;
     if (st != JIGSAW_SUCCESS) return st;
   }
   return JIGSAW_SUCCESS;
@@ -1604,6 +1764,7 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
 
 jigsaw_status_t launch_spmm_grouped(const Format* const* fs, const void* const* Bs, const int64_t* Ns,
                                     void* const* Cs, int count, cudaStream_t s) {
+  last_launch() = jigsaw_launch_desc_t{};
   bool mixed = false;
   for (int i = 1; i < count; ++i) mixed |= fs[i]->P != fs[0]->P;
   if (!mixed) return launch_group(fs, Bs, Ns, Cs, count, s);

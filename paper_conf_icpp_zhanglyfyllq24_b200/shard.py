@@ -52,3 +52,44 @@ def max_over_ranks(x: float, dist=None, device=None) -> float:
     t = torch.tensor([x], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def gather_column_shards(C_local, n0: int, n1: int, N: int, dist, world: int):
+    """Validation gather (untimed; north_star "NCCL only to gather C for
+    validation"): every rank contributes its column shard C[:, n0:n1] (padded to
+    the widest shard, so the collective moves equal-size buffers); returns the
+    assembled M x N tensor on every rank.  Works on any backend (NCCL on GPUs,
+    gloo in the CPU tests)."""
+    import torch
+    M = C_local.shape[0]
+    shards = column_shards(N, world)
+    width = max(b - a for a, b in shards)
+    pad = torch.zeros((M, width), dtype=C_local.dtype, device=C_local.device)
+    pad[:, : n1 - n0] = C_local
+    parts = [torch.empty_like(pad) for _ in range(world)]
+    dist.all_gather(parts, pad)
+    return torch.cat([p[:, : b - a] for p, (a, b) in zip(parts, shards)], dim=1)
+
+
+def format_hash(arrays: dict) -> int:
+    """64-bit hash (BLAKE2b) of a canonical format (jigsaw_export_format arrays,
+    fixed key order): ranks that rebuilt the replicated A must agree."""
+    import hashlib
+    h = hashlib.blake2b(digest_size=8)
+    for k in sorted(arrays):
+        h.update(k.encode())
+        h.update(memoryview(arrays[k]).cast("B"))
+    return int.from_bytes(h.digest(), "little") & 0x7FFFFFFFFFFFFFFF
+
+
+def check_against_dense(C, A_dense, B, rows, tol_rel: float = 1e-2, tol_abs: float = 1e-3):
+    """Sampled-row check of a (gathered) C against a plain dense PyTorch product
+    of the same fp16 inputs in fp32 (no oracle on the benchmark path): |C - A.B|
+    <= tol_rel (|A|.|B|) + tol_abs, the north_star tolerance.  Returns the max
+    excess (<= 0 means pass)."""
+    import torch
+    a = A_dense[rows].float()
+    ref = a @ B.float()
+    mabs = a.abs() @ B.float().abs()
+    err = (C[rows].float() - ref).abs()
+    return float((err - (tol_rel * mabs + tol_abs)).max())

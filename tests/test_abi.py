@@ -68,6 +68,50 @@ def test_reorder_validates_arguments_before_touching_the_device(L):
     opt = jig.Options(128, 0)
     opt.reserved[2] = 1
     assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(128, 0, 2)                       # c_dtype must be 0 (fp16) or 1 (fp32)
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+
+
+def test_binding_struct_layouts_match_header(tmp_path):
+    """The ctypes structures of the binding have the sizes and field offsets the C
+    compiler gives the structs of include/jigsaw.h (compiled here with gcc)."""
+    structs = {"jigsaw_options_t": jig.Options, "jigsaw_info_t": jig.Info, "jigsaw_format_host_t": jig.FormatHost,
+               "jigsaw_launch_desc_t": jig.LaunchDesc, "jigsaw_launch_override_t": jig.LaunchOverride}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "jigsaw.h"', 'int main(void) {']
+    for cname, py in structs.items():
+        lines.append(f'  printf("{cname} size %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'  printf("{cname} {f} %zu\\n", offsetof({cname}, {f}));')
+    lines.append("  return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c99", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
+    got = {}
+    for line in subprocess.check_output([str(exe)], text=True).splitlines():
+        c, f, v = line.split()
+        got[(c, f)] = int(v)
+    for cname, py in structs.items():
+        assert got[(cname, "size")] == ctypes.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert got[(cname, f)] == getattr(py, f).offset, (cname, f)
+
+
+def test_launch_override_and_descriptor(L):
+    """Diagnostic calls work without a device: the override is validated and
+    per-thread, the launch descriptor readable."""
+    for bad in [dict(tile_n=48), dict(split_k=3), dict(host_chunks=-1)]:
+        with pytest.raises(jig.JigsawError) as e:
+            jig.set_launch_override(**bad)
+        assert e.value.status == 1
+    o = jig.LaunchOverride(0, 0, 0, 0)
+    o.reserved[1] = 5
+    assert L.jigsaw_set_launch_override(ctypes.byref(o)) == 1
+    with jig.launch_override(tile_n=64, split_k=2):
+        pass
+    assert L.jigsaw_set_launch_override(None) == 0
+    d = jig.last_launch()
+    assert set(d) >= {"launches", "tile_n", "split_k", "grid", "cta_pair", "dynamic_schedule", "split_slots"}
 
 
 def test_spmm_validates_arguments(L):

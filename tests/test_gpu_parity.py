@@ -31,7 +31,16 @@ def _dev(x: np.ndarray):
 
 
 def _host(t) -> np.ndarray:
+    if t.dtype == torch.float32:
+        return t.cpu().numpy()
     return t.view(torch.int16).cpu().numpy().view(np.uint16)
+
+
+@pytest.fixture
+def override():
+    """jigsaw_set_launch_override for one test (this thread), reset afterwards."""
+    yield jig.set_launch_override
+    jig.set_launch_override()
 
 
 def assert_format_equal(gpu: dict, ref: oracle.Format, panels=None):
@@ -51,9 +60,26 @@ def assert_format_equal(gpu: dict, ref: oracle.Format, panels=None):
     assert np.array_equal(gpu["gather"][sl], ref.gather)
 
 
+def int_exact(C_gpu: np.ndarray, A, B, rows=None):
+    """Integer-valued fixture (A in {+-1,+-2}, B in {-2..2}): every partial sum is
+    an integer below 2^24, exact in fp32 in any order, so the GPU result must
+    equal the oracle bit for bit.  fp16 C: the fixture must stay within
+    |C| <= 2048 (integers exactly representable in fp16) -- asserted, not
+    skipped; fp32 C (c_dtype = 1): exact as is."""
+    C_ref, _ = oracle.spmm(A, B, rows=rows)
+    C = C_gpu if rows is None else C_gpu[rows]
+    if C.dtype == np.float32:
+        got = C.astype(np.float64)
+    else:
+        assert np.abs(C_ref).max() <= 2048, "integer fixture leaves the exactly representable fp16 range"
+        got = C.view(np.float16).astype(np.float64)
+    bad = np.argwhere(got != C_ref)
+    assert bad.size == 0, f"{len(bad)} mismatches, first at {bad[:3].tolist()}"
+
+
 def spmm_check(C_gpu: np.ndarray, A, B, rows=None):
     C_ref, Mabs = oracle.spmm(A, B, rows=rows)
-    C = C_gpu.view(np.float16).astype(np.float64)
+    C = C_gpu.astype(np.float64) if C_gpu.dtype == np.float32 else C_gpu.view(np.float16).astype(np.float64)
     if rows is not None:
         C = C[rows]
     err = np.abs(C - C_ref)
@@ -115,9 +141,7 @@ def test_venom_matrices(M, K, V, Mb, N, P):
     hi = jig.reorder(_dev(Ai), 1, panel_rows=P)
     Ci = _host(hi.spmm(_dev(Bi)))
     torch.cuda.synchronize()
-    C_ref, _ = oracle.spmm(Ai, Bi)
-    if np.abs(C_ref).max() <= 2048:
-        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+    int_exact(Ci, Ai, Bi)
 
 
 @pytest.mark.parametrize("seed", [11, 12])
@@ -295,39 +319,37 @@ def test_parameter_table_capacity_fallbacks(M, P):
     spmm_check(C, A, B, rows=rows)
 
 
-@pytest.mark.parametrize("force", ["1", "2", "4", "8"])
+@pytest.mark.parametrize("force", [1, 2, 4, 8])
 @pytest.mark.parametrize("M,K,v,s,N", [(512, 2048, 4, 0.9, 256), (384, 700, 8, 0.8, 200),
                                        (256, 96, 2, 0.95, 64)])
-def test_spmm_kernel_variants(force, M, K, v, s, N, monkeypatch):
+def test_spmm_kernel_variants(force, M, K, v, s, N, override):
     """Every k_spmm variant (NT = 64 with split-K S = 1/2/4/8 over a cluster and the
     DSMEM reduce-scatter) against the oracle, incl. splits that get no k-block."""
-    monkeypatch.setenv("JIGSAW_FORCE_SPLIT", force)
+    override(split_k=force)
     A = synth.vector_sparse(M, K, v, s, 3)
     B = synth.dense_b(K, N, 3)
     h = jig.reorder(_dev(A), v)
     C = _host(h.spmm(_dev(B)))
     torch.cuda.synchronize()
+    assert jig.last_launch()["split_k"] == force
     spmm_check(C, A, B)
     Ai = synth.vector_sparse(M, K, v, s, 4, kind="int")
     Bi = synth.dense_b(K, N, 4, kind="int")
     hi = jig.reorder(_dev(Ai), v)
     Ci = _host(hi.spmm(_dev(Bi)))
     torch.cuda.synchronize()
-    C_ref, _ = oracle.spmm(Ai, Bi)
-    if np.abs(C_ref).max() <= 2048:
-        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+    int_exact(Ci, Ai, Bi)
 
 
-@pytest.mark.parametrize("force", ["1", "2", "4"])
+@pytest.mark.parametrize("force", [1, 2, 4])
 @pytest.mark.parametrize("M,K,v,s,N", [(512, 2048, 4, 0.9, 256), (384, 700, 8, 0.8, 200),
                                        (256, 96, 2, 0.95, 40), (2048, 512, 8, 0.7, 104)])
-def test_spmm_nt32_variants(force, M, K, v, s, N, monkeypatch):
+def test_spmm_nt32_variants(force, M, K, v, s, N, override):
     """32-column tiles (the latency path of small single products; B staged in
     half of a 64-column SW128 chunk, N = 32 MMAs) with split-K S = 1/2/4, ragged
     N tails (N % 32 != 0), single and grouped launches, against the oracle;
     integer-valued inputs bit-exact."""
-    monkeypatch.setenv("JIGSAW_FORCE_NT", "32")
-    monkeypatch.setenv("JIGSAW_FORCE_SPLIT", force)
+    override(tile_n=32, split_k=force)
     A = synth.vector_sparse(M, K, v, s, 13)
     B = synth.dense_b(K, N, 13)
     h = jig.reorder(_dev(A), v)
@@ -337,10 +359,8 @@ def test_spmm_nt32_variants(force, M, K, v, s, N, monkeypatch):
     hi = jig.reorder(_dev(Ai), v)
     Ci = _host(hi.spmm(_dev(Bi)))
     torch.cuda.synchronize()
-    C_ref, _ = oracle.spmm(Ai, Bi)
-    if np.abs(C_ref).max() <= 2048:
-        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
-    monkeypatch.delenv("JIGSAW_FORCE_SPLIT")
+    int_exact(Ci, Ai, Bi)
+    override(tile_n=32)
     dC = [torch.empty((M, N), dtype=torch.float16, device="cuda") for _ in range(2)]
     jig.spmm_batched([h, hi], [_dev(B), _dev(Bi)], dC)
     torch.cuda.synchronize()
@@ -403,21 +423,19 @@ def test_dense_residual_mode(M, K, v, s, N, seed):
     hi = jig.reorder(_dev(Ai), v, residual_mode=1)
     Ci = _host(hi.spmm(_dev(Bi)))
     torch.cuda.synchronize()
-    C_ref, _ = oracle.spmm(Ai, Bi)
-    if np.abs(C_ref).max() <= 2048:
-        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+    int_exact(Ci, Ai, Bi)
 
 
-@pytest.mark.parametrize("force", ["2", "4"])
-def test_dense_residual_split_and_grouped(force, monkeypatch):
+@pytest.mark.parametrize("force", [2, 4])
+def test_dense_residual_split_and_grouped(force, override):
     """DENSE-mode k-blocks under split-K clusters and in a grouped launch."""
     mats = [synth.vector_sparse(256, 640, 4, 0.6, 70 + i) for i in range(3)]
     Bs = [synth.dense_b(640, 128, 80 + i) for i in range(3)]
     hs = [jig.reorder(_dev(a), 4, residual_mode=1) for a in mats]
-    monkeypatch.setenv("JIGSAW_FORCE_SPLIT", force)
+    override(split_k=force)
     for h, a, b in zip(hs, mats, Bs):
         spmm_check(_host(h.spmm(_dev(b))), a, b)
-    monkeypatch.delenv("JIGSAW_FORCE_SPLIT")
+    override()
     dB = [_dev(b) for b in Bs]
     dC = [torch.empty((256, 128), dtype=torch.float16, device="cuda") for _ in range(3)]
     jig.spmm_batched(hs, dB, dC)
@@ -426,11 +444,11 @@ def test_dense_residual_split_and_grouped(force, monkeypatch):
         spmm_check(_host(c), a, b)
 
 
-@pytest.mark.parametrize("nt", ["64", "128", "256"])
-def test_tile_width_variants(nt, monkeypatch):
+@pytest.mark.parametrize("nt", [64, 128, 256])
+def test_tile_width_variants(nt, override):
     """k_spmm with N tiles of 64 / 128 / 256 columns (single and grouped launches,
     SPTC and DENSE residual), N not a multiple of the tile width."""
-    monkeypatch.setenv("JIGSAW_FORCE_NT", nt)
+    override(tile_n=nt)
     mats = [synth.vector_sparse(384, 700, 8, 0.85, 90 + i) for i in range(2)]
     Bs = [synth.dense_b(700, 328, 91 + i) for i in range(2)]
     hs = [jig.reorder(_dev(mats[0]), 8), jig.reorder(_dev(mats[1]), 8, residual_mode=1)]
@@ -457,12 +475,12 @@ PAIR_CASES = [
 
 
 @pytest.mark.parametrize("M,K,v,s,N,kind,seed,mode", PAIR_CASES)
-@pytest.mark.parametrize("nt", ["128", "256"])
-def test_pair_panels_bit_exact_and_spmm(M, K, v, s, N, kind, seed, mode, nt, monkeypatch):
+@pytest.mark.parametrize("nt", [128, 256])
+def test_pair_panels_bit_exact_and_spmm(M, K, v, s, N, kind, seed, mode, nt, override):
     """panel_rows = 256 (R-Q6): one CTA pair per panel (tcgen05 cta_group::2, M = 256).
     Format bit-exact vs oracle O2 at P = 256 (incl. the two per-half planes the
     kernel reads), C within tolerance for N tiles of 128 and 256, integers bit-exact."""
-    monkeypatch.setenv("JIGSAW_FORCE_NT", nt)
+    override(tile_n=nt)
     A = synth.vector_sparse(M, K, v, s, seed, kind=kind)
     B = synth.dense_b(K, N, seed)
     h = jig.reorder(_dev(A), v, panel_rows=256, residual_mode=mode)
@@ -488,9 +506,8 @@ def test_pair_panels_bit_exact_and_spmm(M, K, v, s, N, kind, seed, mode, nt, mon
     hi = jig.reorder(_dev(Ai), v, panel_rows=256, residual_mode=mode)
     Ci = _host(hi.spmm(_dev(Bi)))
     torch.cuda.synchronize()
-    C_ref, _ = oracle.spmm(Ai, Bi)
-    if np.abs(C_ref).max() <= 2048:
-        assert np.array_equal(Ci.view(np.float16).astype(np.float64), C_ref)
+    assert jig.last_launch()["cta_pair"] == 1 and jig.last_launch()["tile_n"] == nt
+    int_exact(Ci, Ai, Bi)
 
 
 def test_pair_panels_grouped_mixed_with_single():
@@ -529,14 +546,19 @@ def test_pair_panels_full_size_sampled():
 
 
 @pytest.mark.parametrize("P", [128, 256])
-@pytest.mark.parametrize("pieces", ["on", "off"])
-def test_grouped_split_pieces(P, pieces, monkeypatch):
-    """Grouped launch where a few long units dominate: they are split into k-range
-    pieces reduced through the fp32 workspace (last-arriver); with the splitting
-    disabled (JIGSAW_NO_PIECES) the same batch runs whole units.  Both against the
-    oracle, integers bit-exact; replayed twice (the per-unit counters reset)."""
+@pytest.mark.parametrize("pieces", ["nsplit", "kpieces", "off"])
+def test_grouped_split_pieces(P, pieces, override):
+    """Grouped launch where a few long units dominate: they are cut into column
+    slices (N-split, the default: each slice re-reads the unit's A over the whole
+    k-range, no workspace) or, with the k_pieces override, into k-range pieces
+    whose fp32 partial tiles are reduced through the workspace (last-arriver);
+    with splitting disabled (no_pieces) the same batch runs whole units.  All
+    against the oracle, integers bit-exact; replayed twice (the per-unit
+    counters reset)."""
     if pieces == "off":
-        monkeypatch.setenv("JIGSAW_NO_PIECES", "1")
+        override(no_pieces=1)
+    elif pieces == "kpieces":
+        override(k_pieces=1)
     mats, Bs = [], []
     mats.append(synth.vector_sparse(512, 6000, 2, 0.5, 501, kind="int"))   # ~90 k-blocks per panel
     Bs.append(synth.dense_b(6000, 200, 502, kind="int"))
@@ -552,14 +574,12 @@ def test_grouped_split_pieces(P, pieces, monkeypatch):
               for a, b in zip(mats, Bs)]
         jig.spmm_batched(hs, dB, dC)
         torch.cuda.synchronize()
+        d = jig.last_launch()
+        assert (d["split_slots"] > 0) == (pieces == "kpieces"), d
+        assert (d["nsplit_items"] > 0) == (pieces == "nsplit"), d
         for i, (a, b, c) in enumerate(zip(mats, Bs, dC)):
             if i == 0:
-                C_ref, _ = oracle.spmm(a, b)
-                got = _host(c).view(np.float16).astype(np.float64)
-                if np.abs(C_ref).max() <= 2048:
-                    assert np.array_equal(got, C_ref)
-                else:
-                    spmm_check(_host(c), a, b)
+                int_exact(_host(c), a, b)
             else:
                 spmm_check(_host(c), a, b)
 
@@ -602,9 +622,8 @@ def test_spmm_batched_host_pipeline():
         spmm_check(c, a, b)
 
 
-@pytest.mark.gpu
-@pytest.mark.parametrize("chunks", ["1", "8"])
-def test_spmm_batched_host_packed_buffers(monkeypatch, chunks):
+@pytest.mark.parametrize("chunks", [1, 8])
+def test_spmm_batched_host_packed_buffers(override, chunks):
     """jigsaw_spmm_batched_host with every B in one pinned block and every C in
     another (views into one registration, back to back; one product with a
     size that is not a multiple of 256 B), whole batch as one chunk and as
@@ -625,7 +644,7 @@ def test_spmm_batched_host_packed_buffers(monkeypatch, chunks):
         ob += K * N
         oc += M * N
     blkC[...] = 0xFFFF
-    monkeypatch.setenv("JIGSAW_HOST_CHUNKS", chunks)        # 1: the whole batch is one chunk
+    override(host_chunks=chunks)                           # 1: the whole batch is one chunk
     jig.spmm_batched_host(hs, vb, vc)
     for a, b, c in zip(mats, Bs, vc):
         spmm_check(c, a, b)
@@ -645,8 +664,7 @@ def test_grouped_split_pieces_two_streams():
     hs = [jig.reorder(_dev(a), 2 if i == 0 else 4) for i, a in enumerate(mats)]
     dB = [_dev(b) for b in Bs]
     refs = [oracle.spmm(a, b)[0] for a, b in zip(mats, Bs)]
-    if max(np.abs(r).max() for r in refs) > 2048:
-        pytest.skip("integer fixture leaves the exactly representable fp16 range")
+    assert max(np.abs(r).max() for r in refs) <= 2048, "integer fixture must stay exact in fp16"
     streams = [torch.cuda.Stream(), torch.cuda.Stream()]
     big = torch.randn(4096, 4096, device="cuda", dtype=torch.float16)
     torch.cuda.synchronize()

@@ -9,7 +9,7 @@
 #include <cstdio>
 #include <vector>
 
-#include "../paper_conf_icpp_zhanglyfyllq24_b200/csrc/ptx.cuh"
+#include "ptx_tools.cuh"
 
 using namespace jig;
 

@@ -7,7 +7,7 @@
 
 #include <cstdio>
 
-#include "../paper_conf_icpp_zhanglyfyllq24_b200/csrc/ptx.cuh"
+#include "ptx_tools.cuh"
 
 using namespace jig;
 

@@ -17,7 +17,7 @@
 #include <cstring>
 #include <vector>
 
-#include "../paper_conf_icpp_zhanglyfyllq24_b200/csrc/ptx.cuh"
+#include "ptx_tools.cuh"
 
 using namespace jig;
 

@@ -24,11 +24,8 @@ def main():
             for i, (M, K, v, s, N) in enumerate(pts)]
     B2 = [dev(b) for _, b, _ in mats]
     C2 = [torch.empty((a.shape[0], b.shape[1]), dtype=torch.float16, device="cuda") for a, b, _ in mats]
-    for P, nt in [(128, ""), (256, "256"), (256, "256")]:
-        if nt:
-            os.environ["JIGSAW_FORCE_NT"] = nt
-        else:
-            os.environ.pop("JIGSAW_FORCE_NT", None)
+    for P, nt in [(128, 0), (256, 256)]:
+        jig.set_launch_override(tile_n=nt)
         hs = [jig.reorder(dev(a), v, panel_rows=P) for a, _, v in mats]
         for rep in range(3):
             flush.zero_()
@@ -38,7 +35,7 @@ def main():
             e1.record()
             torch.cuda.synchronize()
         tr = jig.debug_trace()
-        report(f"grouped C2 P={P} NT={nt or 'auto'}", e0.elapsed_time(e1) * 1e3, tr, ghz)
+        report(f"grouped C2 P={P} NT={nt or 'auto'} {jig.last_launch()}", e0.elapsed_time(e1) * 1e3, tr, ghz)
         kb = np.zeros(8 * 6 * 32, np.int64)
         jig.lib().jigsaw_debug_trace(kb.ctypes.data_as(ctypes.c_void_p), -1)
         kb = kb.reshape(8, 6, 32)
