@@ -64,6 +64,15 @@ typedef enum {
   JIGSAW_C_F32 = 1  /* C is fp32: the fp32 accumulator as is */
 } jigsaw_c_dtype_t;
 
+/* Row order of the panels (jigsaw_options_t.row_order). */
+typedef enum {
+  JIGSAW_ROWS_GIVEN = 0,     /* panels are consecutive rows of A as given (the paper, default) */
+  JIGSAW_ROWS_CLUSTERED = 1  /* row-clustered panels: rows sorted by their nonzero count (descending,
+                                ties by row index) before the panels are formed, so rows of similar
+                                density share a panel and sparse panels have fewer nonzero columns
+                                (smaller K_p, fewer tiles); the SpMM scatters C rows back */
+} jigsaw_row_order_t;
+
 typedef struct {
   int panel_rows;    /* rows per panel (the BLOCK_TILE analogue, R-Q5/R-Q6): 128 (one CTA per
                         panel; the default when opt is NULL), 256 (a CTA pair per panel:
@@ -74,7 +83,8 @@ typedef struct {
                         JIGSAW_ERROR_UNSUPPORTED (no tcgen05 M below 128 is built) */
   int residual_mode; /* jigsaw_residual_mode_t */
   int c_dtype;       /* jigsaw_c_dtype_t: element type of C for every product with this handle */
-  int reserved[5];   /* must be zero */
+  int row_order;     /* jigsaw_row_order_t */
+  int reserved[4];   /* must be zero */
 } jigsaw_options_t;
 
 /* Statistics of a prepared matrix (jigsaw_get_info). */
@@ -85,7 +95,7 @@ typedef struct {
   int32_t residual_mode;   /* jigsaw_residual_mode_t */
   int32_t device;          /* CUDA ordinal the handle lives on */
   int32_t c_dtype;         /* jigsaw_c_dtype_t */
-  int32_t reserved0;
+  int32_t row_order;       /* jigsaw_row_order_t */
   int64_t npanels;         /* ceil(M / P) */
   int64_t ntiles;          /* sum_p T_p: 2:4 tiles of 16 logical columns */
   int64_t ndtiles;         /* sum_p D_p: dense residual tiles (DENSE mode) */
@@ -114,6 +124,9 @@ typedef struct {
   uint8_t* nevict;   /* [ntiles]           evictions performed while building that tile */
   int32_t* rcol;     /* [ndtiles][16]      DENSE mode residual columns, -1 = PAD */
   uint16_t* dvals;   /* [ndtiles][P][16]   DENSE mode residual fp16 bits */
+  int32_t* rowmap;   /* [M]                row r of the (row-clustered) panels is row rowmap[r] of A
+                                           and of C; the identity for JIGSAW_ROWS_GIVEN.  The other
+                                           arrays describe the matrix A[rowmap] */
 } jigsaw_format_host_t;
 
 /* ---------------------------------------------------------------- north-star calls */

@@ -57,6 +57,8 @@ def lib():
         L.orc_format_copy.argtypes = [p] * 11
         L.orc_format_free.restype = None
         L.orc_format_free.argtypes = [p]
+        L.orc_row_cluster.restype = ctypes.c_int
+        L.orc_row_cluster.argtypes = [p, i64, i64, p]
         _lib = L
     return _lib
 
@@ -139,6 +141,7 @@ class Format:
     nevict: np.ndarray     # [ntiles] uint8
     rcol: np.ndarray       # [ndtiles, 16] int32 (DENSE mode)
     dvals: np.ndarray      # [ndtiles, P, 16] uint16 (DENSE mode)
+    rowmap: np.ndarray = None  # [M] int32: panel row r is row rowmap[r] of A (identity unless row-clustered)
 
     @property
     def tile_off(self):
@@ -154,11 +157,28 @@ class Format:
         return np.take_along_axis(self.col_idx, self.perm.astype(np.int64), axis=1)
 
 
-def reorder(A, P=128, mode=0, panels=None) -> Format:
+def row_cluster(A) -> np.ndarray:
+    """Row order of the row-clustered panels: rows by
+    decreasing nonzero count, ties by ascending index (orc_row_cluster)."""
+    A = _bits(A)
+    M, K = A.shape
+    perm = np.zeros(M, np.int32)
+    rc = lib().orc_row_cluster(_ptr(A), M, K, _ptr(perm))
+    if rc:
+        raise ValueError(f"orc_row_cluster failed ({rc})")
+    return perm
+
+
+def reorder(A, P=128, mode=0, panels=None, row_order=0) -> Format:
     """O2: canonical reorder CR1 of A (M x K fp16), panels of P rows.
     mode 0 = SPTC (paper), 1 = DENSE residual.  ``panels`` = (p0, p1) restricts
-    the work to a contiguous panel range (panels are independent)."""
+    the work to a contiguous panel range (panels are independent).  row_order 1:
+    row-clustered panels -- CR1 of A[row_cluster(A)], rowmap = that order."""
     A = _bits(A)
+    rowmap = None
+    if row_order:
+        rowmap = row_cluster(A)
+        A = np.ascontiguousarray(A[rowmap])
     M, K = A.shape
     npan = (M + P - 1) // P
     p0, p1 = (0, npan) if panels is None else panels
@@ -184,7 +204,7 @@ def reorder(A, P=128, mode=0, panels=None) -> Format:
     finally:
         lib().orc_format_free(h)
     return Format(M, K, P, mode, range(p0, p1), T, D, col_idx, perm, vals, meta, kind,
-                  nevict, rcol, dvals)
+                  nevict, rcol, dvals, rowmap if rowmap is not None else np.arange(M, dtype=np.int32))
 
 
 from .check import check_format, decode, format_bytes, canon  # noqa: E402,F401

@@ -16,6 +16,8 @@
  *       orc_tile_reorder   Alg. 1 + reorder retry on ONE tile, generalised to
  *                          W columns / groups of G / at most Z nonzeros per group
  *                          (CR1 is W=16,G=4,Z=2; the Fig. 6 example is W=4,G=2,Z=1)
+ *       orc_row_cluster    row order of the row-clustered panels (SURVEY §8(f) f2,
+ *                          DESIGN.md R-Q27): CR1 is then applied to A[perm]
  *   (O3, the independent checker/decoder, is oracle/check.py: numpy, no call into O2.)
  *
  * Parity status: every function here is pinned by tests/test_oracle_*.py except
@@ -466,4 +468,28 @@ void orc_format_free(void *h)
     free(f->T); free(f->D); free(f->col_idx); free(f->perm); free(f->vals);
     free(f->meta); free(f->kind); free(f->nevict); free(f->rcol); free(f->dvals);
     free(f);
+}
+
+/* ------------------------------------------------------------------------- */
+/* Row-clustered panels (DESIGN.md R-Q27, not in the paper:  */
+/* the B200 analogue of its small BLOCK_TILE)                   */
+/* ------------------------------------------------------------------------- */
+
+/* perm[i] = the i-th row of A in order of decreasing nonzero count (nz16),
+ * rows with equal counts in ascending index order.  Written as the definition:
+ * for every count from K down to 0, the rows with that count, scanned in order. */
+int orc_row_cluster(const uint16_t *A, int64_t M, int64_t K, int32_t *perm)
+{
+    int64_t *cnt = (int64_t *)malloc(sizeof(int64_t) * (size_t)(M > 0 ? M : 1));
+    if (!cnt) return 1;
+    for (int64_t r = 0; r < M; ++r) {
+        cnt[r] = 0;
+        for (int64_t k = 0; k < K; ++k) cnt[r] += nz16(A[r * K + k]);
+    }
+    int64_t i = 0;
+    for (int64_t c = K; c >= 0; --c)
+        for (int64_t r = 0; r < M; ++r)
+            if (cnt[r] == c) perm[i++] = (int32_t)r;
+    free(cnt);
+    return i == M ? 0 : 2;
 }

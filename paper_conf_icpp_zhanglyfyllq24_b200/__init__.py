@@ -32,6 +32,7 @@ ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_stat
                "jigsaw_debug_trace", "jigsaw_last_launch", "jigsaw_set_launch_override"]
 
 C_F16, C_F32 = 0, 1            # jigsaw_c_dtype_t
+ROWS_GIVEN, ROWS_CLUSTERED = 0, 1   # jigsaw_row_order_t
 
 
 class JigsawError(RuntimeError):
@@ -42,13 +43,13 @@ class JigsawError(RuntimeError):
 
 class Options(ctypes.Structure):
     _fields_ = [("panel_rows", ctypes.c_int), ("residual_mode", ctypes.c_int), ("c_dtype", ctypes.c_int),
-                ("reserved", ctypes.c_int * 5)]
+                ("row_order", ctypes.c_int), ("reserved", ctypes.c_int * 4)]
 
 
 class Info(ctypes.Structure):
     _fields_ = [("M", ctypes.c_int64), ("K", ctypes.c_int64), ("v", ctypes.c_int32),
                 ("panel_rows", ctypes.c_int32), ("residual_mode", ctypes.c_int32),
-                ("device", ctypes.c_int32), ("c_dtype", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+                ("device", ctypes.c_int32), ("c_dtype", ctypes.c_int32), ("row_order", ctypes.c_int32),
                 ("npanels", ctypes.c_int64), ("ntiles", ctypes.c_int64),
                 ("ndtiles", ctypes.c_int64), ("overflow_tiles", ctypes.c_int64),
                 ("evictions", ctypes.c_int64), ("nnz", ctypes.c_int64), ("kp_total", ctypes.c_int64),
@@ -59,7 +60,8 @@ class Info(ctypes.Structure):
 
 class FormatHost(ctypes.Structure):
     _fields_ = [(n, ctypes.c_void_p) for n in
-                ("T", "D", "col_idx", "perm", "gather", "vals", "meta", "kind", "nevict", "rcol", "dvals")]
+                ("T", "D", "col_idx", "perm", "gather", "vals", "meta", "kind", "nevict", "rcol", "dvals",
+                 "rowmap")]
 
 
 class LaunchDesc(ctypes.Structure):
@@ -238,7 +240,7 @@ class Handle:
                    gather=np.zeros((nt, 16), np.int32), vals=np.zeros((nt, P, 8), np.uint16),
                    meta=np.zeros((nt, P), np.uint16), kind=np.zeros(nt, np.uint8),
                    nevict=np.zeros(nt, np.uint8), rcol=np.zeros((nd, 16), np.int32),
-                   dvals=np.zeros((nd, P, 16), np.uint16))
+                   dvals=np.zeros((nd, P, 16), np.uint16), rowmap=np.zeros(inf["M"], np.int32))
         fh = FormatHost(**{k: v.ctypes.data for k, v in arr.items()})
         _raise_if(lib().jigsaw_export_format(self._h, ctypes.byref(fh)))
         return arr
@@ -256,11 +258,11 @@ class Handle:
 
 
 def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: int = C_F16,
-            stream=None) -> Handle:
+            row_order: int = ROWS_GIVEN, stream=None) -> Handle:
     """jigsaw_reorder_ex: multi-granularity reorder + format build of A (CUDA fp16 M x K)."""
     _check_fp16_cuda(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode, c_dtype)
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_ex(ctypes.c_void_p(A.data_ptr()), M, K, v, ctypes.byref(opt),
                                       _stream_ptr(stream), ctypes.byref(out)))
@@ -268,11 +270,11 @@ def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: i
 
 
 def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: int = 0,
-                 c_dtype: int = C_F16) -> Handle:
+                 c_dtype: int = C_F16, row_order: int = ROWS_GIVEN) -> Handle:
     """jigsaw_reorder_host: A given as a host array (fp16 or uint16 bits)."""
     A = _host16(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode, c_dtype)
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_host(A.ctypes.data_as(ctypes.c_void_p), M, K, v,
                                         ctypes.byref(opt), None, ctypes.byref(out)))

@@ -145,7 +145,9 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
     if (opt->c_dtype != JIGSAW_C_F16 && opt->c_dtype != JIGSAW_C_F32)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown c_dtype");
-    for (int i = 0; i < 5; ++i)
+    if (opt->row_order != JIGSAW_ROWS_GIVEN && opt->row_order != JIGSAW_ROWS_CLUSTERED)
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown row_order");
+    for (int i = 0; i < 4; ++i)
       if (opt->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved options must be zero");
   }
   return JIGSAW_SUCCESS;
@@ -195,8 +197,8 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
   if (!h) return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "host allocation failed");
   set_status(JIGSAW_SUCCESS);
   s = build_format(static_cast<const uint16_t*>(A), M, K, v, resolve_panel_rows(opt, M),
-                   opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC, reinterpret_cast<cudaStream_t>(stream),
-                   &h->f);
+                   opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC, opt ? opt->row_order : (int)JIGSAW_ROWS_GIVEN,
+                   reinterpret_cast<cudaStream_t>(stream), &h->f);
   if (s != JIGSAW_SUCCESS) {
     delete h;
     return s;
@@ -491,6 +493,7 @@ jigsaw_status_t jigsaw_get_info(jigsaw_handle_t h, jigsaw_info_t* out) {
   out->residual_mode = f.mode;
   out->device = f.device;
   out->c_dtype = f.c_dtype;
+  out->row_order = f.row_order;
   out->npanels = f.npanels;
   out->ntiles = f.ntiles;
   out->ndtiles = f.ndtiles;
@@ -518,6 +521,12 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
   if (out->D)
     for (int64_t p = 0; p < f.npanels; ++p) out->D[p] = f.D.empty() ? 0 : f.D[p];
   cudaError_t e = cudaSuccess;
+  if (out->rowmap) {
+    if (f.d_rowmap)
+      e = cudaMemcpy(out->rowmap, f.d_rowmap, sizeof(int32_t) * f.M, cudaMemcpyDeviceToHost);
+    else
+      for (int64_t r = 0; r < f.M; ++r) out->rowmap[r] = (int32_t)r;
+  }
   if (nt && out->col_idx && e == cudaSuccess) e = cudaMemcpy(out->col_idx, f.d_colidx, nt * 16 * 4, cudaMemcpyDeviceToHost);
   if (nt && out->perm && e == cudaSuccess) e = cudaMemcpy(out->perm, f.d_perm, nt * 16, cudaMemcpyDeviceToHost);
   if (nt && out->kind && e == cudaSuccess) e = cudaMemcpy(out->kind, f.d_kind, nt, cudaMemcpyDeviceToHost);

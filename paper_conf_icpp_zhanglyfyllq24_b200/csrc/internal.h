@@ -25,6 +25,8 @@ struct Format {
   int64_t M = 0, K = 0;
   int v = 0, P = kPanelRows, mode = 0, device = 0;
   int c_dtype = JIGSAW_C_F16;  // element type of C written by jigsaw_spmm (jigsaw_options_t.c_dtype)
+  int row_order = JIGSAW_ROWS_GIVEN;
+  int32_t* d_rowmap = nullptr;  // [M] (row-clustered panels only): C row of panel row r
   int64_t npanels = 0, ntiles = 0, nksteps = 0, nkblocks = 0, ndtiles = 0;
   // host copies of per-panel counts / offsets
   std::vector<int32_t> T, D, tile_off, ks_off, kb_off;
@@ -71,7 +73,7 @@ LaunchOverride& launch_override();
 jigsaw_launch_desc_t& last_launch();  // this thread's most recent jigsaw_spmm* call
 
 // reorder.cu: builds *f from device A (M x K fp16) on `stream`; synchronous.
-jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
+jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode, int row_order,
                              cudaStream_t stream, Format* f);
 void free_format(Format* f);
 

@@ -744,8 +744,106 @@ void free_format(Format* f) {
     if (_e != cudaSuccess) { cuda_status(_e, what); goto fail; } \
   } while (0)
 
-jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
+// ------------------------------------------------------------------ row-clustered panels (f2)
+// RC1: nonzero count of every row of A (one CTA per row).
+__global__ void __launch_bounds__(256) k_rownnz(const uint16_t* __restrict__ A, int64_t K, int32_t* __restrict__ cnt) {
+  const int64_t r = blockIdx.x;
+  int c = 0;
+  for (int64_t k = threadIdx.x; k < K; k += blockDim.x) c += (A[r * K + k] & 0x7FFF) != 0;
+  for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xFFFFFFFFu, c, o);
+  __shared__ int part[8];
+  if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int t = 0;
+    for (int w = 0; w < 8; ++w) t += part[w];
+    cnt[r] = t;
+  }
+}
+// RC2: A'[i][:] = A[rowmap[i]][:] (one CTA per row).
+__global__ void __launch_bounds__(256) k_permute_rows(const uint16_t* __restrict__ A, int64_t K,
+                                                      const int32_t* __restrict__ rowmap, uint16_t* __restrict__ Ap) {
+  const int64_t i = blockIdx.x, r = rowmap[i];
+  for (int64_t k = threadIdx.x; k < K; k += blockDim.x) Ap[i * K + k] = A[r * K + k];
+}
+
+static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
+                                         cudaStream_t stream, Format* f);
+
+// Row-clustered panels (DESIGN.md R-Q27): the rows are ordered by
+// nonzero count, descending, ties by ascending row index (a stable counting sort
+// on the host), the format is built for A[rowmap] exactly as for any matrix, and
+// the SpMM epilogue writes panel row r to C row rowmap[r].  Panels of sparse
+// rows then have fewer nonzero columns (K_p), hence fewer tiles and fewer B rows
+// to gather.  The row order of vector-sparse rows (v identical rows) is kept.
+jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode, int row_order,
                              cudaStream_t stream, Format* f) {
+  if (row_order != JIGSAW_ROWS_CLUSTERED) return build_format_rows(dA, M, K, v, P, mode, stream, f);
+  int32_t *cnt = nullptr, *rmap = nullptr;
+  uint16_t* Ap = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  std::vector<int32_t> hc(M), hmap(M);
+  jigsaw_status_t st = JIGSAW_SUCCESS;
+  float ms = 0;
+  auto cleanup = [&]() {
+    if (cnt) cudaFree(cnt);
+    if (Ap) cudaFree(Ap);
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+  };
+  if (cudaMalloc(&cnt, sizeof(int32_t) * M) != cudaSuccess || cudaMalloc(&Ap, sizeof(uint16_t) * M * K) != cudaSuccess ||
+      cudaMalloc(&rmap, sizeof(int32_t) * M) != cudaSuccess) {
+    cudaGetLastError();
+    if (rmap) cudaFree(rmap);
+    cleanup();
+    return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "reorder: row clustering buffers");
+  }
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  cudaEventRecord(e0, stream);
+  k_rownnz<<<(unsigned)M, 256, 0, stream>>>(dA, K, cnt);
+  cudaError_t e = cudaMemcpyAsync(hc.data(), cnt, sizeof(int32_t) * M, cudaMemcpyDeviceToHost, stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+  if (e != cudaSuccess) {
+    cudaFree(rmap);
+    cleanup();
+    return cuda_status(e, "reorder: row nonzero counts");
+  }
+  {  // stable counting sort by descending count
+    std::vector<int64_t> start(K + 2, 0);
+    for (int64_t r = 0; r < M; ++r) ++start[K - hc[r] + 1];
+    for (int64_t c = 1; c <= K + 1; ++c) start[c] += start[c - 1];
+    for (int64_t r = 0; r < M; ++r) hmap[start[K - hc[r]]++] = (int32_t)r;
+  }
+  e = cudaMemcpyAsync(rmap, hmap.data(), sizeof(int32_t) * M, cudaMemcpyHostToDevice, stream);
+  if (e == cudaSuccess) {
+    k_permute_rows<<<(unsigned)M, 256, 0, stream>>>(dA, K, rmap, Ap);
+    e = cudaGetLastError();
+  }
+  if (e == cudaSuccess) e = cudaEventRecord(e1, stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+  if (e != cudaSuccess) {
+    cudaFree(rmap);
+    cleanup();
+    return cuda_status(e, "reorder: row clustering");
+  }
+  cudaEventElapsedTime(&ms, e0, e1);
+  st = build_format_rows(Ap, M, K, v, P, mode, stream, f);
+  cleanup();
+  if (st != JIGSAW_SUCCESS) {
+    cudaFree(rmap);
+    return st;
+  }
+  f->row_order = JIGSAW_ROWS_CLUSTERED;
+  f->d_rowmap = rmap;
+  f->allocs.push_back(rmap);
+  f->reorder_ms += ms;
+  f->device_bytes += sizeof(int32_t) * M;
+  return JIGSAW_SUCCESS;
+}
+
+static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
+                                         cudaStream_t stream, Format* f) {
   std::vector<void*> scratch;
   int dev = 0;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;

@@ -145,6 +145,7 @@ struct Problem {
   int unit0;  // first global work unit of this problem
   int pin0;   // offset of this problem's panels in ParamsT::pin (if use_pin)
   int c32;    // 1: C is fp32 (jigsaw_options_t.c_dtype), else fp16
+  const int32_t* rowmap;  // row-clustered panels: C row of panel row r (nullptr: identity)
 };
 // Kernel parameters: a problem table and the panel table, kept in parameter space
 // (read with LDC, no dependent global load at kernel start).  Two sizes: a
@@ -231,6 +232,7 @@ struct Work {
   const __half* B;
   void* C;
   int c32;
+  const int32_t* rowmap;
   int64_t M, N, K;
   int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
   int piece, npieces, pslot;  // split-K piece of a grouped launch (npieces = 1: whole unit)
@@ -270,6 +272,7 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
       w.B = prm.pr[0].B;
       w.C = prm.pr[0].C;
       w.c32 = prm.pr[0].c32;
+      w.rowmap = prm.pr[0].rowmap;
       w.M = prm.pr[0].M;
       w.N = prm.pr[0].N;
       w.K = prm.pr[0].K;
@@ -314,6 +317,7 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.B = prm.pr[i].B;
   w.C = prm.pr[i].C;
   w.c32 = prm.pr[i].c32;
+  w.rowmap = prm.pr[i].rowmap;
   w.M = prm.pr[i].M;
   w.N = prm.pr[i].N;
   w.K = prm.pr[i].K;
@@ -934,6 +938,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it % C_::kAccBufs;
       const int ncols = wk.ncols;                        // C columns of this unit
+      // C row of this lane's panel row (row-clustered panels scatter rows back)
+      int64_t crow = wk.row0 + q * 32 + lane;
+      if (wk.rowmap && crow < M) crow = wk.rowmap[crow];
       if (has_acc) {
         mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
         tc_fence_after();
@@ -1036,10 +1043,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
               const int rr = 8 * i + (lane >> 2), c = lane & 3;
-              const int64_t grow = wk.row0 + q * 32 + rr;
+              const int64_t lrow = wk.row0 + q * 32 + rr;
+              const int64_t grow = wk.rowmap ? __shfl_sync(kFullMask, crow, rr) : lrow;
               const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
               const int col = n0 + ucol(c0 / 32) + 8 * c;
-              if (grow < M && col < N) *reinterpret_cast<uint4*>(static_cast<__half*>(Cm) + grow * N + col) = pk;
+              if (lrow < M && col < N) *reinterpret_cast<uint4*>(static_cast<__half*>(Cm) + grow * N + col) = pk;
             }
             __syncwarp();
           } else {
@@ -1054,10 +1062,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 #pragma unroll
               for (int i = 0; i < 4; ++i) {
                 const int rr = 8 * i + (lane >> 2), c = lane & 3;
-                const int64_t grow = wk.row0 + q * 32 + rr;
+                const int64_t lrow = wk.row0 + q * 32 + rr;
+                const int64_t grow = wk.rowmap ? __shfl_sync(kFullMask, crow, rr) : lrow;
                 const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
                 const int col = n0 + ucol(c0 / 32) + 16 * h + 4 * c;
-                if (grow < M && col < N) *reinterpret_cast<uint4*>(static_cast<float*>(Cm) + grow * N + col) = pk;
+                if (lrow < M && col < N) *reinterpret_cast<uint4*>(static_cast<float*>(Cm) + grow * N + col) = pk;
               }
               __syncwarp();
             }
@@ -1122,9 +1131,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             acc[0] += x.x; acc[1] += x.y; acc[2] += x.z; acc[3] += x.w;
             acc[4] += y.x; acc[5] += y.y; acc[6] += y.z; acc[7] += y.w;
           }
-          const int64_t row = (int64_t)p * 128 + rank * rpo + i;
+          const int64_t lrow = (int64_t)p * 128 + rank * rpo + i;
           const int64_t colg = n0 + c8 * 8;
-          if (row < M && colg < N) {
+          if (lrow < M && colg < N) {
+            const int64_t row = wk.rowmap ? (int64_t)wk.rowmap[lrow] : lrow;
             if (c32) {
               float4* dst = reinterpret_cast<float4*>(static_cast<float*>(Cm) + row * N + colg);
               dst[0] = make_float4(acc[0], acc[1], acc[2], acc[3]);
@@ -1358,6 +1368,7 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
   P.B = reinterpret_cast<const __half*>(dB);
   P.C = dC;
   P.c32 = f.c_dtype == JIGSAW_C_F32 ? 1 : 0;
+  P.rowmap = f.d_rowmap;
   P.M = f.M;
   P.N = N;
   P.K = f.K;

@@ -722,3 +722,41 @@ def test_host_threads_concurrent_calls():
     for t in range(4):
         for a, b, c in zip(mats, Bs, results[t]):
             spmm_check(c, a, b)
+
+
+# ---------------------------------------------------------------- row-clustered panels (f2)
+@pytest.mark.parametrize("M,K,v,s,kind,P,mode,ov", [
+    (512, 2048, 4, 0.9, "skewed", 128, 0, {}),                 # grouped path (C2 shape)
+    (2048, 512, 8, 0.8, "skewed", 128, 0, {}),
+    (600, 300, 4, 0.85, "skewed", 128, 0, dict(split_k=2)),      # split-K cluster, ragged M/K
+    (520, 256, 8, 0.9, "uniform", 256, 0, {}),                   # CTA pairs, ragged last pair panel
+    (384, 640, 4, 0.6, "skewed", 128, 1, {}),                    # DENSE residual mode
+    (256, 200, 2, 0.9, "skewed", 128, 0, dict(tile_n=32, split_k=1)),
+])
+def test_row_clustered_panels(M, K, v, s, kind, P, mode, ov, override):
+    """jigsaw_options_t.row_order = JIGSAW_ROWS_CLUSTERED: the GPU
+    row order equals oracle.row_cluster, the format is bit-exact vs CR1 of A[order],
+    and C -- scattered back to A's row order by the epilogue -- matches the oracle
+    product of the UNPERMUTED A (fp16 and fp32 C; integers bit-exact)."""
+    A = synth.vector_sparse(M, K, v, s, 77, kind=kind)
+    A[3] = 0                                                    # an all-zero row sorts last
+    B = synth.dense_b(K, 136, 77)
+    override(**ov)
+    h = jig.reorder(_dev(A), v, panel_rows=P, residual_mode=mode, row_order=jig.ROWS_CLUSTERED)
+    assert h.info()["row_order"] == jig.ROWS_CLUSTERED
+    g = h.export()
+    ref = oracle.reorder(A, P=P, mode=mode, row_order=1)
+    assert np.array_equal(g["rowmap"], ref.rowmap)
+    assert_format_equal(g, ref)
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    spmm_check(C, A, B)
+    Ai = synth.vector_sparse(M, K, v, s, 78, kind="int")
+    Bi = synth.dense_b(K, 136, 78, kind="int")
+    hi = jig.reorder(_dev(Ai), v, panel_rows=P, residual_mode=mode, row_order=jig.ROWS_CLUSTERED,
+                     c_dtype=jig.C_F32)
+    Ci = _host(hi.spmm(_dev(Bi)))
+    torch.cuda.synchronize()
+    int_exact(Ci, Ai, Bi)
+    h0 = jig.reorder(_dev(A), v, panel_rows=P, residual_mode=mode)
+    assert np.array_equal(h0.export()["rowmap"], np.arange(M))     # identity for the given order
