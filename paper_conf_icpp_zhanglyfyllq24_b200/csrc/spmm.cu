@@ -938,9 +938,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it % C_::kAccBufs;
       const int ncols = wk.ncols;                        // C columns of this unit
-      // C row of this lane's panel row (row-clustered panels scatter rows back)
-      int64_t crow = wk.row0 + q * 32 + lane;
-      if (wk.rowmap && crow < M) crow = wk.rowmap[crow];
       if (has_acc) {
         mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
         tc_fence_after();
@@ -962,6 +959,21 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       if constexpr (!kSplit) {
         const uint32_t stg = smem_u32(sC + q * (32 * 64));
         bool write_c = true;
+        // C rows of the 4 rows this lane stores (rr = 8i + lane / 4 of the warp's
+        // 32): row-clustered panels scatter panel row r to C row rowmap[r]; once
+        // per unit, outside the store loop (M < 2^31 by validation)
+        int64_t srow[4];
+        {
+          const int64_t prow = wk.row0 + q * 32 + lane;
+          int crow = (int)prow;
+          if (wk.rowmap && prow < M) crow = wk.rowmap[prow];
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const int64_t lrow = wk.row0 + q * 32 + 8 * i + (lane >> 2);
+            const int mrow = __shfl_sync(kFullMask, crow, 8 * i + (lane >> 2));
+            srow[i] = lrow < M ? (wk.rowmap ? (int64_t)mrow : lrow) : -1;
+          }
+        }
         const int npc = wk.npieces;
         if (npc > 1) {
           // split-K piece: publish the fp32 partial tile, count the pieces done;
@@ -1043,11 +1055,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
               const int rr = 8 * i + (lane >> 2), c = lane & 3;
-              const int64_t lrow = wk.row0 + q * 32 + rr;
-              const int64_t grow = wk.rowmap ? __shfl_sync(kFullMask, crow, rr) : lrow;
               const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
               const int col = n0 + ucol(c0 / 32) + 8 * c;
-              if (lrow < M && col < N) *reinterpret_cast<uint4*>(static_cast<__half*>(Cm) + grow * N + col) = pk;
+              if (srow[i] >= 0 && col < N) *reinterpret_cast<uint4*>(static_cast<__half*>(Cm) + srow[i] * N + col) = pk;
             }
             __syncwarp();
           } else {
@@ -1062,11 +1072,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
 #pragma unroll
               for (int i = 0; i < 4; ++i) {
                 const int rr = 8 * i + (lane >> 2), c = lane & 3;
-                const int64_t lrow = wk.row0 + q * 32 + rr;
-                const int64_t grow = wk.rowmap ? __shfl_sync(kFullMask, crow, rr) : lrow;
                 const uint4 pk = ld_shared_v4u(stg + rr * 64 + ((c ^ ((rr >> 1) & 3)) << 4));
                 const int col = n0 + ucol(c0 / 32) + 16 * h + 4 * c;
-                if (lrow < M && col < N) *reinterpret_cast<uint4*>(static_cast<float*>(Cm) + grow * N + col) = pk;
+                if (srow[i] >= 0 && col < N) *reinterpret_cast<uint4*>(static_cast<float*>(Cm) + srow[i] * N + col) = pk;
               }
               __syncwarp();
             }

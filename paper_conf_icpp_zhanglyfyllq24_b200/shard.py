@@ -75,10 +75,12 @@ def format_hash(arrays: dict) -> int:
     """64-bit hash (BLAKE2b) of a canonical format (jigsaw_export_format arrays,
     fixed key order): ranks that rebuilt the replicated A must agree."""
     import hashlib
+
+    import numpy as np
     h = hashlib.blake2b(digest_size=8)
     for k in sorted(arrays):
         h.update(k.encode())
-        h.update(memoryview(arrays[k]).cast("B"))
+        h.update(np.ascontiguousarray(arrays[k]).tobytes())
     return int.from_bytes(h.digest(), "little") & 0x7FFFFFFFFFFFFFFF
 
 

@@ -48,7 +48,22 @@ def _worker(rank, world, port, q):
         dist.all_gather(hs, hsh)
         ok_hash = all(int(h) == int(hsh) for h in hs)
         mx = shard.max_over_ranks(float(rank + 1), dist=dist, device="cpu")
-        q.put((rank, ok_cols, ok_hash, mx))
+        # the helpers bench.py uses after the timed region (NCCL on GPUs): padded
+        # shard gather, format hash, sampled-row check against a dense product
+        Ct = torch.from_numpy(Cs.astype(np.float32))
+        full_t = shard.gather_column_shards(Ct, n0, n1, N, dist, world)
+        ok_gather = np.array_equal(full_t.numpy().astype(np.float64), full.astype(np.float32).astype(np.float64))
+        fh = shard.format_hash({"T": f.T, "meta": f.meta, "col_idx": f.col_idx})
+        hs2 = [torch.zeros(1, dtype=torch.int64) for _ in range(world)]
+        dist.all_gather(hs2, torch.tensor([fh], dtype=torch.int64))
+        ok_fh = len({int(h) for h in hs2}) == 1
+        Ad = torch.from_numpy(A.view(np.float16).astype(np.float32))
+        Bd = torch.from_numpy(B.view(np.float16).astype(np.float32))
+        excess = shard.check_against_dense(full_t, Ad, Bd, torch.arange(0, M, 7))
+        bad = full_t.clone()
+        bad[5, 3] += 1.0
+        excess_bad = shard.check_against_dense(bad, Ad, Bd, torch.tensor([5]))
+        q.put((rank, ok_cols and ok_gather and ok_fh and excess <= 0 and excess_bad > 0, ok_hash, mx))
     finally:
         dist.destroy_process_group()
 

@@ -1,8 +1,6 @@
-P=tools/probe_c2_cfg.py
 for r in 1 2; do
-python abold/probe_old.py c2
-python $P c2 0 0 new_c2
-python abold/probe_old.py c4
-python $P c4 0 0 new_c4
+JIGSAW_LIB_AB=abprev/paper_conf_icpp_zhanglyfyllq24_b200/libjigsaw.so python tools/probe_c2_cfg.py c2 0 0 prevlib_c2
+JIGSAW_LIB_AB=tools/libjigsaw_v7.so python tools/probe_c2_cfg.py c2 0 0 v7_c2
+JIGSAW_LIB_AB=abprev/paper_conf_icpp_zhanglyfyllq24_b200/libjigsaw.so python tools/probe_c2_cfg.py c4 0 0 prevlib_c4
+JIGSAW_LIB_AB=tools/libjigsaw_v7.so python tools/probe_c2_cfg.py c4 0 0 v7_c4
 done
-nvidia-smi --query-gpu=clocks.sm,clocks.max.sm,power.draw,temperature.gpu --format=csv
