@@ -317,23 +317,6 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint32_t rbar) {
 __device__ __forceinline__ void mbar_arrive_cluster_relaxed(uint32_t rbar) {
   asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(rbar) : "memory");
 }
-// Non-blocking probe (acquire, cluster scope) of phase `parity` of a local
-// mbarrier that remote CTAs arrive on: true once that phase has completed.
-__device__ __forceinline__ bool mbar_test_cluster(uint64_t* bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred P1;\n\t"
-      "mbarrier.test_wait.parity.acquire.cluster.shared::cta.b64 P1, [%1], %2;\n\t"
-      "selp.u32 %0, 1, 0, P1;\n\t}"
-      : "=r"(ok)
-      : "r"(smem_u32(bar)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-// 32-bit store to the shared memory of a CTA of the cluster (shared::cluster address).
-__device__ __forceinline__ void st_cluster_s32(uint32_t raddr, int32_t v) {
-  asm volatile("st.shared::cluster.b32 [%0], %1;" ::"r"(raddr), "r"(v) : "memory");
-}
 // Wait (acquire, cluster scope) for phase `parity` of a local mbarrier that remote CTAs arrive on.
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
   asm volatile(

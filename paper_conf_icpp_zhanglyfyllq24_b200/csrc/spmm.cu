@@ -126,7 +126,7 @@ struct Cfg {
   static constexpr int kGS = (2 * kStages + kBGroups - 1) / kBGroups * kBGroups;
   static constexpr int kGAhead = kStages;
   static constexpr size_t kSmem =
-      1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 1024;
+      1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 512;
   static_assert(kSmem <= 232448, "shared memory budget");
 };
 
@@ -369,12 +369,6 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
 // tag launches instead: CUDA-graph replays reuse the value fixed at
 // instantiation, tools/gridid_probe.cu.)
 constexpr int kSD = 4;  // unit-ring depth
-// CTA pairs under the dynamic scheduler: the even CTA takes the tickets and
-// forwards every unit id, in order, through a kMB-deep mailbox in the odd CTA's
-// shared memory (remote store + release arrive on the odd CTA's mfull; the odd
-// CTA frees the slot with a release arrive on the even CTA's mempty), so both
-// CTAs of the pair run the same unit sequence.
-constexpr int kMB = 16;
 
 // Unit-ring consumer: the A/E producer publishes each unit id (or -1 = done)
 // into a kSD-deep ring in shared memory; every consumer warp reads the same
@@ -422,11 +416,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   uint64_t* rfull = recv_full + 1;   // unit ring (dynamic scheduler)
   uint64_t* rempty = rfull + kSD;
   uint64_t* pfull = rempty + kSD;    // kPair, even CTA: the odd CTA's stage has landed
-  uint64_t* mfull = pfull + C_::kStages;  // kPair + dynamic, odd CTA: mailbox slot written by the even CTA
-  uint64_t* mempty = mfull + kMB;         // kPair + dynamic, even CTA: mailbox slot read by the odd CTA
-  volatile int* ring = reinterpret_cast<volatile int*>(mempty + kMB);
-  int* mbox = const_cast<int*>(ring) + kSD;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(mbox + kMB);
+  volatile int* ring = reinterpret_cast<volatile int*>(pfull + C_::kStages);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pfull + C_::kStages) + kSD;
   const uint32_t s_last = smem_u32(tmem_slot + 1);  // split piece: this CTA reduces (int flag)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -435,7 +426,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   const int CS = kPair ? 2 : S;  // CTAs per cluster
   const uint32_t rank = (kSplit || kPair) ? cluster_ctarank() : 0;
   const int cluster_id = blockIdx.x / CS, nclusters = gridDim.x / CS;
-  const bool dyn = !kSplit && prm.dyn;
+  const bool dyn = !kSplit && !kPair && prm.dyn;  // CTA pairs always run a static plan
   if (threadIdx.x == 0 && prm.trace && blockIdx.x < kTraceCTAs) {
     g_trace[blockIdx.x * kTraceSlots + 15] = gtimer();
     g_trace[blockIdx.x * kTraceSlots + 14] = smid();
@@ -467,7 +458,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   // are contiguous in shared memory: full, empty, gfull, gempty, tfull, tempty,
   // recv_full, rfull, rempty, pfull.
   if (warp == 0) {
-    constexpr int nb = 3 * C_::kStages + 2 * C_::kGS + 7 + 2 * kSD + 2 * kMB;
+    constexpr int nb = 3 * C_::kStages + 2 * C_::kGS + 7 + 2 * kSD;
     for (int i = lane; i < nb; i += 32) {
       int k = i;
       uint32_t cnt;
@@ -479,8 +470,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       else if ((k -= 3) < 3) cnt = kPair ? 8 : 4;          // tempty: epilogue warps (of both CTAs of a pair)
       else if ((k -= 3) < 1) cnt = 1;                      // recv_full
       else if ((k -= 1) < kSD) cnt = 1;                    // rfull
-      else if ((k -= kSD) < kSD) cnt = kBProdWarps + 1 + 4;  // rempty: B-producer warps + MMA / relay + epilogue warps
-      else cnt = 1;                                        // pfull, mfull, mempty
+      else if ((k -= kSD) < kSD) cnt = kBProdWarps + 1 + 4;  // rempty: B-producer warps + MMA + epilogue warps
+      else cnt = 1;                                        // pfull
       mbar_init(full + i, cnt);
     }
     fence_barrier_init();
@@ -559,12 +550,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     }
   }
 
-  if constexpr (kPair) {  // the unit mailbox is remote: the peer's barriers must be initialised
-    if (warp == 0 && dyn) {
-      cluster_wait();
-      cl_waited = true;
-    }
-  }
   if (warp == 0) {
     // ------------------------------------------------------------ A / E producer
     if (lane == 0) {
@@ -583,38 +568,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       constexpr int kQ = 16;
       int uq[kQ];
       int qn = 0, mq = 0, next_un = cluster_id;
-      // Queues the CTA's next unit (-1 = none left).  Pairs under the dynamic
-      // scheduler: the even CTA forwards each unit to the odd CTA's mailbox, the
-      // odd CTA reads it from there.  Non-blocking calls (the gather cursor) give
-      // up when the mailbox slot is not ready, so only the A/E cursor -- which
-      // has issued every k-block of the units before -- ever waits on the peer.
-      auto fetch = [&](bool block) -> bool {
-        int un;
-        if (kPair && dyn) {
-          const int slot = qn % kMB;
-          const uint32_t ph = (uint32_t)(qn / kMB) & 1u;
-          if (rank == 0) {
-            if (!block && !mbar_test_cluster(&mempty[slot], ph ^ 1)) return false;
-            mbar_wait_cluster(&mempty[slot], ph ^ 1);
-            un = next_un < prm.nunits ? next_un : -1;
-            // forward first: the release arrive would otherwise wait for the
-            // ticket atomic below (the next ticket is only needed at the next fetch)
-            st_cluster_s32(mapa_shared(smem_u32(mbox + slot), 1), un);
-            mbar_arrive_cluster(mapa_shared(smem_u32(&mfull[slot]), 1));
-            if (un >= 0) next_un = nclusters + atomicAdd(ctr, 1);
-          } else {
-            if (!block && !mbar_test_cluster(&mfull[slot], ph)) return false;
-            mbar_wait_cluster(&mfull[slot], ph);
-            un = ld_shared_s32(smem_u32(mbox + slot));
-            mbar_arrive_cluster(mapa_shared(smem_u32(&mempty[slot]), 0));
-          }
-        } else {
-          un = next_un < prm.nunits ? next_un : -1;
-          if (un >= 0) next_un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : un + nclusters;
-        }
+      // Queues the CTA's next unit (-1 = none left); the dynamic scheduler's
+      // ticket for the one after is taken here, its value needed only then
+      auto fetch = [&]() {
+        const int un = next_un < prm.nunits ? next_un : -1;
+        if (un >= 0) next_un = dyn ? (int)gridDim.x + atomicAdd(ctr, 1) : un + nclusters;
         uq[qn % kQ] = un;
         ++qn;
-        return true;
       };
       // gather-list cursor
       int gq = 0, ghint = 0, gkb = 0, gkbe = 0, gslot = nG0 % C_::kGS;
@@ -623,7 +583,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       bool gend = false;
       Work gwk = w0;
       if (nG0 > 0) {  // the gather cursor continues inside the first unit
-        fetch(true);
+        fetch();
         gq = 1;
         gkb = w0.kb_lo + nG0;
         gkbe = w0.kb_hi;
@@ -633,7 +593,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (gkb >= gkbe) {  // next unit with work
             if (gq == qn) {
               if (qn - mq >= kQ) return;  // queue full: the A/E cursor catches up first
-              if (!fetch(false)) return;  // pair mailbox not ready: the A/E cursor goes on
+              fetch();
             }
             const int u = uq[gq % kQ];
             if (u < 0) {
@@ -658,7 +618,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       };
       int64_t mi = nA0;  // k-blocks issued by the A/E cursor
       for (;;) {
-        if (mq == qn) fetch(true);
+        if (mq == qn) fetch();
         if (mq == 0) JIG_TRACE(16);
         const int u = uq[mq % kQ];
         ++mq;
@@ -698,9 +658,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
         }
       }
-      if (dyn && rank == 0) {  // the last CTA to stop fetching resets the ticket for the next launch
+      if (dyn) {  // the last CTA to stop fetching resets the ticket for the next launch
         __threadfence();
-        if (atomicAdd(ctr + 1, 1) == nclusters - 1) {
+        if (atomicAdd(ctr + 1, 1) == (int)gridDim.x - 1) {
           atomicExch(ctr, 0);
           atomicExch(ctr + 1, 0);
         }
@@ -798,13 +758,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     // The even CTA issues the pair's MMAs; it may read this CTA's stage only once
     // this CTA's A/E bulk copies and B cp.async have landed: relay full -> pfull.
     if (lane == 0) {
-      int stage = 0, hint = 0, nrel = 0, rslot = 0;
-      uint32_t phase = 0, rph = 0;
+      int stage = 0, hint = 0, nrel = 0;
+      uint32_t phase = 0;
       const uint32_t rpfull = mapa_shared(smem_u32(pfull), 0);
-      for (int us = cluster_id;; us += nclusters) {
-        const int u = dyn ? ring_take(ring, rfull, rempty, rslot, rph, false, lane) : (us < prm.nunits ? us : -1);
-        if (u < 0) break;
-        const Work wk = decode_unit<NT, kPair, Prm>(prm, u, rank, S, hint);
+      for (int us = cluster_id; us < prm.nunits; us += nclusters) {
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
         if (!wk.valid) continue;
         for (int kb = wk.kb_lo; kb < wk.kb_hi; ++kb) {
           mbar_wait(&full[stage], phase);
@@ -1202,14 +1160,14 @@ struct Knobs {
   bool pdl = true, trace = false;
   int dbg = 0;               // JIGSAW_DBG (timing only, results invalid)
   bool no_prefetch = false;  // JIGSAW_NO_PREFETCH: no per-unit metadata prefetch into L2
-  bool static_sched = false; // JIGSAW_STATIC_SCHEDULE: no dynamic tile scheduler
+  bool dyn_sched = false;    // JIGSAW_DYN_SCHEDULE: dynamic tile scheduler for grouped launches
+                             // (measured 4-12 % slower than the static LPT plan, profiles/r02x)
   int unit_cost = -1;        // JIGSAW_UNIT_COST: per-unit cost in k-block equivalents
   bool sched_loc = false;    // JIGSAW_SCHED=loc: locality order, no cost sort, no pieces
   bool debug_sched = false;  // JIGSAW_DEBUG_SCHED: print the pair schedule balance
   int64_t group_bpf = 0;     // JIGSAW_GROUP_BPF (MB): L2 prefetch of all B's of a grouped launch
   bool bpf = false;          // JIGSAW_BPF: L2 prefetch of B for single products
   bool no_ctab = false;      // JIGSAW_NO_CTAB: no host-decoded first units
-  bool pair_dyn = false;     // JIGSAW_PAIR_DYN: dynamic scheduler for CTA pairs (measured slower than static LPT)
   int split_pct = 125;       // JIGSAW_SPLIT_PCT: split a unit into pieces above this % of the per-slot load
 };
 const Knobs& knobs() {
@@ -1221,14 +1179,13 @@ const Knobs& knobs() {
 #if JIG_DEV
     r.dbg = env("JIGSAW_DBG") ? atoi(env("JIGSAW_DBG")) : 0;
     r.no_prefetch = env("JIGSAW_NO_PREFETCH") != nullptr;
-    r.static_sched = env("JIGSAW_STATIC_SCHEDULE") != nullptr;
+    r.dyn_sched = env("JIGSAW_DYN_SCHEDULE") != nullptr;
     r.unit_cost = env("JIGSAW_UNIT_COST") ? atoi(env("JIGSAW_UNIT_COST")) : -1;
     r.sched_loc = env("JIGSAW_SCHED") && std::string(env("JIGSAW_SCHED")) == "loc";
     r.debug_sched = env("JIGSAW_DEBUG_SCHED") != nullptr;
     r.group_bpf = env("JIGSAW_GROUP_BPF") ? atoll(env("JIGSAW_GROUP_BPF")) : 0;
     r.bpf = env("JIGSAW_BPF") != nullptr;
     r.no_ctab = env("JIGSAW_NO_CTAB") != nullptr;
-    r.pair_dyn = env("JIGSAW_PAIR_DYN") != nullptr;
     r.split_pct = env("JIGSAW_SPLIT_PCT") ? atoi(env("JIGSAW_SPLIT_PCT")) : 125;
 #endif
     return r;
@@ -1480,11 +1437,13 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   }
   prm.nunits = npieces_total >= 0 ? npieces_total : u;
   // (a CTA per unit needs no scheduler: its one unit is known at kernel start)
-  // CTA pairs: static greedy-LPT schedule (the dynamic one, with the even CTA
-  // forwarding tickets through a mailbox, measured 8-20 % slower on C2 / C4:
-  // units fetched ahead of time unbalance the tail); single CTAs: dynamic
-  prm.dyn = (S == 1 && (pair ? grid / 2 : grid) < prm.nunits && !knobs().static_sched &&
-             (!pair || knobs().pair_dyn)) ? 1 : 0;
+  // Grouped launches run the host's static greedy-LPT plan (prm.use_ulist): the
+  // dynamic tile scheduler measured 4-12 % slower on C2 / C3 / C5a (units taken
+  // ahead of time unbalance the tail; profiles/r02w, r02x) and is a developer
+  // option there; a CTA-pair variant (the even CTA forwarding tickets through a
+  // mailbox) measured 8-20 % slower on C2 / C4 and was removed (profiles/r02e).
+  // Single products whose units outnumber the CTAs (no host plan) use it.
+  prm.dyn = (S == 1 && !pair && grid < prm.nunits && (!prm.use_ulist || knobs().dyn_sched)) ? 1 : 0;
   Workspace w;
   if (prm.dyn || pslots > 0) {
     jigsaw_status_t st = acquire_workspace(dev, kWsHead + (size_t)pslots * tile_bytes, s, &w);
@@ -1627,12 +1586,12 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
     const int64_t units = NT == 256 ? u256 : NT == 128 ? u128 : u64;
     const int slots_max = pair ? sms / 2 : sms;                  // CTAs or CTA pairs
     int slots = (int)std::min<int64_t>(units, slots_max);
-    // Schedule: units sorted by cost (k-blocks of their panel), longest first;
-    // pair launches deal them to the pairs in snake order (slot c takes positions
-    // c, c + slots, ...), single-CTA launches hand them out through the dynamic
-    // scheduler in this order (LPT-like either way).  A unit much longer than the
-    // per-slot average is split into up to 8 k-range pieces (split-K inside the
-    // persistent launch) so one long panel does not set the makespan.
+    // Schedule: units sorted by cost (k-blocks of their panel + a fixed per-unit
+    // cost), longest first, dealt by greedy LPT to the least loaded CTA (or CTA
+    // pair); every slot runs its own queue, known at launch.  A unit much longer
+    // than the per-slot average is cut into column slices (or, on request,
+    // k-range pieces reduced through the workspace) so one long panel does not
+    // set the makespan.
     prm.use_ulist = 0;
     int npieces_total = -1, pslots = 0, nsplit_items = 0;
     const size_t tile = (size_t)128 * NT * sizeof(float) * (pair ? 2 : 1);
@@ -1642,12 +1601,13 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
       us.clear();
       int64_t total = 0;
       // fixed per-unit cost in k-block equivalents (accumulator drain, pipeline
-      // refill).  Pairs with NT = 256 have a single accumulator buffer, so a
+      // refill): 2 for single CTAs (C2 static plan: 1 -> 32.4, 2 -> 31.8 us,
+      // profiles/r02w); pairs with NT = 256 have a single accumulator buffer, so a
       // unit's epilogue is not overlapped with the next unit's mainloop: 4
       // (C2 at P = 256: 41.1 -> 35.3 us; the larger cost also stops the split
       // pieces whose workspace reduction cost more than the balance they bought,
       // profiles/r01w_unit_cost.txt).
-      const int unit_cost = kn.unit_cost >= 0 ? kn.unit_cost : (pair && NT == 256 ? 4 : 1);
+      const int unit_cost = kn.unit_cost >= 0 ? kn.unit_cost : (pair && NT == 256 ? 4 : 2);
       for (int i = 0; i < n; ++i) {
         const Format& f = *fs[i0 + i];
         const int ntn = (int)((Ns[i0 + i] + NT - 1) / NT);
@@ -1710,14 +1670,13 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
                          [](const std::pair<int, uint32_t>& a, const std::pair<int, uint32_t>& b) { return a.first < b.first; });
       const int nslots = (int)std::min<int64_t>(slots_max, (int64_t)order.size());
       npieces_total = (int)order.size();
-      if (!pair || kn.pair_dyn) {
-        // cost order, handed out by the dynamic scheduler (CTA pairs, developer
-        // option: the even CTA takes the tickets and forwards them to its peer)
+      if (kn.dyn_sched && !pair) {
+        // developer option: cost order, handed out by the dynamic scheduler
         for (size_t k = 0; k < order.size(); ++k) prm.ulist[k] = order[k].second;
       } else {
         // static schedule: greedy LPT (each piece, longest first, to the least
-        // loaded pair); pair c runs positions c, c + nslots, ... of the list,
-        // padded with kNoWork where its queue is shorter than the longest
+        // loaded CTA or CTA pair); slot c runs positions c, c + nslots, ... of
+        // the list, padded with kNoWork where its queue is shorter than the longest
         thread_local std::vector<std::vector<uint32_t>> q;
         q.assign(nslots, {});
         std::vector<std::pair<int64_t, int>> heap;  // (load, slot), min-heap

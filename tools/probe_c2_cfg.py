@@ -19,7 +19,7 @@ dev = torch.device("cuda", 0)
 stream = torch.cuda.current_stream()
 flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 b = bench.Batch(name, 0, 1, P, dev, torch, jig)
-jig.set_launch_override(tile_n=nt)
+jig.set_launch_override(tile_n=nt, k_pieces=int(os.environ.get("KPIECES", "0")))
 b.step(jig)
 torch.cuda.synchronize()
 d = jig.last_launch()

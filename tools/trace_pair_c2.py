@@ -24,8 +24,9 @@ def main():
             for i, (M, K, v, s, N) in enumerate(pts)]
     B2 = [dev(b) for _, b, _ in mats]
     C2 = [torch.empty((a.shape[0], b.shape[1]), dtype=torch.float16, device="cuda") for a, b, _ in mats]
+    kp = int(os.environ.get("KPIECES", "0"))
     for P, nt in [(128, 0), (256, 256)]:
-        jig.set_launch_override(tile_n=nt)
+        jig.set_launch_override(tile_n=nt, k_pieces=kp)
         hs = [jig.reorder(dev(a), v, panel_rows=P) for a, _, v in mats]
         for rep in range(3):
             flush.zero_()
