@@ -332,41 +332,55 @@ class Batch:
             h.free()
 
 
-def timed_steps(fn, steps, warmup, flush, stream, torch, dist=None, world=1, dev_index=0):
-    """fn captured in a CUDA graph; W warm-up replays, then K replays each preceded
-    by an L2 flush (outside the events), CUDA events on `stream` around each
-    replay, barrier + synchronize on both sides, clocks sampled during the timed
-    region.  Returns (ms per step, max over ranks; clocks)."""
+def timed_steps(fn, steps, warmup, flush, stream, torch, dist=None, world=1, dev_index=0, outside=None):
+    """fn captured in a CUDA graph together with two timing events recorded as
+    graph nodes immediately before and after it (external event nodes: the
+    measured interval is the step's own device work, not the graph launch);
+    W warm-up replays, then K replays each preceded by an L2 flush (outside the
+    events), barrier + synchronize on both sides of the timed loop, clocks
+    sampled during it.  Returns (ms per step, max over ranks; clocks).  If
+    `outside` is a dict, it also receives the same steps timed by events around
+    the whole graph replay (graph launch latency included)."""
     fn()
     torch.cuda.synchronize()
+    e_in0 = torch.cuda.Event(enable_timing=True, external=True)
+    e_in1 = torch.cuda.Event(enable_timing=True, external=True)
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g):
+        e_in0.record()
         fn()
+        e_in1.record()
     torch.cuda.synchronize()
     for _ in range(max(3, warmup)):
         flush.zero_()
         g.replay()
     torch.cuda.synchronize()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
     sampler = ClockSampler(dev_index)
     sampler.start()
     time.sleep(0.15)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    t_in, t_out = [], []
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for k in range(steps):
         flush.zero_()                     # L2 flush, outside the timed events
-        evs[k][0].record(stream)
+        e0.record(stream)
         g.replay()
-        evs[k][1].record(stream)
+        e1.record(stream)
+        e1.synchronize()                  # the graph's event nodes are re-recorded by the next replay
+        t_in.append(e_in0.elapsed_time(e_in1))
+        t_out.append(e0.elapsed_time(e1))
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
-    total_ms = sum(a.elapsed_time(b) for a, b in evs)
     from paper_conf_icpp_zhanglyfyllq24_b200 import shard
-    total_ms = shard.max_over_ranks(total_ms, dist=dist if world > 1 else None,
-                                    device=torch.device("cuda", dev_index))
+    dv = torch.device("cuda", dev_index)
+    total_ms = shard.max_over_ranks(sum(t_in), dist=dist if world > 1 else None, device=dv)
+    if outside is not None:
+        outside["ms_per_step"] = shard.max_over_ranks(sum(t_out), dist=dist if world > 1 else None,
+                                                      device=dv) / steps
     del g
     return total_ms / steps, clocks
 
@@ -463,7 +477,8 @@ def cublas_compare(b: Batch, flush, stream, torch, jig, jig_step_ms, steps, warm
     out["batched_step_ms_16F_32F"] = [batched["16F"], batched["32F"]]
     out["speedup_vs_batched_cublas"] = batched[best] / jig_step_ms
     out["batched_how"] = ("one cublasGemmStridedBatchedEx per (M, K, N) group of the batch, best of "
-                          "CUBLAS_COMPUTE_16F / 32F, graph-replayed and timed exactly like the jigsaw step")
+                          "CUBLAS_COMPUTE_16F / 32F, graph-replayed and timed exactly like the jigsaw step "
+                          "(event nodes around the step inside its graph, L2 flushed before)")
     if not per_matrix:
         return out
     detail, sp = [], {}
@@ -555,8 +570,9 @@ def main():
     b.step(jig)
     torch.cuda.synchronize()
     launches = jig.last_launch()["launches"]
+    outside = {}
     ms, clocks = timed_steps(lambda: b.step(jig), args.steps, args.warmup, flush, stream, torch,
-                             dist=dist_, world=world, dev_index=dev.index or 0)
+                             dist=dist_, world=world, dev_index=dev.index or 0, outside=outside)
     value = total_eff / (ms * 1e-3) / 1e12
     roof = roofline(b, ms / max(1, launches), peaks)
 
@@ -588,6 +604,9 @@ def main():
                    "l2": "flushed (256 MB write) before every timed step",
                    "launch": "step = one jigsaw_spmm_batched call over the batch (one grouped k_spmm launch per "
                              "64 matrices of one panel height), captured in a CUDA graph",
+                   "timing": "CUDA events recorded as nodes of the step's graph around the k_spmm launch "
+                             "(stream of the launch); events around the whole graph replay, graph launch latency "
+                             f"included: {outside.get('ms_per_step', 0) * 1e3:.1f} us per step",
                    "seeds": "synth.SEED_BASE + 1000*rank + index",
                    "format": f"panel_rows={args.panel_rows or 'auto'} (P used: {b.panel_rows_used}), SPTC residual"},
         "roofline": roof,
