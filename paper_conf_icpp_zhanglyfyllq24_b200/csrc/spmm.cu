@@ -100,7 +100,10 @@ struct Cfg {
   // chunk (the MMA with N = 32 reads only those columns of the swizzled atom)
   static constexpr int kChunks = kNTL >= 64 ? kNTL / 64 : 1;
   static constexpr int kStageB = kChunks * kChunkB;
-  static constexpr int kStages = kPair ? (NT == 256 ? 4 : 6) : NT == 256 ? 2 : NT == 128 ? 4 : 5;
+#ifndef JIG_STAGE_DELTA
+#define JIG_STAGE_DELTA 0  // developer: stage-count sensitivity experiments
+#endif
+  static constexpr int kStages = (kPair ? (NT == 256 ? 4 : 6) : NT == 256 ? 2 : NT == 128 ? 4 : 5) + JIG_STAGE_DELTA;
   static constexpr int kAccCols = NT;
   // TMEM (512 columns): double-buffered fp32 accumulators, one for NT = 256
   // (two half-width accumulators issued as N = 128 MMAs measured slower in

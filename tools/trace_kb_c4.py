@@ -1,4 +1,4 @@
-"""Per-k-block timeline (library built with JIGSAW_NVCC_DEFINES=JIG_TRACE_KB_ON=1,
+"""Per-k-block timeline (library built with tools/build_dev.sh "JIG_TRACE_KB_ON=1",
 loaded through JIGSAW_LIB_AB) of CTAs 0/1 on one C4 matrix: the interval between
 successive A/E issues, B issues, stage-full observations and commits shows which
 role paces the pipeline.  Developer tool."""
