@@ -51,6 +51,8 @@ typedef enum {
   JIGSAW_ERROR_INTERNAL = 6       /* a builder invariant failed (bug) */
 } jigsaw_status_t;
 
+#define JIGSAW_PANEL_AUTOTUNE (-1)
+
 /* Residual handling for columns evicted by the reorder retry. */
 typedef enum {
   JIGSAW_RESIDUAL_SPTC = 0, /* paper: evicted columns re-queued into later 2:4 tiles (default) */
@@ -77,14 +79,19 @@ typedef struct {
   int panel_rows;    /* rows per panel (the BLOCK_TILE analogue, R-Q5/R-Q6): 128 (one CTA per
                         panel; the default when opt is NULL), 256 (a CTA pair per panel:
                         tcgen05 cta_group::2, M = 256, each dense B tile staged once per
-                        pair) or 0 = auto (256 when M >= 4096, else 128).  16, 32 and 64
+                        pair), 0 = auto (256 when M >= 4096, else 128) or -1 = autotune
+                        (JIGSAW_PANEL_AUTOTUNE: build both the 128- and the 256-row format,
+                        time one jigsaw_spmm of each on the device with N = autotune_n
+                        columns of B, keep the faster; the timing is part of the reorder's
+                        preprocessing time).  16, 32 and 64
                         (the paper's BLOCK_TILE sizes) build the format for
                         export / statistics only: jigsaw_spmm on such a handle returns
                         JIGSAW_ERROR_UNSUPPORTED (no tcgen05 M below 128 is built) */
   int residual_mode; /* jigsaw_residual_mode_t */
   int c_dtype;       /* jigsaw_c_dtype_t: element type of C for every product with this handle */
   int row_order;     /* jigsaw_row_order_t */
-  int reserved[4];   /* must be zero */
+  int autotune_n;    /* panel_rows = -1: columns of the probe product (0 = 256); else must be 0 */
+  int reserved[3];   /* must be zero */
 } jigsaw_options_t;
 
 /* Statistics of a prepared matrix (jigsaw_get_info). */

@@ -33,6 +33,7 @@ ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_stat
 
 C_F16, C_F32 = 0, 1            # jigsaw_c_dtype_t
 ROWS_GIVEN, ROWS_CLUSTERED = 0, 1   # jigsaw_row_order_t
+PANEL_AUTOTUNE = -1                  # panel_rows: time 128- and 256-row formats, keep the faster
 
 
 class JigsawError(RuntimeError):
@@ -43,7 +44,7 @@ class JigsawError(RuntimeError):
 
 class Options(ctypes.Structure):
     _fields_ = [("panel_rows", ctypes.c_int), ("residual_mode", ctypes.c_int), ("c_dtype", ctypes.c_int),
-                ("row_order", ctypes.c_int), ("reserved", ctypes.c_int * 4)]
+                ("row_order", ctypes.c_int), ("autotune_n", ctypes.c_int), ("reserved", ctypes.c_int * 3)]
 
 
 class Info(ctypes.Structure):
@@ -258,11 +259,13 @@ class Handle:
 
 
 def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: int = C_F16,
-            row_order: int = ROWS_GIVEN, stream=None) -> Handle:
-    """jigsaw_reorder_ex: multi-granularity reorder + format build of A (CUDA fp16 M x K)."""
+            row_order: int = ROWS_GIVEN, autotune_n: int = 0, stream=None) -> Handle:
+    """jigsaw_reorder_ex: multi-granularity reorder + format build of A (CUDA fp16 M x K).
+    panel_rows = PANEL_AUTOTUNE times both panel heights on an autotune_n-column
+    product (0 = 256) and keeps the faster format."""
     _check_fp16_cuda(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode, c_dtype, row_order)
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order, autotune_n)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_ex(ctypes.c_void_p(A.data_ptr()), M, K, v, ctypes.byref(opt),
                                       _stream_ptr(stream), ctypes.byref(out)))

@@ -139,15 +139,18 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
   if (M % v) return set_status(JIGSAW_ERROR_INVALID_VALUE, "M must be a multiple of v");
   if (opt) {
     const int pr = opt->panel_rows;
-    if (!(pr == 0 || pr == 16 || pr == 32 || pr == 64 || pr == kPanelRows || pr == kPairPanelRows))
-      return set_status(JIGSAW_ERROR_INVALID_VALUE, "panel_rows must be 0 (auto), 16, 32, 64, 128 or 256");
+    if (!(pr == 0 || pr == JIGSAW_PANEL_AUTOTUNE || pr == 16 || pr == 32 || pr == 64 || pr == kPanelRows ||
+          pr == kPairPanelRows))
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "panel_rows must be 0 (auto), -1 (autotune), 16, 32, 64, 128 or 256");
+    if (opt->autotune_n < 0 || opt->autotune_n % 8 || (opt->autotune_n && pr != JIGSAW_PANEL_AUTOTUNE))
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "autotune_n must be 0, or a multiple of 8 with panel_rows = -1");
     if (opt->residual_mode != JIGSAW_RESIDUAL_SPTC && opt->residual_mode != JIGSAW_RESIDUAL_DENSE)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown residual_mode");
     if (opt->c_dtype != JIGSAW_C_F16 && opt->c_dtype != JIGSAW_C_F32)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown c_dtype");
     if (opt->row_order != JIGSAW_ROWS_GIVEN && opt->row_order != JIGSAW_ROWS_CLUSTERED)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown row_order");
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < 3; ++i)
       if (opt->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved options must be zero");
   }
   return JIGSAW_SUCCESS;
@@ -167,6 +170,57 @@ jigsaw_status_t validate_spmm(jigsaw_handle_t h, const void* B, int64_t N, const
     return set_status(JIGSAW_ERROR_UNSUPPORTED,
                       "formats with panel_rows < 128 are for analysis (export / statistics); the SpMM needs "
                       "128 or 256 (tcgen05 M)");
+  return JIGSAW_SUCCESS;
+}
+
+// Per-shape panel-height autotune: both formats are built,
+// one jigsaw_spmm of each is timed on the device (zero B of autotune_n columns,
+// best of 3 after a warm-up, CUDA events on the reorder's stream), the faster
+// is kept.  Ties (within 2 %) go to 128-row panels (split-K for small products).
+jigsaw_status_t autotune_panels(const uint16_t* dA, int64_t M, int64_t K, int v, int mode, int row_order, int n,
+                                cudaStream_t st, Format* out) {
+  Format f[2];
+  const int P[2] = {kPanelRows, kPairPanelRows};
+  for (int i = 0; i < 2; ++i) {
+    jigsaw_status_t s = build_format(dA, M, K, v, P[i], mode, row_order, st, &f[i]);
+    if (s != JIGSAW_SUCCESS) {
+      if (i) free_format(&f[0]);
+      return s;
+    }
+  }
+  const int64_t N = n > 0 ? n : 256;
+  void *dB = nullptr, *dC = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  float best[2] = {1e30f, 1e30f};
+  cudaError_t e = cudaMalloc(&dB, (size_t)K * N * 2);
+  if (e == cudaSuccess) e = cudaMalloc(&dC, (size_t)M * N * 4);
+  if (e == cudaSuccess) e = cudaMemsetAsync(dB, 0, (size_t)K * N * 2, st);
+  if (e == cudaSuccess) e = cudaEventCreate(&e0);
+  if (e == cudaSuccess) e = cudaEventCreate(&e1);
+  jigsaw_status_t s = e == cudaSuccess ? JIGSAW_SUCCESS : cuda_status(e, "autotune buffers");
+  for (int i = 0; i < 2 && s == JIGSAW_SUCCESS; ++i)
+    for (int rep = 0; rep < 4 && s == JIGSAW_SUCCESS; ++rep) {
+      cudaEventRecord(e0, st);
+      s = launch_spmm(f[i], dB, N, dC, st);
+      cudaEventRecord(e1, st);
+      if (s == JIGSAW_SUCCESS && (e = cudaEventSynchronize(e1)) != cudaSuccess) s = cuda_status(e, "autotune timing");
+      float ms = 0;
+      if (s == JIGSAW_SUCCESS && rep > 0 && cudaEventElapsedTime(&ms, e0, e1) == cudaSuccess)
+        best[i] = std::min(best[i], ms);
+    }
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (dB) cudaFree(dB);
+  if (dC) cudaFree(dC);
+  if (s != JIGSAW_SUCCESS) {
+    free_format(&f[0]);
+    free_format(&f[1]);
+    return s;
+  }
+  const int keep = best[1] < 0.98f * best[0] ? 1 : 0;
+  free_format(&f[1 - keep]);
+  *out = std::move(f[keep]);
+  out->reorder_ms = f[0].reorder_ms + f[1].reorder_ms + 4 * (best[0] + best[1]);
   return JIGSAW_SUCCESS;
 }
 
@@ -196,9 +250,14 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
   jigsaw_handle_s* h = new (std::nothrow) jigsaw_handle_s();
   if (!h) return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, "host allocation failed");
   set_status(JIGSAW_SUCCESS);
-  s = build_format(static_cast<const uint16_t*>(A), M, K, v, resolve_panel_rows(opt, M),
-                   opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC, opt ? opt->row_order : (int)JIGSAW_ROWS_GIVEN,
-                   reinterpret_cast<cudaStream_t>(stream), &h->f);
+  const int mode = opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC;
+  const int rows = opt ? opt->row_order : (int)JIGSAW_ROWS_GIVEN;
+  if (opt && opt->panel_rows == JIGSAW_PANEL_AUTOTUNE)
+    s = autotune_panels(static_cast<const uint16_t*>(A), M, K, v, mode, rows, opt->autotune_n,
+                        reinterpret_cast<cudaStream_t>(stream), &h->f);
+  else
+    s = build_format(static_cast<const uint16_t*>(A), M, K, v, resolve_panel_rows(opt, M), mode, rows,
+                     reinterpret_cast<cudaStream_t>(stream), &h->f);
   if (s != JIGSAW_SUCCESS) {
     delete h;
     return s;

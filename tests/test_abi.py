@@ -70,6 +70,12 @@ def test_reorder_validates_arguments_before_touching_the_device(L):
     assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
     opt = jig.Options(128, 0, 2)                       # c_dtype must be 0 (fp16) or 1 (fp32)
     assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(128, 0, 0, 0, 256)               # autotune_n only with panel_rows = -1
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(-1, 0, 0, 0, 100)                # autotune_n must be a multiple of 8
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(-1, 0, 0, 0, 0)                  # valid: fails only for want of a device
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 2
 
 
 def test_binding_struct_layouts_match_header(tmp_path):

@@ -760,3 +760,22 @@ def test_row_clustered_panels(M, K, v, s, kind, P, mode, ov, override):
     int_exact(Ci, Ai, Bi)
     h0 = jig.reorder(_dev(A), v, panel_rows=P, residual_mode=mode)
     assert np.array_equal(h0.export()["rowmap"], np.arange(M))     # identity for the given order
+
+
+
+@pytest.mark.parametrize("M,K,v,s,N", [(512, 2048, 4, 0.9, 256), (4096, 2048, 8, 0.9, 1024)])
+def test_panel_height_autotune(M, K, v, s, N):
+    """panel_rows = JIGSAW_PANEL_AUTOTUNE (per-shape panel height):
+    both formats are built and timed on the device, the faster kept; whichever it
+    is, the format is bit-exact vs the oracle at that height and C correct."""
+    A = synth.vector_sparse(M, K, v, s, 66)
+    B = synth.dense_b(K, N, 66)
+    h = jig.reorder(_dev(A), v, panel_rows=jig.PANEL_AUTOTUNE, autotune_n=N)
+    P = h.info()["panel_rows"]
+    assert P in (128, 256)
+    npan = (M + P - 1) // P
+    for p in sorted({0, npan - 1}):
+        assert_format_equal(h.export(), oracle.reorder(A, P=P, panels=(p, p + 1)), panels=(p, p + 1))
+    C = _host(h.spmm(_dev(B)))
+    torch.cuda.synchronize()
+    spmm_check(C, A, B, rows=np.unique(np.r_[np.arange(0, M, 37), M - 1]))
