@@ -416,16 +416,18 @@ def per_call_us(fn, flush, stream, torch, R=8, reps=7):
     return (timeit(graphed(fn)) - t0) / R * 1e3
 
 
-def roofline(b: Batch, ms_per_launch, peaks, traffic_key=None):
-    """Roofline of k_spmm (the only kernel of the step): algorithmic bytes or
-    executed flops per launch over the measured average launch duration; the
-    binding roof is the larger of bytes / HBM and executed flops / the measured
-    tcgen05.mma.sp peak of the variant (CTA pair or single CTA)."""
+def roofline(b: Batch, ms_per_step, launches, peaks, traffic_key=None):
+    """Roofline of k_spmm (the only kernel of the step, `launches` grouped
+    launches of <= 64 products each): algorithmic bytes or executed flops per
+    launch over the measured average launch duration (= the step's totals over
+    the step time); the binding roof is the larger of bytes / HBM and executed
+    flops / the measured tcgen05.mma.sp peak of the variant (CTA pair or single
+    CTA)."""
     hbm, bf16, src, sp = peaks
     sp_peak = sp["pair_m256_n256_tflops"] if b.pair else sp["single_m128_n256_tflops"]
     t_hbm = b.alg_bytes / (hbm * 1e9)
     t_tc = b.exec_flops / (sp_peak * 1e12)
-    s = ms_per_launch * 1e-3
+    s = ms_per_step * 1e-3
     if t_hbm >= t_tc:
         r = {"bound": "hbm", "achieved": b.alg_bytes / s / 1e9, "peak": hbm, "unit": "GB/s",
              "peak_source": src}
@@ -435,12 +437,14 @@ def roofline(b: Batch, ms_per_launch, peaks, traffic_key=None):
                             f"({sp.get('source', '')}); dense bf16 MEASURED_PEAKS x2 would be {2 * bf16:.0f}"}
     r["frac"] = r["achieved"] / r["peak"]
     r["traffic"] = None
-    r["alg_bytes_per_launch"] = b.alg_bytes
-    r["exec_flops_per_launch"] = b.exec_flops
-    r["t_roof_us"] = max(t_hbm, t_tc) * 1e6
+    r["launches_per_step"] = launches
+    r["per_launch_us"] = ms_per_step * 1e3 / max(1, launches)
+    r["alg_bytes_per_launch"] = b.alg_bytes / max(1, launches)
+    r["exec_flops_per_launch"] = b.exec_flops / max(1, launches)
+    r["t_roof_us_per_step"] = max(t_hbm, t_tc) * 1e6
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))[traffic_key or b.name]
-        r["traffic"] = prof["bytes_per_launch"]
+        r["traffic"] = prof["bytes_per_launch"] if launches == 1 else None
         r["traffic_unit"] = "bytes per launch"
         r["traffic_source"] = prof.get("source")
     except Exception:
@@ -476,6 +480,8 @@ def cublas_compare(b: Batch, flush, stream, torch, jig, jig_step_ms, steps, warm
     out["batched_compute"] = best
     out["batched_step_ms_16F_32F"] = [batched["16F"], batched["32F"]]
     out["speedup_vs_batched_cublas"] = batched[best] / jig_step_ms
+    if b.name == "venom":
+        out["cusparselt"] = cusparselt_compare(b, flush, stream, torch, jig_step_ms, steps, warmup)
     out["batched_how"] = ("one cublasGemmStridedBatchedEx per (M, K, N) group of the batch, best of "
                           "CUBLAS_COMPUTE_16F / 32F, graph-replayed and timed exactly like the jigsaw step "
                           "(event nodes around the step inside its graph, L2 flushed before)")
@@ -501,6 +507,35 @@ def cublas_compare(b: Batch, flush, stream, torch, jig, jig_step_ms, steps, warm
                              "the dense A, [graph of 8 x (L2 flush, call)] - [graph of 8 x flush], / 8, median of 7")
     out["detail"] = detail
     return out
+
+
+def cusparselt_compare(b: Batch, flush, stream, torch, jig_step_ms, steps, warmup):
+    """f4 (Table 3): the library 2:4 SpMM (cuSPARSELt via
+    torch._cslt_compress / torch._cslt_sparse_mm) on the natively 2:4 VENOM-style
+    A -- it cannot skip the all-zero columns Jigsaw's reorder removes -- per
+    matrix and as a batch, timed like the jigsaw step."""
+    try:
+        comp = [torch._cslt_compress(a) for a in b.dA]
+        torch._cslt_sparse_mm(comp[0], b.dB[0])
+        torch.cuda.synchronize()
+    except Exception as e:  # library without an sm_100 build, or API absent
+        return {"unavailable": f"{type(e).__name__}: {str(e).splitlines()[0][:200]}"}
+    outs = [None] * len(comp)
+
+    def step():
+        for i, (a, bb) in enumerate(zip(comp, b.dB)):
+            outs[i] = torch._cslt_sparse_mm(a, bb)
+    ms, _ = timed_steps(step, steps, warmup, flush, stream, torch)
+    per = {}
+    for i, (M, K, v, s, N) in enumerate(b.points):
+        tj = per_call_us(lambda: b.hs[i].spmm(b.dB[i], C=b.dC[i]), flush, stream, torch)
+        tc = per_call_us(lambda: torch._cslt_sparse_mm(comp[i], b.dB[i]), flush, stream, torch)
+        per.setdefault(point_tag(b.name, i, v, s), []).append(tc / tj)
+    return {"step_ms": ms, "speedup_step": ms / jig_step_ms,
+            "speedup_geomean_by_point": {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(per.items())},
+            "how": "torch._cslt_compress / torch._cslt_sparse_mm (cuSPARSELt 2:4 SpMM) on the natively 2:4 A; "
+                   "batch = one graph of the per-matrix calls timed like the jigsaw step, per matrix = graph "
+                   "difference with L2 flushed"}
 
 
 def e2e_host(b: Batch, jig, torch, steps, dist=None, world=1, dev=None):
@@ -574,7 +609,7 @@ def main():
     ms, clocks = timed_steps(lambda: b.step(jig), args.steps, args.warmup, flush, stream, torch,
                              dist=dist_, world=world, dev_index=dev.index or 0, outside=outside)
     value = total_eff / (ms * 1e-3) / 1e12
-    roof = roofline(b, ms / max(1, launches), peaks)
+    roof = roofline(b, ms, launches, peaks)
 
     cub = None
     if not args.no_cublas and b.points:
@@ -633,7 +668,7 @@ def main():
                                 dist=dist_, world=world, dev_index=dev.index or 0)
         eff4 = sum(2 * M * K * N for (M, K, v, s, N) in b4.all_points) * world
         c4 = {"workload": b4.desc, "value": eff4 / (ms4 * 1e-3) / 1e12, "unit": "TFLOP/s", "ms_per_step": ms4,
-              "steps": st4, "gpu_launches": l4 * st4, "roofline": roofline(b4, ms4 / max(1, l4), peaks),
+              "steps": st4, "gpu_launches": l4 * st4, "roofline": roofline(b4, ms4, l4, peaks),
               "clocks": clk4, "format": f"panel_rows=auto (P used: {b4.panel_rows_used})",
               "reorder_ms_total": b4.reorder_ms}
         if not args.no_cublas:
