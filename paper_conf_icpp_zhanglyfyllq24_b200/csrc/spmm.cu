@@ -1367,9 +1367,15 @@ int g_trace_ctas = 0;
 //     every replay zeroes its own workspace, and graph replays never share one
 //     with any other launch (a graph exec never runs concurrently with itself).
 constexpr size_t kWsTicket = 256, kWsHead = kWsTicket + 512 * 2 * 4;
+// Regions of streams that are no longer used are reclaimed once more than
+// kMaxRegions streams of a device have one: a region whose last launch has
+// completed (its event) and that no host thread is launching on is freed.
+constexpr size_t kMaxRegions = 64;
 struct StreamRegion {
   char* base = nullptr;
   size_t size = 0;
+  cudaEvent_t done = nullptr;  // recorded after every launch that used the region
+  int inflight = 0;            // host threads between acquire and the event record
 };
 std::mutex g_ws_mu;
 std::unordered_map<unsigned long long, StreamRegion> g_ws[64];
@@ -1377,7 +1383,19 @@ std::unordered_map<unsigned long long, StreamRegion> g_ws[64];
 struct Workspace {
   char* base = nullptr;
   bool graph_owned = false;
+  int dev = -1;
+  unsigned long long stream_id = 0;
 };
+
+// Eager launches: after the kernel that used the stream's region is enqueued.
+static void release_workspace(const Workspace& w, cudaStream_t s) {
+  if (w.graph_owned || !w.base || w.dev < 0) return;
+  std::lock_guard<std::mutex> lock(g_ws_mu);
+  auto it = g_ws[w.dev].find(w.stream_id);
+  if (it == g_ws[w.dev].end()) return;
+  if (it->second.done) cudaEventRecord(it->second.done, s);
+  --it->second.inflight;
+}
 
 static jigsaw_status_t acquire_workspace(int dev, size_t bytes, cudaStream_t s, Workspace* w) {
   if (dev < 0 || dev >= 64) return set_status(JIGSAW_ERROR_INTERNAL, "device ordinal out of range");
@@ -1398,7 +1416,25 @@ static jigsaw_status_t acquire_workspace(int dev, size_t bytes, cudaStream_t s, 
   e = cudaStreamGetId(s, &id);
   if (e != cudaSuccess) return cuda_status(e, "cudaStreamGetId");
   std::lock_guard<std::mutex> lock(g_ws_mu);
-  StreamRegion& r = g_ws[dev][id];
+  auto& map = g_ws[dev];
+  if (map.size() >= kMaxRegions && map.find(id) == map.end()) {
+    for (auto it = map.begin(); it != map.end();) {
+      StreamRegion& o = it->second;
+      if (o.inflight == 0 && (!o.done || cudaEventQuery(o.done) == cudaSuccess)) {
+        if (o.base) cudaFreeAsync(o.base, s);  // idle: its last launch has completed
+        if (o.done) cudaEventDestroy(o.done);
+        it = map.erase(it);
+      } else {
+        ++it;
+      }
+    }
+    cudaGetLastError();  // cudaEventQuery's cudaErrorNotReady is not an error here
+  }
+  StreamRegion& r = map[id];
+  if (!r.done && cudaEventCreateWithFlags(&r.done, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    r.done = nullptr;
+  }
   if (r.size < bytes) {
     const size_t sz = std::max<size_t>({bytes, (size_t)4 << 20, 2 * r.size});
     e = pool_alloc_async(&p, sz, s);
@@ -1411,6 +1447,9 @@ static jigsaw_status_t acquire_workspace(int dev, size_t bytes, cudaStream_t s, 
   }
   w->base = r.base;
   w->graph_owned = false;
+  w->dev = dev;
+  w->stream_id = id;
+  ++r.inflight;
   return JIGSAW_SUCCESS;
 }
 
@@ -1485,6 +1524,8 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   if (w.graph_owned) {
     cudaError_t e = cudaFreeAsync(w.base, s);  // free node right after the kernel node
     if (st == JIGSAW_SUCCESS && e != cudaSuccess) st = cuda_status(e, "workspace free node");
+  } else {
+    release_workspace(w, s);
   }
   return st;
 }

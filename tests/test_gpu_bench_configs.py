@@ -305,3 +305,27 @@ def test_single_product_dynamic_scheduler():
     torch.cuda.synchronize()
     for c in [C1] + outs:
         assert np.array_equal(_host(c).view(np.float16).astype(np.float64), ref)
+
+
+def test_many_streams_reclaim_regions():
+    """Launches that need a workspace on 80 different streams (more than the 64
+    per-stream regions kept per device): idle regions of earlier streams are
+    reclaimed while later streams run; every result bit-exact."""
+    mats, Bs, hs, refs = _int_batch(n_small=2, seed0=950)
+    dB = [_dev(b) for b in Bs]
+    outs = []
+    with jig.launch_override(k_pieces=1):
+        for i in range(80):
+            st = torch.cuda.Stream()
+            with torch.cuda.stream(st):
+                dC = [torch.empty((a.shape[0], b.shape[1]), dtype=torch.float16, device="cuda")
+                      for a, b in zip(mats, Bs)]
+                jig.spmm_batched(hs, dB, dC, stream=st)
+                assert jig.last_launch()["split_slots"] > 0
+                outs.append((st, dC))
+            if i % 16 == 15:
+                torch.cuda.synchronize()
+    torch.cuda.synchronize()
+    for st, dC in outs:
+        for r, c in zip(refs, dC):
+            assert np.array_equal(_host(c).view(np.float16).astype(np.float64), r)
