@@ -189,6 +189,17 @@ JIGSAW_API jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K
                                   const jigsaw_options_t* opt, jigsaw_stream_t stream,
                                   jigsaw_handle_t* out);
 
+/* jigsaw_reorder_ex for `count` matrices at once (a batch of independent
+ * matrices, e.g. every layer of a model): As[i] device fp16 Ms[i] x Ks[i]
+ * (ld = Ks[i]), vs[i], the same options for all.  The builds run concurrently
+ * on internal streams of the current device (host worker threads, one build
+ * each at a time), ordered after prior work on `stream`; synchronous.  On
+ * success out[i] receives the handles; on error every handle built so far is
+ * freed, out[] is all NULL and the first failure's status is returned. */
+JIGSAW_API jigsaw_status_t jigsaw_reorder_batched(const void* const* As, const int64_t* Ms, const int64_t* Ks,
+                                                  const int* vs, int count, const jigsaw_options_t* opt,
+                                                  jigsaw_stream_t stream, jigsaw_handle_t* out);
+
 /* Same as jigsaw_reorder_ex but A is a HOST pointer (copied to the device inside). */
 JIGSAW_API jigsaw_status_t jigsaw_reorder_host(const void* A_host, int64_t M, int64_t K, int v,
                                     const jigsaw_options_t* opt, jigsaw_stream_t stream,

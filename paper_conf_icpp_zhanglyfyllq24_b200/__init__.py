@@ -29,7 +29,7 @@ ABI_SYMBOLS = ["jigsaw_reorder", "jigsaw_spmm", "jigsaw_free", "jigsaw_last_stat
                "jigsaw_last_error_string", "jigsaw_version", "jigsaw_reorder_ex",
                "jigsaw_reorder_host", "jigsaw_get_info", "jigsaw_export_format",
                "jigsaw_spmm_host", "jigsaw_spmm_batched", "jigsaw_spmm_batched_host", "jigsaw_spmm_launches_per_call",
-               "jigsaw_debug_trace", "jigsaw_last_launch", "jigsaw_set_launch_override"]
+               "jigsaw_debug_trace", "jigsaw_last_launch", "jigsaw_set_launch_override", "jigsaw_reorder_batched"]
 
 C_F16, C_F32 = 0, 1            # jigsaw_c_dtype_t
 ROWS_GIVEN, ROWS_CLUSTERED = 0, 1   # jigsaw_row_order_t
@@ -104,6 +104,8 @@ def lib(build_if_missing: bool = True):
         "jigsaw_version": (ctypes.c_char_p, []),
         "jigsaw_reorder_ex": (ci, [vp, i64, i64, ci, ctypes.POINTER(Options), vp, ctypes.POINTER(vp)]),
         "jigsaw_reorder_host": (ci, [vp, i64, i64, ci, ctypes.POINTER(Options), vp, ctypes.POINTER(vp)]),
+        "jigsaw_reorder_batched": (ci, [ctypes.POINTER(vp), ctypes.POINTER(i64), ctypes.POINTER(i64),
+                                        ctypes.POINTER(ci), ci, ctypes.POINTER(Options), vp, ctypes.POINTER(vp)]),
         "jigsaw_get_info": (ci, [vp, ctypes.POINTER(Info)]),
         "jigsaw_export_format": (ci, [vp, ctypes.POINTER(FormatHost)]),
         "jigsaw_spmm_host": (ci, [vp, vp, i64, vp, vp]),
@@ -270,6 +272,25 @@ def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: i
     _raise_if(lib().jigsaw_reorder_ex(ctypes.c_void_p(A.data_ptr()), M, K, v, ctypes.byref(opt),
                                       _stream_ptr(stream), ctypes.byref(out)))
     return Handle(out.value)
+
+
+def reorder_batched(As, vs, panel_rows: int = 128, residual_mode: int = 0, c_dtype: int = C_F16,
+                    row_order: int = ROWS_GIVEN, autotune_n: int = 0, stream=None):
+    """jigsaw_reorder_batched: the formats of many matrices (CUDA fp16), built
+    concurrently on internal streams; returns a list of Handles."""
+    n = len(As)
+    if len(vs) != n:
+        raise ValueError("As and vs must have the same length")
+    for A in As:
+        _check_fp16_cuda(A, "A")
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order, autotune_n)
+    ap = (ctypes.c_void_p * n)(*[A.data_ptr() for A in As])
+    ms = (ctypes.c_int64 * n)(*[A.shape[0] for A in As])
+    ks = (ctypes.c_int64 * n)(*[A.shape[1] for A in As])
+    vv = (ctypes.c_int * n)(*vs)
+    out = (ctypes.c_void_p * n)()
+    _raise_if(lib().jigsaw_reorder_batched(ap, ms, ks, vv, n, ctypes.byref(opt), _stream_ptr(stream), out))
+    return [Handle(p) for p in out]
 
 
 def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: int = 0,

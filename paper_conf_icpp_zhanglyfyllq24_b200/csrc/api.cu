@@ -5,9 +5,12 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 #include <new>
 #include <string>
+#include <thread>
+#include <vector>
 
 #include "internal.h"
 
@@ -264,6 +267,72 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
   }
   h->f.c_dtype = opt ? opt->c_dtype : (int)JIGSAW_C_F16;
   *out = h;
+  return set_status(JIGSAW_SUCCESS);
+}
+
+jigsaw_status_t jigsaw_reorder_batched(const void* const* As, const int64_t* Ms, const int64_t* Ks, const int* vs,
+                                       int count, const jigsaw_options_t* opt, jigsaw_stream_t stream,
+                                       jigsaw_handle_t* out) {
+  if (count < 0 || (count > 0 && (!As || !Ms || !Ks || !vs || !out)))
+    return set_status(JIGSAW_ERROR_INVALID_VALUE, "bad batch arguments");
+  for (int i = 0; i < count; ++i) out[i] = nullptr;
+  for (int i = 0; i < count; ++i) {
+    jigsaw_status_t s = validate_reorder(As[i], Ms[i], Ks[i], vs[i], opt);
+    if (s != JIGSAW_SUCCESS) return s;
+    if (!aligned16(As[i])) return set_status(JIGSAW_ERROR_INVALID_VALUE, "A must be 16-byte aligned");
+  }
+  if (count == 0) return set_status(JIGSAW_SUCCESS);
+  int dev = 0;
+  jigsaw_status_t s = check_device(&dev);
+  if (s != JIGSAW_SUCCESS) return s;
+  // ordered after prior work on the caller's stream
+  cudaEvent_t ev = nullptr;
+  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventRecord(ev, reinterpret_cast<cudaStream_t>(stream)) != cudaSuccess) {
+    cudaError_t e = cudaGetLastError();
+    if (ev) cudaEventDestroy(ev);
+    return cuda_status(e, "jigsaw_reorder_batched: event");
+  }
+  int nthreads = std::min(count, 8);
+#if defined(JIG_DEV) && JIG_DEV
+  if (getenv("JIGSAW_REORDER_THREADS")) nthreads = std::max(1, std::min(count, atoi(getenv("JIGSAW_REORDER_THREADS"))));
+#endif
+  std::atomic<int> next{0};
+  std::vector<jigsaw_status_t> st(count, JIGSAW_SUCCESS);
+  std::vector<std::string> msg(count);
+  auto worker = [&]() {
+    cudaSetDevice(dev);
+    cudaStream_t ws = nullptr;
+    if (cudaStreamCreateWithFlags(&ws, cudaStreamNonBlocking) != cudaSuccess) {
+      cudaGetLastError();
+      ws = nullptr;
+    } else {
+      cudaStreamWaitEvent(ws, ev, 0);
+    }
+    for (int i; (i = next.fetch_add(1)) < count;) {
+      if (!ws) {
+        st[i] = JIGSAW_ERROR_CUDA;
+        msg[i] = "cudaStreamCreate failed";
+        continue;
+      }
+      st[i] = jigsaw_reorder_ex(As[i], Ms[i], Ks[i], vs[i], opt, reinterpret_cast<jigsaw_stream_t>(ws), &out[i]);
+      if (st[i] != JIGSAW_SUCCESS) msg[i] = jigsaw_last_error_string();
+    }
+    if (ws) cudaStreamDestroy(ws);
+  };
+  std::vector<std::thread> pool;
+  for (int t = 0; t + 1 < nthreads; ++t) pool.emplace_back(worker);
+  worker();
+  for (auto& t : pool) t.join();
+  cudaEventDestroy(ev);
+  for (int i = 0; i < count; ++i)
+    if (st[i] != JIGSAW_SUCCESS) {
+      for (int j = 0; j < count; ++j) {
+        jigsaw_free(out[j]);
+        out[j] = nullptr;
+      }
+      return set_status(st[i], "matrix " + std::to_string(i) + ": " + msg[i]);
+    }
   return set_status(JIGSAW_SUCCESS);
 }
 

@@ -17,8 +17,10 @@
 // (R-Q11) -- the definition the oracle (oracle/oracle.c) implements
 // independently; tests/test_gpu_parity.py compares the two bit for bit.
 #include <climits>
+#include <atomic>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
 
 #include "internal.h"
 
@@ -32,10 +34,13 @@ constexpr unsigned kFull = 0xFFFFFFFFu;
 
 __device__ uint16_t g_subs[kNumSubsets];  // all 4-subsets of 16 slots, lexicographic
 
-bool g_tables_ready[64] = {false};
+std::atomic<bool> g_tables_ready[64] = {};
+std::mutex g_tables_mu;
 
 jigsaw_status_t init_tables(int dev) {
-  if (dev >= 0 && dev < 64 && g_tables_ready[dev]) return JIGSAW_SUCCESS;
+  if (dev >= 0 && dev < 64 && g_tables_ready[dev].load(std::memory_order_acquire)) return JIGSAW_SUCCESS;
+  std::lock_guard<std::mutex> lock(g_tables_mu);
+  if (dev >= 0 && dev < 64 && g_tables_ready[dev].load(std::memory_order_acquire)) return JIGSAW_SUCCESS;
   uint16_t subs[kNumSubsets];
   int n = 0;
   for (int a = 0; a < 16; ++a)
@@ -45,7 +50,7 @@ jigsaw_status_t init_tables(int dev) {
           subs[n++] = (uint16_t)((1u << a) | (1u << b) | (1u << c) | (1u << d));
   cudaError_t e = cudaMemcpyToSymbol(g_subs, subs, sizeof subs);
   if (e != cudaSuccess) return cuda_status(e, "cudaMemcpyToSymbol(subsets)");
-  if (dev >= 0 && dev < 64) g_tables_ready[dev] = true;
+  if (dev >= 0 && dev < 64) g_tables_ready[dev].store(true, std::memory_order_release);
   return JIGSAW_SUCCESS;
 }
 
@@ -726,6 +731,22 @@ jigsaw_status_t dalloc(T** p, size_t bytes, std::vector<void*>& list) {
   return JIGSAW_SUCCESS;
 }
 
+// Scratch of one build: stream-ordered (the library's pool), released with
+// cudaFreeAsync on the build's stream -- no implicit device synchronisation, so
+// builds on different streams (jigsaw_reorder_batched) overlap.
+template <class T>
+jigsaw_status_t salloc(T** p, size_t bytes, std::vector<void*>& list, cudaStream_t s) {
+  *p = nullptr;
+  if (bytes == 0) bytes = 16;
+  cudaError_t e = pool_alloc_async((void**)p, bytes, s);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_status(JIGSAW_ERROR_OUT_OF_MEMORY, std::string("scratch allocation failed: ") + cudaGetErrorString(e));
+  }
+  list.push_back(*p);
+  return JIGSAW_SUCCESS;
+}
+
 }  // namespace
 
 void free_format(Format* f) {
@@ -786,12 +807,13 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
   jigsaw_status_t st = JIGSAW_SUCCESS;
   float ms = 0;
   auto cleanup = [&]() {
-    if (cnt) cudaFree(cnt);
-    if (Ap) cudaFree(Ap);
+    if (cnt) cudaFreeAsync(cnt, stream);
+    if (Ap) cudaFreeAsync(Ap, stream);
     if (e0) cudaEventDestroy(e0);
     if (e1) cudaEventDestroy(e1);
   };
-  if (cudaMalloc(&cnt, sizeof(int32_t) * M) != cudaSuccess || cudaMalloc(&Ap, sizeof(uint16_t) * M * K) != cudaSuccess ||
+  if (pool_alloc_async((void**)&cnt, sizeof(int32_t) * M, stream) != cudaSuccess ||
+      pool_alloc_async((void**)&Ap, sizeof(uint16_t) * M * K, stream) != cudaSuccess ||
       cudaMalloc(&rmap, sizeof(int32_t) * M) != cudaSuccess) {
     cudaGetLastError();
     if (rmap) cudaFree(rmap);
@@ -868,18 +890,18 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   f->npanels = npan;
   if ((st = init_tables(dev)) != JIGSAW_SUCCESS) return st;
 
-  JIG_TRY(dalloc(&masks, sizeof(RowMask) * npan * K, scratch));
-  JIG_TRY(dalloc(&S, sizeof(int32_t) * npan * K, scratch));
-  JIG_TRY(dalloc(&Kp, sizeof(int32_t) * npan, scratch));
-  JIG_TRY(dalloc(&T, sizeof(int32_t) * npan, scratch));
-  JIG_TRY(dalloc(&nres, sizeof(int32_t) * npan, scratch));
-  JIG_TRY(dalloc(&err, sizeof(int), scratch));
-  JIG_TRY(dalloc(&nnz, sizeof(unsigned long long), scratch));
-  JIG_TRY(dalloc(&queue, sizeof(int32_t) * npan * qcap, scratch));
-  JIG_TRY(dalloc(&sc.tcols, sizeof(int32_t) * npan * cap * 16, scratch));
-  JIG_TRY(dalloc(&sc.tperm, (size_t)npan * cap * 16, scratch));
-  JIG_TRY(dalloc(&sc.tev, sizeof(int32_t) * npan * cap * 16, scratch));
-  JIG_TRY(dalloc(&sc.tnev, (size_t)npan * cap, scratch));
+  JIG_TRY(salloc(&masks, sizeof(RowMask) * npan * K, scratch, stream));
+  JIG_TRY(salloc(&S, sizeof(int32_t) * npan * K, scratch, stream));
+  JIG_TRY(salloc(&Kp, sizeof(int32_t) * npan, scratch, stream));
+  JIG_TRY(salloc(&T, sizeof(int32_t) * npan, scratch, stream));
+  JIG_TRY(salloc(&nres, sizeof(int32_t) * npan, scratch, stream));
+  JIG_TRY(salloc(&err, sizeof(int), scratch, stream));
+  JIG_TRY(salloc(&nnz, sizeof(unsigned long long), scratch, stream));
+  JIG_TRY(salloc(&queue, sizeof(int32_t) * npan * qcap, scratch, stream));
+  JIG_TRY(salloc(&sc.tcols, sizeof(int32_t) * npan * cap * 16, scratch, stream));
+  JIG_TRY(salloc(&sc.tperm, (size_t)npan * cap * 16, scratch, stream));
+  JIG_TRY(salloc(&sc.tev, sizeof(int32_t) * npan * cap * 16, scratch, stream));
+  JIG_TRY(salloc(&sc.tnev, (size_t)npan * cap, scratch, stream));
   sc.cap = cap;
 
   JIG_CU(cudaEventCreate(&ev0), "cudaEventCreate");
@@ -892,7 +914,7 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   k_main_tiles<<<dim3((unsigned)((K / 16 + kR3Warps - 1) / kR3Warps), npan), 32 * kR3Warps, 0, stream>>>(
       masks, S, Kp, K, sc);
   {
-    static bool attr_set[64] = {};
+    static std::atomic<bool> attr_set[64] = {};
     if (dev >= 0 && dev < 64 && !attr_set[dev]) {
       JIG_CU(cudaFuncSetAttribute(k_overflow, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   (int)(kR4Warps * sizeof(TileSmem))), "cudaFuncSetAttribute(k_overflow)");
@@ -948,9 +970,9 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
     f->pin.resize(npan);
     for (int p = 0; p < npan; ++p) f->pin[p] = make_int4((hT[p] + 1) / 2, f->ks_off[p], f->kb_off[p], f->D[p]);
     JIG_TRY(dalloc(&f->d_pin, sizeof(int4) * npan, f->allocs));
-    JIG_TRY(dalloc(&d_ksoff, sizeof(int32_t) * (npan + 1), scratch));
-    JIG_TRY(dalloc(&d_kboff, sizeof(int32_t) * (npan + 1), scratch));
-    JIG_TRY(dalloc(&tile_off, sizeof(int32_t) * (npan + 1), scratch));
+    JIG_TRY(salloc(&d_ksoff, sizeof(int32_t) * (npan + 1), scratch, stream));
+    JIG_TRY(salloc(&d_kboff, sizeof(int32_t) * (npan + 1), scratch, stream));
+    JIG_TRY(salloc(&tile_off, sizeof(int32_t) * (npan + 1), scratch, stream));
     JIG_TRY(dalloc(&f->d_colidx, sizeof(int32_t) * 16 * f->ntiles, f->allocs));
     JIG_TRY(dalloc(&f->d_perm, (size_t)16 * f->ntiles, f->allocs));
     JIG_TRY(dalloc(&f->d_kind, (size_t)f->ntiles, f->allocs));
@@ -990,12 +1012,12 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   f->device_bytes += (int64_t)f->nksteps * (kKStepBytesA * f->halves() + 128) +
                      (int64_t)f->nkblocks * kEBlockBytes * f->halves() +
                      (int64_t)f->ntiles * (16 * 4 + 16 + 2) + (int64_t)npan * 12;
-  for (void* p : scratch) cudaFree(p);
+  for (void* p : scratch) cudaFreeAsync(p, stream);
   cudaEventDestroy(ev0);
   cudaEventDestroy(ev1);
   return JIGSAW_SUCCESS;
 fail:
-  for (void* p : scratch) cudaFree(p);
+  for (void* p : scratch) cudaFreeAsync(p, stream);
   if (ev0) cudaEventDestroy(ev0);
   if (ev1) cudaEventDestroy(ev1);
   free_format(f);
