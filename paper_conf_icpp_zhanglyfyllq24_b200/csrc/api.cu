@@ -421,16 +421,48 @@ jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const void* const
   return set_status(JIGSAW_SUCCESS);
 }
 
-// Several independent copies on one stream: one cudaMemcpyAsync per copy.
-// (The one-submission batch-copy call is not used: it faulted the GPU on this
-// pool's boxes, so the per-copy submission cost stays.)
+// Start of the CUDA allocation (pinned host or device) that holds p, or 0 for
+// memory CUDA does not know (pageable host memory).  Driver entry point looked
+// up once through the runtime (no link-time dependency on libcuda).
+static uintptr_t alloc_start(const void* p) {
+  using Fn = int (*)(void*, int, unsigned long long);
+  static Fn fn = []() -> Fn {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuPointerGetAttribute", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    return reinterpret_cast<Fn>(f);
+  }();
+  if (!fn) return 0;
+  unsigned long long start = 0;
+  constexpr int kRangeStartAddr = 11;  // CU_POINTER_ATTRIBUTE_RANGE_START_ADDR
+  return fn(&start, kRangeStartAddr, (unsigned long long)reinterpret_cast<uintptr_t>(p)) == 0 ? (uintptr_t)start : 0;
+}
+
+// True when host buffer b starts right where a (of `bytes`) ends, inside the
+// same CUDA allocation: the two copies can be one (two adjacent buffers of
+// separate pinned registrations cannot -- such a copy is rejected).
+static bool host_contiguous(const void* a, size_t bytes, const void* b) {
+  if (reinterpret_cast<const char*>(a) + bytes != reinterpret_cast<const char*>(b)) return false;
+  const uintptr_t s = alloc_start(a);
+  return s != 0 && s == alloc_start(b);
+}
+
+// Independent copies on one stream, one cudaMemcpyAsync per run of copies whose
+// host AND device sides are both contiguous (runs[] marks where a new copy
+// starts).  (The one-submission batch-copy call is not used: it faulted the GPU
+// on this pool's boxes.)
 static cudaError_t copy_batch(std::vector<void*>& dst, std::vector<void*>& src, std::vector<size_t>& sz,
-                              cudaMemcpyKind kind, cudaStream_t st) {
-  // No merging of address-adjacent copies: two host buffers can sit back to
-  // back yet belong to separate pinned registrations, and one copy spanning
-  // both is rejected (invalid argument).
+                              const std::vector<char>& joins, cudaMemcpyKind kind, cudaStream_t st) {
   cudaError_t e = cudaSuccess;
-  for (size_t i = 0; i < dst.size() && (e = cudaMemcpyAsync(dst[i], src[i], sz[i], kind, st)) == cudaSuccess; ++i) {
+  for (size_t i = 0; i < dst.size() && e == cudaSuccess;) {
+    size_t j = i + 1, bytes = sz[i];
+    while (j < dst.size() && joins[j]) bytes += sz[j++];
+    e = cudaMemcpyAsync(dst[i], src[i], bytes, kind, st);
+    i = j;
   }
   return e;
 }
@@ -464,13 +496,26 @@ static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_hand
                                             jigsaw_stream_t stream) {
   cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
   // staging for the whole batch (one pool allocation each for B and C)
+  // Staging offsets: products whose host buffers are contiguous in one pinned
+  // allocation (a caller that packs its batch) get contiguous staging too (16-byte
+  // aligned: K*N*2 and M*N*esize are multiples of 16), so their copies merge
+  // into one per chunk and direction; otherwise 256-byte aligned slots.
   size_t bb = 0, cb = 0;
   std::vector<size_t> boff(count), coff(count);
+  std::vector<char> bjoin(count, 0), cjoin(count, 0);
   for (int i = 0; i < count; ++i) {
+    const size_t bsz = (size_t)hs[i]->f.K * Ns[i] * 2, csz = (size_t)hs[i]->f.M * Ns[i] * c_elem_bytes(hs[i]->f);
+    if (i > 0) {
+      const size_t pb = (size_t)hs[i - 1]->f.K * Ns[i - 1] * 2, pc = (size_t)hs[i - 1]->f.M * Ns[i - 1] * c_elem_bytes(hs[i - 1]->f);
+      bjoin[i] = host_contiguous(Bs_host[i - 1], pb, Bs_host[i]);
+      cjoin[i] = host_contiguous(Cs_host[i - 1], pc, Cs_host[i]);
+    }
+    if (!bjoin[i]) bb = (bb + 255) & ~size_t(255);
+    if (!cjoin[i]) cb = (cb + 255) & ~size_t(255);
     boff[i] = bb;
     coff[i] = cb;
-    bb += ((size_t)hs[i]->f.K * Ns[i] * 2 + 255) & ~size_t(255);
-    cb += ((size_t)hs[i]->f.M * Ns[i] * c_elem_bytes(hs[i]->f) + 255) & ~size_t(255);
+    bb += bsz;
+    cb += csz;
   }
   cudaEvent_t ev0;
   if (cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming) != cudaSuccess) return cuda_status(cudaGetLastError(), "event");
@@ -507,12 +552,14 @@ static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_hand
     }
     std::vector<void*> cd, cs;
     std::vector<size_t> cz;
+    std::vector<char> jn;
     for (int i = i0; i < i1; ++i) {
       cd.push_back(dB + boff[i]);
       cs.push_back(const_cast<void*>(Bs_host[i]));
       cz.push_back((size_t)hs[i]->f.K * Ns[i] * 2);
+      jn.push_back(i > i0 && bjoin[i]);
     }
-    if (e == cudaSuccess) e = copy_batch(cd, cs, cz, cudaMemcpyHostToDevice, P.h2d);
+    if (e == cudaSuccess) e = copy_batch(cd, cs, cz, jn, cudaMemcpyHostToDevice, P.h2d);
     cudaEvent_t in, done;
     cudaEventCreateWithFlags(&in, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&done, cudaEventDisableTiming);
@@ -530,13 +577,14 @@ static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_hand
     if (e == cudaSuccess) st = launch_spmm_grouped(fs.data(), pb.data(), pn.data(), pc.data(), i1 - i0, P.comp);
     cudaEventRecord(done, P.comp);
     cudaStreamWaitEvent(P.d2h, done, 0);
-    cd.clear(); cs.clear(); cz.clear();
+    cd.clear(); cs.clear(); cz.clear(); jn.clear();
     for (int i = i0; i < i1; ++i) {
       cd.push_back(Cs_host[i]);
       cs.push_back(dC + coff[i]);
       cz.push_back((size_t)hs[i]->f.M * Ns[i] * c_elem_bytes(hs[i]->f));
+      jn.push_back(i > i0 && cjoin[i]);
     }
-    if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, cudaMemcpyDeviceToHost, P.d2h);
+    if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, jn, cudaMemcpyDeviceToHost, P.d2h);
     i0 = i1;
   }
   // staging goes back to the pool after the last copy-out

@@ -127,7 +127,10 @@ struct Cfg {
   static constexpr int kBGroups = JIG_BGROUPS < kStages ? JIG_BGROUPS : kStages;
   static constexpr int kWPG = kBProdWarps / kBGroups;  // warps per group
   static constexpr int kGS = (2 * kStages + kBGroups - 1) / kBGroups * kBGroups;
-  static constexpr int kGAhead = kStages;
+#ifndef JIG_GAHEAD_EXTRA
+#define JIG_GAHEAD_EXTRA 0  // developer: gather-list lead beyond the stage count
+#endif
+  static constexpr int kGAhead = kStages + JIG_GAHEAD_EXTRA;
   static constexpr size_t kSmem =
       1024 + (size_t)kStages * (kStageB + kStageA + kStageE) + (size_t)kGS * kStageG + kRecvBytes + kStageC + 512;
   static_assert(kSmem <= 232448, "shared memory budget");
