@@ -215,7 +215,9 @@ JIGSAW_API jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format
 /* C = A x B with B and C in HOST memory (end-to-end path): copies B in, runs
  * jigsaw_spmm, copies C out, all on `stream`, then synchronises `stream`.
  * C_host holds M x N elements of the handle's c_dtype.  Device staging buffers
- * are taken from the library's stream-ordered pool. */
+ * are taken from the library's stream-ordered pool, which afterwards keeps the
+ * largest host-buffer call's staging + 256 MB reserved (at most 1/4 of the
+ * device's memory) so repeated calls do not map memory again. */
 JIGSAW_API jigsaw_status_t jigsaw_spmm_host(jigsaw_handle_t h, const void* B_host, int64_t N, void* C_host,
                                  jigsaw_stream_t stream);
 
@@ -234,8 +236,8 @@ JIGSAW_API jigsaw_status_t jigsaw_spmm_batched(const jigsaw_handle_t* hs, const 
  * copies run on three streams of the handles' device, so the copy engines of
  * both directions and the SMs work at the same time; pinned host buffers are
  * needed for the copies to overlap (pageable memory is correct but serial).
- * Device staging comes from the stream-ordered pool and is returned before the
- * call returns; each call uses helper streams of its own (concurrent calls from
+ * Device staging comes from the stream-ordered pool (kept reserved as for
+ * jigsaw_spmm_host) and is returned to it before the call returns; each call uses helper streams of its own (concurrent calls from
  * several host threads do not wait for each other).  Ordered after prior work
  * on `stream`; synchronous: returns after every C is in host memory.  Errors as jigsaw_spmm_batched; a failure
  * in a later chunk leaves earlier Cs written. */

@@ -27,8 +27,10 @@ for w in sys.argv[1:] or ["c2", "c4"]:
         pk_B.append(blk_b[ob:ob + B.size].reshape(B.shape)); pk_B[-1][...] = B
         pk_C.append(blk_c[oc:oc + M * N].reshape(M, N)); ob += B.size; oc += M * N
     res = {}
-    for rep in range(3):
-        for name, (Bs, Cs) in (("separate", (sep_B, sep_C)), ("packed", (pk_B, pk_C))):
+    variants = (("separate", (sep_B, sep_C)), ("packed", (pk_B, pk_C)),
+                ("packed_B_only", (pk_B, sep_C)), ("packed_C_only", (sep_B, pk_C)))
+    for rep in range(int(os.environ.get("REPS", "3"))):
+        for name, (Bs, Cs) in variants:
             jig.spmm_batched_host(b.hs, Bs, Cs)
             t0 = time.perf_counter()
             for _ in range(5):
