@@ -142,6 +142,15 @@ class Format:
     rcol: np.ndarray       # [ndtiles, 16] int32 (DENSE mode)
     dvals: np.ndarray      # [ndtiles, P, 16] uint16 (DENSE mode)
     rowmap: np.ndarray = None  # [M] int32: panel row r is row rowmap[r] of A (identity unless row-clustered)
+    # CUDA-core tiles (cuda_core_split): per panel the
+    # number of 2:4 tiles moved off the tensor cores, and the nonzeros of their
+    # columns as panel-local (row, column, fp16 bits) entries, ordered by row
+    # then column; panel p owns entries cc_eoff[p] : cc_eoff[p + 1]
+    cc_T: np.ndarray = None     # [npanels] int64
+    cc_eoff: np.ndarray = None  # [npanels + 1] int64
+    cc_row: np.ndarray = None   # [nent] int32 (row within the panel)
+    cc_col: np.ndarray = None   # [nent] int32 (column of A)
+    cc_val: np.ndarray = None   # [nent] uint16 (fp16 bits, nonzero)
 
     @property
     def tile_off(self):
@@ -150,6 +159,11 @@ class Format:
     @property
     def dtile_off(self):
         return np.concatenate([[0], np.cumsum(self.D)]).astype(np.int64)
+
+    @property
+    def cc(self):
+        """CUDA-core entries (eoff, row, col, val) as check.check_format takes them."""
+        return None if self.cc_eoff is None else (self.cc_eoff, self.cc_row, self.cc_col, self.cc_val)
 
     @property
     def gather(self):
@@ -169,11 +183,12 @@ def row_cluster(A) -> np.ndarray:
     return perm
 
 
-def reorder(A, P=128, mode=0, panels=None, row_order=0) -> Format:
+def reorder(A, P=128, mode=0, panels=None, row_order=0, cc_max_nnz=0) -> Format:
     """O2: canonical reorder CR1 of A (M x K fp16), panels of P rows.
     mode 0 = SPTC (paper), 1 = DENSE residual.  ``panels`` = (p0, p1) restricts
     the work to a contiguous panel range (panels are independent).  row_order 1:
-    row-clustered panels -- CR1 of A[row_cluster(A)], rowmap = that order."""
+    row-clustered panels -- CR1 of A[row_cluster(A)], rowmap = that order.
+    cc_max_nnz > 0: then cuda_core_split(format, cc_max_nnz) (f3)."""
     A = _bits(A)
     rowmap = None
     if row_order:
@@ -203,8 +218,70 @@ def reorder(A, P=128, mode=0, panels=None, row_order=0) -> Format:
                               _ptr(meta), _ptr(kind), _ptr(nevict), _ptr(rcol), _ptr(dvals))
     finally:
         lib().orc_format_free(h)
-    return Format(M, K, P, mode, range(p0, p1), T, D, col_idx, perm, vals, meta, kind,
-                  nevict, rcol, dvals, rowmap if rowmap is not None else np.arange(M, dtype=np.int32))
+    f = Format(M, K, P, mode, range(p0, p1), T, D, col_idx, perm, vals, meta, kind,
+               nevict, rcol, dvals, rowmap if rowmap is not None else np.arange(M, dtype=np.int32))
+    return cuda_core_split(f, A, cc_max_nnz)
+
+
+def cuda_core_split(f: Format, A, Z: int) -> Format:
+    """f3 (§4.7: "For sparser data tile, even with a few
+    nonzero elements, using SpTC can result in low resource utilization ...
+    we can accelerate the sparser data tiles using CUDA cores").  Reading R-Q28:
+    a 2:4 tile of panel p is a CUDA-core tile iff its nonzero count -- the
+    nonzeros of A in the panel's rows and the tile's real (non-PAD) columns -- is
+    at most Z (Z = 0: none).  CUDA-core tiles leave the tile list (the other
+    tiles keep their order and contents); the nonzeros of their columns become
+    the panel's CUDA-core entries (panel row, column, fp16 bits), ordered by row,
+    then by column.  ``A`` is the matrix the format was built from (A[rowmap]
+    for row-clustered panels).  Written as the definition, panel by panel."""
+    A = canon_bits(A)
+    M = A.shape[0]
+    P = f.P
+    npan = len(f.T)
+    toff = f.tile_off
+    keep, ccT, eoff, rows, cols, vals = [], [], [0], [], [], []
+    for i, p in enumerate(f.panels):
+        r0 = p * P
+        nr = min(P, M - r0)
+        blk = A[r0:r0 + nr]
+        cc_cols = []
+        n_cc = 0
+        for t in range(toff[i], toff[i + 1]):
+            real = [int(c) for c in f.col_idx[t] if c != PAD]
+            nnz = int(sum(np.count_nonzero(blk[:, c]) for c in real))
+            if Z > 0 and nnz <= Z:
+                cc_cols.extend(real)
+                n_cc += 1
+            else:
+                keep.append(t)
+        ccT.append(n_cc)
+        cc_cols.sort()
+        for r in range(nr):
+            for c in cc_cols:
+                if blk[r, c] != 0:
+                    rows.append(r)
+                    cols.append(c)
+                    vals.append(blk[r, c])
+        eoff.append(len(rows))
+    keep = np.asarray(keep, dtype=np.int64)
+    ccT = np.asarray(ccT, dtype=np.int64)
+    f.T = np.asarray(f.T, dtype=np.int64) - ccT
+    f.col_idx, f.perm, f.vals, f.meta = f.col_idx[keep], f.perm[keep], f.vals[keep], f.meta[keep]
+    f.kind, f.nevict = f.kind[keep], f.nevict[keep]
+    f.cc_T = ccT
+    f.cc_eoff = np.asarray(eoff, dtype=np.int64)
+    f.cc_row = np.asarray(rows, dtype=np.int32)
+    f.cc_col = np.asarray(cols, dtype=np.int32)
+    f.cc_val = np.asarray(vals, dtype=np.uint16)
+    assert len(f.cc_eoff) == npan + 1
+    return f
+
+
+def canon_bits(A) -> np.ndarray:
+    """fp16 bits with -0 mapped to +0 (R-Q3): nonzero iff the value is != 0."""
+    A = _bits(A).copy()
+    A[(A & 0x7FFF) == 0] = 0
+    return A
 
 
 from .check import check_format, decode, format_bytes, canon  # noqa: E402,F401

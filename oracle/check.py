@@ -12,6 +12,9 @@ Checks:
                    columns, every one of them selected by the metadata (P:96);
   * metadata    -- i0 < i1 in every nibble;
   * PAD         -- values at PAD positions are +0;
+  * CUDA-core   -- (f3, R-Q28) entries (row, column, value) of a panel are in
+    entries        strictly increasing (row, column) order, inside the panel,
+                   nonzero; their columns are disjoint from the tiles' columns;
   * decode      -- decode(format) == canon(A) bitwise (canon: -0 -> +0, R-Q3).
 """
 from __future__ import annotations
@@ -32,8 +35,9 @@ def _nz(x):
     return (x & 0x7FFF) != 0
 
 
-def decode(M, K, P, T, gather, vals, meta, D=None, rcol=None, dvals=None):
-    """Rebuild the M x K fp16-bit matrix from the format."""
+def decode(M, K, P, T, gather, vals, meta, D=None, rcol=None, dvals=None, cc=None):
+    """Rebuild the M x K fp16-bit matrix from the format.
+    ``cc`` = (eoff, row, col, val): CUDA-core entries per panel (f3)."""
     out = np.zeros((M, K), np.uint16)
     npan = len(T)
     toff = np.concatenate([[0], np.cumsum(T)]).astype(np.int64)
@@ -57,6 +61,10 @@ def decode(M, K, P, T, gather, vals, meta, D=None, rcol=None, dvals=None):
                     c = rcol[d, j]
                     if c != PAD:
                         out[r0:r0 + nr, c] = dvals[d, :nr, j]
+        if cc is not None:
+            eoff, crow, ccol, cval = cc
+            e = slice(int(eoff[p]), int(eoff[p + 1]))
+            out[r0 + crow[e].astype(np.int64), ccol[e]] = cval[e]
     return out
 
 
@@ -71,10 +79,11 @@ def format_bytes(T, P, D=None):
 
 
 def check_format(A, P, T, gather, vals, meta, perm=None, D=None, rcol=None, dvals=None,
-                 panels=None):
+                 panels=None, cc=None):
     """Raise AssertionError if the format is not a valid encoding of A.
 
-    ``panels``: range of panel indices the format covers (default: all)."""
+    ``panels``: range of panel indices the format covers (default: all).
+    ``cc`` = (eoff, row, col, val): CUDA-core entries per panel (f3)."""
     A = np.asarray(A).view(np.uint16)
     M, K = A.shape
     npan_all = (M + P - 1) // P
@@ -96,6 +105,15 @@ def check_format(A, P, T, gather, vals, meta, perm=None, D=None, rcol=None, dval
         if doff is not None:
             rc = rcol[doff[i]:doff[i + 1]].reshape(-1)
             used = np.concatenate([used, rc[rc != PAD]])
+        if cc is not None:
+            eoff, crow, ccol, cval = cc
+            e = slice(int(eoff[i]), int(eoff[i + 1]))
+            er, ec, ev = crow[e].astype(np.int64), ccol[e].astype(np.int64), cval[e]
+            assert np.all((er >= 0) & (er < nr)), f"panel {p}: CUDA-core entry outside the panel"
+            assert np.all(_nz(ev)), f"panel {p}: CUDA-core entry holds a zero"
+            key = er * (K + 1) + ec
+            assert np.all(np.diff(key) > 0), f"panel {p}: CUDA-core entries not in (row, column) order"
+            used = np.concatenate([used, np.unique(ec)])
         assert len(used) == len(np.unique(used)), f"panel {p}: a column appears twice"
         assert np.array_equal(np.sort(used), S), f"panel {p}: gather is not a bijection onto S_p"
         for t in range(toff[i], toff[i + 1]):
@@ -117,7 +135,7 @@ def check_format(A, P, T, gather, vals, meta, perm=None, D=None, rcol=None, dval
                     colnz = _nz(blk[:, c])
                     assert np.all(sel[:nr] | ~colnz), f"tile {t} group {q}: a nonzero not selected"
     dec = decode(M, K, P, np.asarray(T), gather, vals, meta,
-                 D=D, rcol=rcol, dvals=dvals) if panels == range(npan_all) else None
+                 D=D, rcol=rcol, dvals=dvals, cc=cc) if panels == range(npan_all) else None
     if dec is not None:
         assert np.array_equal(dec, canon(A)), "decode(format) != canon(A)"
     else:
@@ -128,9 +146,14 @@ def check_format(A, P, T, gather, vals, meta, perm=None, D=None, rcol=None, dval
             sub_T = T[i:i + 1]
             sl = slice(toff[i], toff[i + 1])
             dsl = slice(doff[i], doff[i + 1]) if doff is not None else None
+            sub_cc = None
+            if cc is not None:
+                eoff, crow, ccol, cval = cc
+                e = slice(int(eoff[i]), int(eoff[i + 1]))
+                sub_cc = (np.array([0, e.stop - e.start]), crow[e], ccol[e], cval[e])
             d = decode(nr, K, P, sub_T, gather[sl], vals[sl], meta[sl],
                        D=None if D is None else np.asarray(D)[i:i + 1],
                        rcol=None if rcol is None else rcol[dsl],
-                       dvals=None if dvals is None else dvals[dsl])
+                       dvals=None if dvals is None else dvals[dsl], cc=sub_cc)
             assert np.array_equal(d, canon(A[r0:r0 + nr])), f"panel {p}: decode != canon(A)"
     return True
