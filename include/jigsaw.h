@@ -91,7 +91,17 @@ typedef struct {
   int c_dtype;       /* jigsaw_c_dtype_t: element type of C for every product with this handle */
   int row_order;     /* jigsaw_row_order_t */
   int autotune_n;    /* panel_rows = -1: columns of the probe product (0 = 256); else must be 0 */
-  int reserved[3];   /* must be zero */
+  int cc_max_nnz;    /* CUDA-core tiles (§4.7: "for sparser data tile ...
+                        accelerate the sparser data tiles using CUDA cores"; DESIGN.md R-Q28):
+                        Z >= 0.  A 2:4 tile of the canonical reorder (main or overflow) whose
+                        nonzero count -- the nonzeros of A in the panel's rows and the tile's
+                        real columns -- is <= Z leaves the tile list (the other tiles keep their
+                        order); the nonzeros of its columns become the panel's CUDA-core
+                        entries (panel row, column, value), which the SpMM epilogue multiplies
+                        on CUDA cores into the same fp32 accumulator row before C is written.
+                        0 (default): no CUDA-core tiles.  DENSE residual tiles are not
+                        affected.  Must be < 2^24. */
+  int reserved[2];   /* must be zero */
 } jigsaw_options_t;
 
 /* Statistics of a prepared matrix (jigsaw_get_info). */
@@ -115,6 +125,10 @@ typedef struct {
   int64_t format_bytes;    /* canonical format size: per tile 16P + 2P + 64 B (DESIGN.md R-Q19) */
   int64_t device_bytes;    /* device memory held by the handle */
   double reorder_ms;       /* device time of the reorder/format build */
+  int32_t cc_max_nnz;      /* jigsaw_options_t.cc_max_nnz the handle was built with */
+  int32_t reserved0;
+  int64_t cc_tiles;        /* sum_p of the tiles moved to the CUDA cores (not in ntiles) */
+  int64_t cc_entries;      /* CUDA-core entries (nonzeros of those tiles' columns) */
 } jigsaw_info_t;
 
 /* Caller-allocated host buffers for jigsaw_export_format; any member may be
@@ -134,6 +148,11 @@ typedef struct {
   int32_t* rowmap;   /* [M]                row r of the (row-clustered) panels is row rowmap[r] of A
                                            and of C; the identity for JIGSAW_ROWS_GIVEN.  The other
                                            arrays describe the matrix A[rowmap] */
+  int64_t* cc_T;     /* [npanels]          tiles moved to the CUDA cores per panel (cc_max_nnz) */
+  int64_t* cc_eoff;  /* [npanels + 1]      panel p owns CUDA-core entries cc_eoff[p] .. cc_eoff[p+1] */
+  int32_t* cc_row;   /* [cc_entries]       row of the entry within its panel, entries ordered by */
+  int32_t* cc_col;   /* [cc_entries]       (row, column): column of A */
+  uint16_t* cc_val;  /* [cc_entries]       fp16 bits of A at (row, column), nonzero */
 } jigsaw_format_host_t;
 
 /* ---------------------------------------------------------------- north-star calls */

@@ -44,7 +44,8 @@ class JigsawError(RuntimeError):
 
 class Options(ctypes.Structure):
     _fields_ = [("panel_rows", ctypes.c_int), ("residual_mode", ctypes.c_int), ("c_dtype", ctypes.c_int),
-                ("row_order", ctypes.c_int), ("autotune_n", ctypes.c_int), ("reserved", ctypes.c_int * 3)]
+                ("row_order", ctypes.c_int), ("autotune_n", ctypes.c_int), ("cc_max_nnz", ctypes.c_int),
+                ("reserved", ctypes.c_int * 2)]
 
 
 class Info(ctypes.Structure):
@@ -56,13 +57,14 @@ class Info(ctypes.Structure):
                 ("evictions", ctypes.c_int64), ("nnz", ctypes.c_int64), ("kp_total", ctypes.c_int64),
                 ("max_tiles", ctypes.c_int64), ("nksteps", ctypes.c_int64),
                 ("format_bytes", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
-                ("reorder_ms", ctypes.c_double)]
+                ("reorder_ms", ctypes.c_double), ("cc_max_nnz", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+                ("cc_tiles", ctypes.c_int64), ("cc_entries", ctypes.c_int64)]
 
 
 class FormatHost(ctypes.Structure):
     _fields_ = [(n, ctypes.c_void_p) for n in
                 ("T", "D", "col_idx", "perm", "gather", "vals", "meta", "kind", "nevict", "rcol", "dvals",
-                 "rowmap")]
+                 "rowmap", "cc_T", "cc_eoff", "cc_row", "cc_col", "cc_val")]
 
 
 class LaunchDesc(ctypes.Structure):
@@ -238,12 +240,15 @@ class Handle:
         """Canonical format (jigsaw_export_format) as numpy arrays."""
         inf = self.info()
         npan, nt, nd, P = inf["npanels"], inf["ntiles"], inf["ndtiles"], inf["panel_rows"]
+        ne = inf["cc_entries"]
         arr = dict(T=np.zeros(npan, np.int64), D=np.zeros(npan, np.int64),
                    col_idx=np.zeros((nt, 16), np.int32), perm=np.zeros((nt, 16), np.uint8),
                    gather=np.zeros((nt, 16), np.int32), vals=np.zeros((nt, P, 8), np.uint16),
                    meta=np.zeros((nt, P), np.uint16), kind=np.zeros(nt, np.uint8),
                    nevict=np.zeros(nt, np.uint8), rcol=np.zeros((nd, 16), np.int32),
-                   dvals=np.zeros((nd, P, 16), np.uint16), rowmap=np.zeros(inf["M"], np.int32))
+                   dvals=np.zeros((nd, P, 16), np.uint16), rowmap=np.zeros(inf["M"], np.int32),
+                   cc_T=np.zeros(npan, np.int64), cc_eoff=np.zeros(npan + 1, np.int64),
+                   cc_row=np.zeros(ne, np.int32), cc_col=np.zeros(ne, np.int32), cc_val=np.zeros(ne, np.uint16))
         fh = FormatHost(**{k: v.ctypes.data for k, v in arr.items()})
         _raise_if(lib().jigsaw_export_format(self._h, ctypes.byref(fh)))
         return arr
@@ -261,13 +266,14 @@ class Handle:
 
 
 def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: int = C_F16,
-            row_order: int = ROWS_GIVEN, autotune_n: int = 0, stream=None) -> Handle:
+            row_order: int = ROWS_GIVEN, autotune_n: int = 0, cc_max_nnz: int = 0, stream=None) -> Handle:
     """jigsaw_reorder_ex: multi-granularity reorder + format build of A (CUDA fp16 M x K).
     panel_rows = PANEL_AUTOTUNE times both panel heights on an autotune_n-column
-    product (0 = 256) and keeps the faster format."""
+    product (0 = 256) and keeps the faster format.  cc_max_nnz = Z > 0 moves the
+    tiles with <= Z nonzeros to the CUDA cores (f3, R-Q28)."""
     _check_fp16_cuda(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode, c_dtype, row_order, autotune_n)
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order, autotune_n, cc_max_nnz)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_ex(ctypes.c_void_p(A.data_ptr()), M, K, v, ctypes.byref(opt),
                                       _stream_ptr(stream), ctypes.byref(out)))
@@ -275,7 +281,7 @@ def reorder(A, v: int, panel_rows: int = 128, residual_mode: int = 0, c_dtype: i
 
 
 def reorder_batched(As, vs, panel_rows: int = 128, residual_mode: int = 0, c_dtype: int = C_F16,
-                    row_order: int = ROWS_GIVEN, autotune_n: int = 0, stream=None):
+                    row_order: int = ROWS_GIVEN, autotune_n: int = 0, cc_max_nnz: int = 0, stream=None):
     """jigsaw_reorder_batched: the formats of many matrices (CUDA fp16), built
     concurrently on internal streams; returns a list of Handles."""
     n = len(As)
@@ -283,7 +289,7 @@ def reorder_batched(As, vs, panel_rows: int = 128, residual_mode: int = 0, c_dty
         raise ValueError("As and vs must have the same length")
     for A in As:
         _check_fp16_cuda(A, "A")
-    opt = Options(panel_rows, residual_mode, c_dtype, row_order, autotune_n)
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order, autotune_n, cc_max_nnz)
     ap = (ctypes.c_void_p * n)(*[A.data_ptr() for A in As])
     ms = (ctypes.c_int64 * n)(*[A.shape[0] for A in As])
     ks = (ctypes.c_int64 * n)(*[A.shape[1] for A in As])
@@ -294,11 +300,11 @@ def reorder_batched(As, vs, panel_rows: int = 128, residual_mode: int = 0, c_dty
 
 
 def reorder_host(A: np.ndarray, v: int, panel_rows: int = 128, residual_mode: int = 0,
-                 c_dtype: int = C_F16, row_order: int = ROWS_GIVEN) -> Handle:
+                 c_dtype: int = C_F16, row_order: int = ROWS_GIVEN, cc_max_nnz: int = 0) -> Handle:
     """jigsaw_reorder_host: A given as a host array (fp16 or uint16 bits)."""
     A = _host16(A, "A")
     M, K = A.shape
-    opt = Options(panel_rows, residual_mode, c_dtype, row_order)
+    opt = Options(panel_rows, residual_mode, c_dtype, row_order, 0, cc_max_nnz)
     out = ctypes.c_void_p(0)
     _raise_if(lib().jigsaw_reorder_host(A.ctypes.data_as(ctypes.c_void_p), M, K, v,
                                         ctypes.byref(opt), None, ctypes.byref(out)))

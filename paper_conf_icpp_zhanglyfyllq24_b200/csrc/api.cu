@@ -200,7 +200,9 @@ jigsaw_status_t validate_reorder(const void* A, int64_t M, int64_t K, int v, con
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown c_dtype");
     if (opt->row_order != JIGSAW_ROWS_GIVEN && opt->row_order != JIGSAW_ROWS_CLUSTERED)
       return set_status(JIGSAW_ERROR_INVALID_VALUE, "unknown row_order");
-    for (int i = 0; i < 3; ++i)
+    if (opt->cc_max_nnz < 0 || opt->cc_max_nnz >= (1 << 24))
+      return set_status(JIGSAW_ERROR_INVALID_VALUE, "cc_max_nnz must be in [0, 2^24)");
+    for (int i = 0; i < 2; ++i)
       if (opt->reserved[i]) return set_status(JIGSAW_ERROR_INVALID_VALUE, "reserved options must be zero");
   }
   return JIGSAW_SUCCESS;
@@ -228,11 +230,11 @@ jigsaw_status_t validate_spmm(jigsaw_handle_t h, const void* B, int64_t N, const
 // best of 3 after a warm-up, CUDA events on the reorder's stream), the faster
 // is kept.  Ties (within 2 %) go to 128-row panels (split-K for small products).
 jigsaw_status_t autotune_panels(const uint16_t* dA, int64_t M, int64_t K, int v, int mode, int row_order, int n,
-                                cudaStream_t st, Format* out) {
+                                int cc, cudaStream_t st, Format* out) {
   Format f[2];
   const int P[2] = {kPanelRows, kPairPanelRows};
   for (int i = 0; i < 2; ++i) {
-    jigsaw_status_t s = build_format(dA, M, K, v, P[i], mode, row_order, st, &f[i]);
+    jigsaw_status_t s = build_format(dA, M, K, v, P[i], mode, row_order, cc, st, &f[i]);
     if (s != JIGSAW_SUCCESS) {
       if (i) free_format(&f[0]);
       return s;
@@ -302,11 +304,12 @@ jigsaw_status_t jigsaw_reorder_ex(const void* A, int64_t M, int64_t K, int v, co
   set_status(JIGSAW_SUCCESS);
   const int mode = opt ? opt->residual_mode : (int)JIGSAW_RESIDUAL_SPTC;
   const int rows = opt ? opt->row_order : (int)JIGSAW_ROWS_GIVEN;
+  const int cc = opt ? opt->cc_max_nnz : 0;
   if (opt && opt->panel_rows == JIGSAW_PANEL_AUTOTUNE)
-    s = autotune_panels(static_cast<const uint16_t*>(A), M, K, v, mode, rows, opt->autotune_n,
+    s = autotune_panels(static_cast<const uint16_t*>(A), M, K, v, mode, rows, opt->autotune_n, cc,
                         reinterpret_cast<cudaStream_t>(stream), &h->f);
   else
-    s = build_format(static_cast<const uint16_t*>(A), M, K, v, resolve_panel_rows(opt, M), mode, rows,
+    s = build_format(static_cast<const uint16_t*>(A), M, K, v, resolve_panel_rows(opt, M), mode, rows, cc,
                      reinterpret_cast<cudaStream_t>(stream), &h->f);
   if (s != JIGSAW_SUCCESS) {
     delete h;
@@ -732,6 +735,9 @@ jigsaw_status_t jigsaw_get_info(jigsaw_handle_t h, jigsaw_info_t* out) {
   out->format_bytes = (int64_t)(16 * f.P + 2 * f.P + 64) * f.ntiles + (int64_t)(32 * f.P + 64) * f.ndtiles;
   out->device_bytes = f.device_bytes;
   out->reorder_ms = f.reorder_ms;
+  out->cc_max_nnz = f.cc_max_nnz;
+  out->cc_tiles = f.cc_tiles;
+  out->cc_entries = f.cc_entries;
   return set_status(JIGSAW_SUCCESS);
 }
 
@@ -758,6 +764,27 @@ jigsaw_status_t jigsaw_export_format(jigsaw_handle_t h, jigsaw_format_host_t* ou
   if (nt && out->kind && e == cudaSuccess) e = cudaMemcpy(out->kind, f.d_kind, nt, cudaMemcpyDeviceToHost);
   if (nt && out->nevict && e == cudaSuccess) e = cudaMemcpy(out->nevict, f.d_nevict, nt, cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return cuda_status(e, "export copy");
+  if (out->cc_T)
+    for (int64_t p = 0; p < f.npanels; ++p) out->cc_T[p] = f.ccT.empty() ? 0 : f.ccT[p];
+  if (out->cc_eoff || out->cc_row || out->cc_col || out->cc_val) {
+    // CUDA-core entries (f3): per-row offsets over the padded panel rows -> per panel
+    std::vector<int32_t> off;
+    std::vector<int2> ent((size_t)f.cc_entries);
+    if (f.d_ccoff) {
+      off.resize((size_t)f.npanels * P + 1);
+      e = cudaMemcpy(off.data(), f.d_ccoff, off.size() * 4, cudaMemcpyDeviceToHost);
+      if (e == cudaSuccess && !ent.empty()) e = cudaMemcpy(ent.data(), f.d_ccent, ent.size() * 8, cudaMemcpyDeviceToHost);
+      if (e != cudaSuccess) return cuda_status(e, "export copy (CUDA-core entries)");
+    }
+    for (int64_t p = 0; p <= f.npanels; ++p)
+      if (out->cc_eoff) out->cc_eoff[p] = off.empty() ? 0 : off[p * P];
+    for (int64_t i = 0; !off.empty() && i < f.npanels * P; ++i)
+      for (int32_t k = off[i]; k < off[i + 1]; ++k) {
+        if (out->cc_row) out->cc_row[k] = (int32_t)(i % P);
+        if (out->cc_col) out->cc_col[k] = ent[k].x;
+        if (out->cc_val) out->cc_val[k] = (uint16_t)ent[k].y;
+      }
+  }
   if ((nt && (out->gather || out->vals || out->meta)) || (f.ndtiles && (out->rcol || out->dvals))) {
     // read back the device layout and invert it
     std::vector<uint8_t> A((size_t)f.planeA() * f.halves());

@@ -44,6 +44,15 @@ struct Format {
   uint8_t* d_Aimg = nullptr;  // [halves][nksteps][4096]: UMMA K-major no-swizzle core matrices
   uint8_t* d_Eimg = nullptr;  // [halves][nkblocks][128][4] u32: TMEM metadata lanes
   int32_t* d_G = nullptr;     // [nksteps][32]: B row per logical column (PAD -> K, TMA zero fill)
+  // CUDA-core tiles (f3, R-Q28; jigsaw_options_t.cc_max_nnz): the entries of row
+  // r of the (padded) panel rows -- global panel-row index pr = p * P + r -- are
+  // d_ccent[d_ccoff[pr] .. d_ccoff[pr + 1]), each {column, fp16 bits}, ordered
+  // by column; null when no tile moved
+  int cc_max_nnz = 0;
+  int64_t cc_tiles = 0, cc_entries = 0;
+  std::vector<int32_t> ccT;     // [npanels] tiles moved per panel
+  int32_t* d_ccoff = nullptr;   // [npanels * P + 1]
+  int2* d_ccent = nullptr;      // [cc_entries]
   int halves() const { return P > kPanelRows ? P / kPanelRows : 1; }
   int64_t planeA() const { return nksteps * (int64_t)kKStepBytesA; }
   int64_t planeE() const { return nkblocks * (int64_t)kEBlockBytes; }
@@ -74,7 +83,7 @@ jigsaw_launch_desc_t& last_launch();  // this thread's most recent jigsaw_spmm* 
 
 // reorder.cu: builds *f from device A (M x K fp16) on `stream`; synchronous.
 jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode, int row_order,
-                             cudaStream_t stream, Format* f);
+                             int cc_max_nnz, cudaStream_t stream, Format* f);
 void free_format(Format* f);
 
 // spmm.cu

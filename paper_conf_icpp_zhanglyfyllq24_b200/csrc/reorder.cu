@@ -416,6 +416,8 @@ struct Scratch {
   uint8_t* tperm;  // [npan][cap][16]
   int32_t* tev;    // [npan][cap][16]
   uint8_t* tnev;   // [npan][cap]
+  int32_t* tmap;   // [npan][cap] (CUDA-core split only, else null): tile t of the final list is
+                   // tile tmap[t] of the canonical reorder
   int cap;
 };
 
@@ -607,14 +609,15 @@ __global__ void __launch_bounds__(256) k_emit(const uint16_t* __restrict__ A, in
     const int h = tid >> 4, j = tid & 15, t = 2 * ks + h;
     int32_t g = kPad;
     if (t < Tp) {
-      const int64_t o = ((int64_t)p * sc.cap + t) * 16;
+      const int to = sc.tmap ? sc.tmap[(int64_t)p * sc.cap + t] : t;  // canonical tile index
+      const int64_t o = ((int64_t)p * sc.cap + to) * 16;
       g = sc.tcols[o + sc.tperm[o + j]];
       const int64_t ft = (int64_t)tile_off[p] + t;
       colidx[ft * 16 + j] = sc.tcols[o + j];
       perm[ft * 16 + j] = sc.tperm[o + j];
       if (j == 0) {
-        kind[ft] = t < (Kp[p] + 15) / 16 ? 0 : 1;
-        nevict[ft] = sc.tnev[(int64_t)p * sc.cap + t];
+        kind[ft] = to < (Kp[p] + 15) / 16 ? 0 : 1;
+        nevict[ft] = sc.tnev[(int64_t)p * sc.cap + to];
       }
     }
     gat[h][j] = g;
@@ -718,6 +721,86 @@ __global__ void __launch_bounds__(256) k_emit_dense(const uint16_t* __restrict__
   }
 }
 
+// ------------------------------------------------------------------ CC (f3)
+// CUDA-core tiles (DESIGN.md R-Q28).  CC1: one CTA
+// per panel; thread i of a chunk takes tile t = base + i of the canonical list,
+// counts its nonzeros (popcounts of its real columns' row masks) and keeps it
+// iff the count exceeds Z.  Kept tiles are numbered in list order (tmap: final
+// tile -> canonical tile); the real columns of the others are marked in the
+// panel's column bitmap ccbm (bit c of word c / 32).  T[p] becomes the kept count.
+__global__ void __launch_bounds__(256) k_cc_split(const RowMask* __restrict__ masks, int64_t K, Scratch sc,
+                                                  int32_t* __restrict__ T, int32_t* __restrict__ ccT,
+                                                  uint32_t* __restrict__ ccbm, int64_t KW, int Z) {
+  __shared__ int wsum[8];
+  const int p = blockIdx.x, tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int Tp = T[p];
+  int kept = 0;
+  for (int base = 0; base < Tp; base += 256) {
+    const int t = base + tid;
+    bool keep = false;
+    if (t < Tp) {
+      const int64_t o = ((int64_t)p * sc.cap + t) * 16;
+      int nnz = 0;
+      for (int j = 0; j < 16; ++j) {
+        const int32_t c = sc.tcols[o + j];
+        if (c == kPad) continue;
+        const RowMask m = masks[(int64_t)p * K + c];
+        nnz += __popc(m.lo.x) + __popc(m.lo.y) + __popc(m.lo.z) + __popc(m.lo.w) + __popc(m.hi.x) +
+               __popc(m.hi.y) + __popc(m.hi.z) + __popc(m.hi.w);
+      }
+      keep = nnz > Z;
+      if (!keep)
+        for (int j = 0; j < 16; ++j) {
+          const int32_t c = sc.tcols[o + j];
+          if (c != kPad) atomicOr(ccbm + (int64_t)p * KW + (c >> 5), 1u << (c & 31));
+        }
+    }
+    const unsigned b = __ballot_sync(kFull, keep);
+    if (lane == 0) wsum[warp] = __popc(b);
+    __syncthreads();
+    int pre = kept;
+    for (int w = 0; w < warp; ++w) pre += wsum[w];
+    int tot = 0;
+    for (int w = 0; w < 8; ++w) tot += wsum[w];
+    if (keep) sc.tmap[(int64_t)p * sc.cap + pre + __popc(b & ((1u << lane) - 1u))] = t;
+    kept += tot;
+    __syncthreads();
+  }
+  if (tid == 0) {
+    T[p] = kept;
+    ccT[p] = Tp - kept;
+  }
+}
+
+// CC2: one thread per panel row: the nonzeros of A in the panel's CUDA-core
+// columns (bitmap order = ascending column).  fill == 0: count them into
+// cnt[p * P + r]; fill == 1: write them as {column, fp16 bits} from off[p * P + r].
+__global__ void k_cc_entries(const uint16_t* __restrict__ A, int64_t M, int64_t K, int P,
+                             const uint32_t* __restrict__ ccbm, int64_t KW, int fill,
+                             int32_t* __restrict__ cnt, const int32_t* __restrict__ off, int2* __restrict__ ent) {
+  const int p = blockIdx.x, r = threadIdx.x;
+  if (r >= P) return;
+  const int64_t row = (int64_t)p * P + r;
+  int n = 0;
+  int64_t o = fill ? off[row] : 0;
+  if (row < M) {
+    const uint32_t* bm = ccbm + (int64_t)p * KW;
+    for (int64_t w = 0; w < KW; ++w) {
+      uint32_t b = bm[w];
+      while (b) {
+        const int c = (int)(w * 32) + __ffs(b) - 1;
+        b &= b - 1;
+        const uint16_t x = A[row * K + c];
+        if (x & 0x7FFFu) {
+          if (fill) ent[o++] = make_int2(c, x);
+          ++n;
+        }
+      }
+    }
+  }
+  if (!fill) cnt[row] = n;
+}
+
 template <class T>
 jigsaw_status_t dalloc(T** p, size_t bytes, std::vector<void*>& list) {
   *p = nullptr;
@@ -789,7 +872,7 @@ __global__ void __launch_bounds__(256) k_permute_rows(const uint16_t* __restrict
 }
 
 static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
-                                         cudaStream_t stream, Format* f);
+                                         int Z, cudaStream_t stream, Format* f);
 
 // Row-clustered panels (DESIGN.md R-Q27): the rows are ordered by
 // nonzero count, descending, ties by ascending row index (a stable counting sort
@@ -798,8 +881,8 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
 // rows then have fewer nonzero columns (K_p), hence fewer tiles and fewer B rows
 // to gather.  The row order of vector-sparse rows (v identical rows) is kept.
 jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode, int row_order,
-                             cudaStream_t stream, Format* f) {
-  if (row_order != JIGSAW_ROWS_CLUSTERED) return build_format_rows(dA, M, K, v, P, mode, stream, f);
+                             int cc_max_nnz, cudaStream_t stream, Format* f) {
+  if (row_order != JIGSAW_ROWS_CLUSTERED) return build_format_rows(dA, M, K, v, P, mode, cc_max_nnz, stream, f);
   int32_t *cnt = nullptr, *rmap = nullptr;
   uint16_t* Ap = nullptr;
   cudaEvent_t e0 = nullptr, e1 = nullptr;
@@ -850,7 +933,7 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
     return cuda_status(e, "reorder: row clustering");
   }
   cudaEventElapsedTime(&ms, e0, e1);
-  st = build_format_rows(Ap, M, K, v, P, mode, stream, f);
+  st = build_format_rows(Ap, M, K, v, P, mode, cc_max_nnz, stream, f);
   cleanup();
   if (st != JIGSAW_SUCCESS) {
     cudaFree(rmap);
@@ -865,7 +948,7 @@ jigsaw_status_t build_format(const uint16_t* dA, int64_t M, int64_t K, int v, in
 }
 
 static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t K, int v, int P, int mode,
-                                         cudaStream_t stream, Format* f) {
+                                         int Z, cudaStream_t stream, Format* f) {
   std::vector<void*> scratch;
   int dev = 0;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -884,9 +967,15 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   unsigned long long hnnz = 0;
   int herr = 0;
   int maxks = 0;
+  // CUDA-core split (f3): column bitmap per panel, per-row entry counts / offsets
+  const int64_t KW = (K + 31) / 32;
+  uint32_t* ccbm = nullptr;
+  int32_t *ccT = nullptr, *cccnt = nullptr, *ccoff = nullptr;
+  std::vector<int32_t> hccT(Z > 0 ? npan : 0), hcnt(Z > 0 ? (size_t)npan * P : 0);
 
   cudaGetDevice(&dev);
   f->M = M; f->K = K; f->v = v; f->P = P; f->mode = mode; f->device = dev;
+  f->cc_max_nnz = Z;
   f->npanels = npan;
   if ((st = init_tables(dev)) != JIGSAW_SUCCESS) return st;
 
@@ -903,6 +992,13 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   JIG_TRY(salloc(&sc.tev, sizeof(int32_t) * npan * cap * 16, scratch, stream));
   JIG_TRY(salloc(&sc.tnev, (size_t)npan * cap, scratch, stream));
   sc.cap = cap;
+  sc.tmap = nullptr;
+  if (Z > 0) {
+    JIG_TRY(salloc(&sc.tmap, sizeof(int32_t) * npan * cap, scratch, stream));
+    JIG_TRY(salloc(&ccbm, sizeof(uint32_t) * npan * KW, scratch, stream));
+    JIG_TRY(salloc(&ccT, sizeof(int32_t) * npan, scratch, stream));
+    JIG_TRY(salloc(&cccnt, sizeof(int32_t) * npan * P, scratch, stream));
+  }
 
   JIG_CU(cudaEventCreate(&ev0), "cudaEventCreate");
   JIG_CU(cudaEventCreate(&ev1), "cudaEventCreate");
@@ -923,6 +1019,13 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   }
   k_overflow<<<npan, 32 * kR4Warps, kR4Warps * sizeof(TileSmem), stream>>>(masks, S, Kp, K, sc, queue, qcap, T, err,
                                                                           mode, nres);
+  if (Z > 0) {  // f3: CUDA-core tiles leave the list (CC1), their entries are counted (CC2)
+    JIG_CU(cudaMemsetAsync(ccbm, 0, sizeof(uint32_t) * npan * KW, stream), "memset");
+    k_cc_split<<<npan, 256, 0, stream>>>(masks, K, sc, T, ccT, ccbm, KW, Z);
+    k_cc_entries<<<npan, P < 32 ? 32 : P, 0, stream>>>(dA, M, K, P, ccbm, KW, 0, cccnt, nullptr, nullptr);
+    JIG_CU(cudaMemcpyAsync(hccT.data(), ccT, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy ccT");
+    JIG_CU(cudaMemcpyAsync(hcnt.data(), cccnt, sizeof(int32_t) * npan * P, cudaMemcpyDeviceToHost, stream), "copy cc counts");
+  }
   JIG_CU(cudaGetLastError(), "reorder kernels launch");
   JIG_CU(cudaMemcpyAsync(hKp.data(), Kp, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy Kp");
   JIG_CU(cudaMemcpyAsync(hT.data(), T, sizeof(int32_t) * npan, cudaMemcpyDeviceToHost, stream), "copy T");
@@ -956,8 +1059,33 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
     f->kb_off[p + 1] = f->kb_off[p] + (nks + kStepsPerBlock - 1) / kStepsPerBlock;
     f->kp_total += hKp[p];
     f->max_tiles = std::max<int64_t>(f->max_tiles, hT[p]);
-    f->overflow_tiles += hT[p] - (hKp[p] + 15) / 16;
     maxks = std::max(maxks, nks);
+  }
+  f->ccT = hccT;
+  f->cc_tiles = 0;
+  for (int32_t x : hccT) f->cc_tiles += x;
+  f->cc_entries = 0;
+  if (f->cc_tiles > 0) {  // per-row entry offsets (host prefix sum), then the entries (CC2, fill)
+    std::vector<int32_t> hoff((size_t)npan * P + 1);
+    int64_t acc = 0;
+    for (size_t i = 0; i < hcnt.size(); ++i) {
+      hoff[i] = (int32_t)acc;
+      acc += hcnt[i];
+    }
+    if (acc >= ((int64_t)1 << 31)) {
+      st = set_status(JIGSAW_ERROR_UNSUPPORTED, "reorder: more than 2^31 CUDA-core entries");
+      goto fail;
+    }
+    hoff.back() = (int32_t)acc;
+    f->cc_entries = acc;
+    JIG_TRY(dalloc(&f->d_ccoff, sizeof(int32_t) * hoff.size(), f->allocs));
+    JIG_TRY(dalloc(&f->d_ccent, sizeof(int2) * acc, f->allocs));
+    JIG_CU(cudaMemcpyAsync(f->d_ccoff, hoff.data(), sizeof(int32_t) * hoff.size(), cudaMemcpyHostToDevice, stream),
+           "upload cc offsets");
+    k_cc_entries<<<npan, P < 32 ? 32 : P, 0, stream>>>(dA, M, K, P, ccbm, KW, 1, nullptr, f->d_ccoff, f->d_ccent);
+    JIG_CU(cudaGetLastError(), "k_cc_entries launch");
+    // the host copy of the offsets must outlive the async upload
+    JIG_CU(cudaStreamSynchronize(stream), "cc offsets");
   }
   f->ntiles = f->tile_off[npan];
   f->ndtiles = 0;
@@ -996,12 +1124,16 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
     JIG_CU(cudaGetLastError(), "k_emit launch");
     JIG_CU(cudaEventRecord(ev1, stream), "cudaEventRecord");
     // total evictions = sum of per-tile counts
-    std::vector<uint8_t> hnev(f->ntiles);
-    if (f->ntiles)
+    std::vector<uint8_t> hnev(f->ntiles), hkind(f->ntiles);
+    if (f->ntiles) {
       JIG_CU(cudaMemcpyAsync(hnev.data(), f->d_nevict, f->ntiles, cudaMemcpyDeviceToHost, stream), "copy nevict");
+      JIG_CU(cudaMemcpyAsync(hkind.data(), f->d_kind, f->ntiles, cudaMemcpyDeviceToHost, stream), "copy kind");
+    }
     JIG_CU(cudaStreamSynchronize(stream), "reorder R5");
     f->evictions = 0;
     for (uint8_t x : hnev) f->evictions += x;
+    f->overflow_tiles = 0;  // overflow tiles of the final list (kind 1)
+    for (uint8_t x : hkind) f->overflow_tiles += x;
   }
   {
     float ms = 0;
@@ -1012,6 +1144,7 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
   f->device_bytes += (int64_t)f->nksteps * (kKStepBytesA * f->halves() + 128) +
                      (int64_t)f->nkblocks * kEBlockBytes * f->halves() +
                      (int64_t)f->ntiles * (16 * 4 + 16 + 2) + (int64_t)npan * 12;
+  if (f->cc_tiles > 0) f->device_bytes += ((int64_t)npan * P + 1) * 4 + f->cc_entries * 8;
   for (void* p : scratch) cudaFreeAsync(p, stream);
   cudaEventDestroy(ev0);
   cudaEventDestroy(ev1);

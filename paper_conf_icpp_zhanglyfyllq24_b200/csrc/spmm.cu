@@ -144,14 +144,17 @@ struct Problem {
   const int4* pin;  // per panel {k-steps, first k-step, first E block, 0} (device)
   const __half* B;
   void* C;  // fp16 or fp32 (c32) row-major M x N
-  int64_t M, N, K;
-  int64_t planeA, planeE;  // bytes between the A / E planes of the two 128-row halves (P = 256)
+  const int32_t* rowmap;  // row-clustered panels: C row of panel row r (nullptr: identity)
+  const int32_t* ccoff;   // CUDA-core entries (f3): offsets per padded panel row (nullptr: none)
+  const int2* ccent;      //   {column, fp16 bits} per entry
   int64_t boff;  // offset of this problem's B in the concatenation of all B's (L2 prefetch)
+  // 32-bit fields keep the 64-problem table of grouped launches in parameter space
+  int32_t M, N, K;  // M < 2^31, N, K <= 2^30 (validated)
+  int32_t nksA, nkbE;  // k-steps / E blocks between the A / E planes of the two 128-row halves (P = 256)
   int npanels;
   int unit0;  // first global work unit of this problem
   int pin0;   // offset of this problem's panels in ParamsT::pin (if use_pin)
   int c32;    // 1: C is fp32 (jigsaw_options_t.c_dtype), else fp16
-  const int32_t* rowmap;  // row-clustered panels: C row of panel row r (nullptr: identity)
 };
 // Kernel parameters: a problem table and the panel table, kept in parameter space
 // (read with LDC, no dependent global load at kernel start).  Two sizes: a
@@ -239,6 +242,8 @@ struct Work {
   void* C;
   int c32;
   const int32_t* rowmap;
+  const int32_t* ccoff;
+  const int2* ccent;
   int64_t M, N, K;
   int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
   int piece, npieces, pslot;  // split-K piece of a grouped launch (npieces = 1: whole unit)
@@ -279,6 +284,8 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
       w.C = prm.pr[0].C;
       w.c32 = prm.pr[0].c32;
       w.rowmap = prm.pr[0].rowmap;
+      w.ccoff = prm.pr[0].ccoff;
+      w.ccent = prm.pr[0].ccent;
       w.M = prm.pr[0].M;
       w.N = prm.pr[0].N;
       w.K = prm.pr[0].K;
@@ -324,6 +331,8 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.C = prm.pr[i].C;
   w.c32 = prm.pr[i].c32;
   w.rowmap = prm.pr[i].rowmap;
+  w.ccoff = prm.pr[i].ccoff;
+  w.ccent = prm.pr[i].ccent;
   w.M = prm.pr[i].M;
   w.N = prm.pr[i].N;
   w.K = prm.pr[i].K;
@@ -350,8 +359,8 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.npieces = npieces;
   w.pslot = pslot;
   if constexpr (kPair) {
-    w.Aimg += rank * prm.pr[i].planeA;
-    w.Eimg += rank * prm.pr[i].planeE;
+    w.Aimg += rank * (int64_t)prm.pr[i].nksA * kKStepBytesA;
+    w.Eimg += rank * (int64_t)prm.pr[i].nkbE * kEBlockBytes;
     w.row0 = (int64_t)w.p * kPairPanelRows + rank * kPanelRows;
     w.kb_lo = piece * nkb / npieces;
     w.kb_hi = (piece + 1) * nkb / npieces;
@@ -398,6 +407,37 @@ __device__ __forceinline__ float4 ld_shared_f4(uint32_t saddr) {
 __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   __half2 h = __floats2half2_rn(a, b);
   return *reinterpret_cast<uint32_t*>(&h);
+}
+
+// CUDA-core tiles (f3, §4.7; DESIGN.md R-Q28): acc[j] += a * B[col][col0 + j]
+// for the entries {col, a} of this lane's panel row, j < width (columns past N
+// are skipped: N % 8 == 0, 16-byte B reads).  fp32 FMA into the tensor-core
+// accumulator before C is written.
+__device__ __forceinline__ float cc_f(float x) { return x; }
+__device__ __forceinline__ float cc_f(uint32_t x) { return __uint_as_float(x); }
+__device__ __forceinline__ void cc_set(float& d, float x) { d = x; }
+__device__ __forceinline__ void cc_set(uint32_t& d, float x) { d = __float_as_uint(x); }
+template <int W, class T>
+__device__ __forceinline__ void cc_accum(T (&acc)[W], const int2* __restrict__ ent, int e0, int e1,
+                                         const __half* __restrict__ B, int64_t N, int64_t col0, int width) {
+  for (int e = e0; e < e1; ++e) {
+    const int2 en = __ldg(ent + e);
+    const float a = __half2float(__ushort_as_half((unsigned short)en.y));
+    const __half* brow = B + (int64_t)en.x * N + col0;
+#pragma unroll
+    for (int j = 0; j < W / 8; ++j) {
+      if (8 * j < width && col0 + 8 * j < N) {
+        const uint4 b = __ldg(reinterpret_cast<const uint4*>(brow + 8 * j));
+        const __half2* h = reinterpret_cast<const __half2*>(&b);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const float2 f = __half22float2(h[k]);
+          cc_set(acc[8 * j + 2 * k], fmaf(a, f.x, cc_f(acc[8 * j + 2 * k])));
+          cc_set(acc[8 * j + 2 * k + 1], fmaf(a, f.y, cc_f(acc[8 * j + 2 * k + 1])));
+        }
+      }
+    }
+  }
 }
 
 template <int NT, bool kSplit, bool kPair, class Prm>
@@ -534,7 +574,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   } else if (warp == 0 && prm.bpf_bytes > 0) {
     const int64_t lo = (int64_t)blockIdx.x * prm.bpf_chunk, hi = min(prm.bpf_bytes, lo + prm.bpf_chunk);
     for (int i = 31 - lane; i < prm.nprob; i += 32) {  // lane 31 takes problem 0
-      const int64_t b0 = prm.pr[i].boff, b1 = b0 + prm.pr[i].K * prm.pr[i].N * 2;
+      const int64_t b0 = prm.pr[i].boff, b1 = b0 + (int64_t)prm.pr[i].K * prm.pr[i].N * 2;
       const int64_t x0 = max(lo, b0), x1 = min(hi, b1);
       if (x0 < x1)
         bulk_prefetch_l2(reinterpret_cast<const uint8_t*>(prm.pr[i].B) + (x0 - b0), (uint32_t)(x1 - x0));
@@ -938,6 +978,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             srow[i] = lrow < M ? (wk.rowmap ? (int64_t)mrow : lrow) : -1;
           }
         }
+        int ce0 = 0, ce1 = 0;  // this lane's CUDA-core entries (f3)
+        if (wk.ccent) {
+          const int64_t pr = wk.row0 + q * 32 + lane;  // padded panel-row index
+          ce0 = wk.ccoff[pr];
+          ce1 = wk.ccoff[pr + 1];
+        }
         const int npc = wk.npieces;
         if (npc > 1) {
           // split-K piece: publish the fp32 partial tile, count the pieces done;
@@ -1000,6 +1046,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
               }
             }
           }
+          if (ce1 > ce0)
+            cc_accum(v, wk.ccent, ce0, ce1, wk.B, N, n0 + ucol(c0 / 32), ncols - c0);
           // Transposed through shared memory so that each store instruction
           // writes 8 rows x 64 contiguous bytes (4 lanes per row) instead of 32
           // rows x 16 bytes; 16-byte chunks swizzled by (row >> 1) & 3.
@@ -1105,6 +1153,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           }
           const int64_t lrow = (int64_t)p * 128 + rank * rpo + i;
           const int64_t colg = n0 + c8 * 8;
+          if (wk.ccent) {  // CUDA-core entries of this row (f3)
+            const int e0 = wk.ccoff[lrow], e1 = wk.ccoff[lrow + 1];
+            if (e1 > e0) cc_accum(acc, wk.ccent, e0, e1, wk.B, N, colg, 8);
+          }
           if (lrow < M && colg < N) {
             const int64_t row = wk.rowmap ? (int64_t)wk.rowmap[lrow] : lrow;
             if (c32) {
@@ -1332,17 +1384,19 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
     prm.use_pin = 0;
   P.Aimg = f.d_Aimg;
   P.Eimg = f.d_Eimg;
-  P.planeA = f.planeA();
-  P.planeE = f.planeE();
+  P.nksA = (int32_t)f.nksteps;
+  P.nkbE = (int32_t)f.nkblocks;
   P.G = f.d_G;
   P.pin = f.d_pin;
   P.B = reinterpret_cast<const __half*>(dB);
   P.C = dC;
   P.c32 = f.c_dtype == JIGSAW_C_F32 ? 1 : 0;
   P.rowmap = f.d_rowmap;
-  P.M = f.M;
-  P.N = N;
-  P.K = f.K;
+  P.ccoff = f.d_ccoff;
+  P.ccent = f.d_ccent;
+  P.M = (int32_t)f.M;
+  P.N = (int32_t)N;
+  P.K = (int32_t)f.K;
   P.npanels = (int)f.npanels;
   P.boff = i == 0 ? 0 : prm.pr[i - 1].boff + prm.pr[i - 1].K * prm.pr[i - 1].N * 2;
 }

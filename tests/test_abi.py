@@ -66,8 +66,14 @@ def test_reorder_validates_arguments_before_touching_the_device(L):
     opt = jig.Options(128, 7)
     assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
     opt = jig.Options(128, 0)
-    opt.reserved[2] = 1
+    opt.reserved[1] = 1
     assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(128, 0, 0, 0, 0, -1)             # cc_max_nnz must be >= 0
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(128, 0, 0, 0, 0, 1 << 24)        # ... and < 2^24
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
+    opt = jig.Options(128, 0, 0, 0, 0, 16)             # valid: fails only for want of a device
+    assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 2
     opt = jig.Options(128, 0, 2)                       # c_dtype must be 0 (fp16) or 1 (fp32)
     assert L.jigsaw_reorder_ex(p, 8, 8, 1, ctypes.byref(opt), None, ctypes.byref(out)) == 1
     opt = jig.Options(128, 0, 0, 0, 256)               # autotune_n only with panel_rows = -1
