@@ -202,6 +202,9 @@ def algorithmic(info: dict, M: int, K: int, N: int, rows_touched: int, c_bytes_p
     b_bytes = 2 * N * rows_touched
     c_bytes = c_bytes_per_elem * M * N
     exec_flops = 2 * P * 16 * info["ntiles"] * N
+    if info.get("cc_entries"):  # CUDA-core entries (f3): {column, value} 8 B each + per-row offsets
+        a_bytes += 8 * info["cc_entries"] + 4 * (info["npanels"] * P + 1)
+        exec_flops += 2 * info["cc_entries"] * N
     return a_bytes + b_bytes + c_bytes, exec_flops
 
 
@@ -292,8 +295,9 @@ class Batch:
     """One rank's share of a workload, prepared: formats (jigsaw_reorder, untimed,
     P:263), device B / C, host copies of A / B, and the roofline terms."""
 
-    def __init__(self, name, rank, world, panel_rows, dev, torch, jig):
+    def __init__(self, name, rank, world, panel_rows, dev, torch, jig, cc_max_nnz=0):
         self.name = name
+        self.cc_max_nnz = cc_max_nnz
         self.all_points, self.desc, self.scaling = workload(name)
         jobs = local_jobs(name, self.all_points, rank, world)
         self.points = [(M, K, v, s, n1 - n0) for (M, K, v, s, N, seed, n0, n1) in jobs]
@@ -309,7 +313,7 @@ class Batch:
             N = n1 - n0
             self.mats.append((A, B))
             a_t = torch.from_numpy(A.view(np.int16)).to(dev).view(torch.float16)
-            h = jig.reorder(a_t, v, panel_rows=panel_rows)
+            h = jig.reorder(a_t, v, panel_rows=panel_rows, cc_max_nnz=cc_max_nnz)
             info = h.info()
             self.reorder_ms += info["reorder_ms"]
             self.hs.append(h)
@@ -599,6 +603,8 @@ def main():
     ap.add_argument("--no-extra", action="store_true", help="skip the c4 sub-object of the default run")
     ap.add_argument("--multi", action="store_true", help="also run the C5a / C5b sharded sweep at N = 1")
     ap.add_argument("--detail", action="store_true", help="print the per-point table to stderr")
+    ap.add_argument("--cc-max-nnz", type=int, default=0,
+                    help="CUDA-core tiles (f3, R-Q28): tiles with <= Z nonzeros run on CUDA cores (0 = none)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -627,7 +633,7 @@ def main():
     flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
     dist_ = dist if world > 1 else None
 
-    b = Batch(args.workload, rank, world, args.panel_rows, dev, torch, jig)
+    b = Batch(args.workload, rank, world, args.panel_rows, dev, torch, jig, cc_max_nnz=args.cc_max_nnz)
     total_eff = sum(2 * M * K * N for (M, K, v, s, N) in b.all_points) * (world if b.scaling == "weak" else 1)
     b.step(jig)
     torch.cuda.synchronize()
@@ -670,7 +676,8 @@ def main():
                              "(stream of the launch); events around the whole graph replay, graph launch latency "
                              f"included: {outside.get('ms_per_step', 0) * 1e3:.1f} us per step",
                    "seeds": "synth.SEED_BASE + 1000*rank + index",
-                   "format": f"panel_rows={args.panel_rows or 'auto'} (P used: {b.panel_rows_used}), SPTC residual"},
+                   "format": f"panel_rows={args.panel_rows or 'auto'} (P used: {b.panel_rows_used}), SPTC residual"
+                             + (f", cc_max_nnz={args.cc_max_nnz}" if args.cc_max_nnz else "")},
         "roofline": roof,
         "cpu_baseline": None,
         "e2e": {"value": total_eff / e2e_s / 1e12, "unit": "TFLOP/s",

@@ -19,6 +19,7 @@ constexpr int kKStepBytesA = 4096;  // 128 rows x 16 halves (compressed 32 logic
 constexpr int kStepsPerBlock = 4;   // k-steps per E block (tcgen05.cp 128x128b = 4 TMEM columns)
 constexpr int kEBlockBytes = 2048;  // 128 lanes x 16 B
 constexpr int kPad = -1;
+constexpr int kPinCC = 1 << 30;     // flag in the device copy of a panel's pin.w: the panel has CUDA-core entries
 
 // Device-resident prepared matrix (the reorder-aware format).
 struct Format {
@@ -31,8 +32,14 @@ struct Format {
   // host copies of per-panel counts / offsets
   std::vector<int32_t> T, D, tile_off, ks_off, kb_off;
   // device per-panel arrays
-  int4* d_pin = nullptr;       // [npanels] {k-steps = ceil(T_p/2), first k-step, first E block, 0}
-  std::vector<int4> pin;       // host copy of d_pin
+  int4* d_pin = nullptr;       // [npanels] {k-steps = ceil(T_p/2), first k-step, first E block, dense k-steps},
+                               // .w | kPinCC on the device when the panel has CUDA-core entries (f3)
+  std::vector<int4> pin;       // host copy of d_pin, without the kPinCC flag
+  int4 pin_dev(int64_t p) const {  // the device form of pin[p]
+    int4 x = pin[p];
+    if (!ccT.empty() && ccT[p] > 0) x.w |= kPinCC;
+    return x;
+  }
   // canonical arrays (device)
   int32_t* d_colidx = nullptr;  // [ntiles][16]
   uint8_t* d_perm = nullptr;    // [ntiles][16]

@@ -689,7 +689,7 @@ __global__ void __launch_bounds__(256) k_emit_dense(const uint16_t* __restrict__
   __shared__ int32_t cols[16];
   const int p = blockIdx.y, j = blockIdx.x, tid = threadIdx.x;
   const int4 pi = pin[p];
-  if (j >= pi.w) return;
+  if (j >= (pi.w & ~kPinCC)) return;
   const int64_t gks = (int64_t)pi.y + ((pi.x + kStepsPerBlock - 1) / kStepsPerBlock) * kStepsPerBlock + j;
   const int n = nres[p];
   if (tid < 32) {
@@ -1108,7 +1108,9 @@ static jigsaw_status_t build_format_rows(const uint16_t* dA, int64_t M, int64_t 
     JIG_TRY(dalloc(&f->d_Aimg, (size_t)kKStepBytesA * f->nksteps * f->halves(), f->allocs));
     JIG_TRY(dalloc(&f->d_Eimg, (size_t)kEBlockBytes * f->nkblocks * f->halves(), f->allocs));
     JIG_TRY(dalloc(&f->d_G, sizeof(int32_t) * 32 * f->nksteps, f->allocs));
-    JIG_CU(cudaMemcpyAsync(f->d_pin, f->pin.data(), sizeof(int4) * npan, cudaMemcpyHostToDevice, stream), "upload");
+    std::vector<int4> pin_dev(npan);  // the device form (kPinCC flags); synchronised below before it goes
+    for (int p = 0; p < npan; ++p) pin_dev[p] = f->pin_dev(p);
+    JIG_CU(cudaMemcpyAsync(f->d_pin, pin_dev.data(), sizeof(int4) * npan, cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(d_ksoff, f->ks_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(d_kboff, f->kb_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");
     JIG_CU(cudaMemcpyAsync(tile_off, f->tile_off.data(), sizeof(int32_t) * (npan + 1), cudaMemcpyHostToDevice, stream), "upload");

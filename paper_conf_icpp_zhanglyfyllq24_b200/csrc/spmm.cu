@@ -247,6 +247,7 @@ struct Work {
   int64_t M, N, K;
   int p, n0, nks, ndk, nkb_s, kb_lo, kb_hi;
   int piece, npieces, pslot;  // split-K piece of a grouped launch (npieces = 1: whole unit)
+  bool ccp;                   // the panel has CUDA-core entries (f3; kPinCC)
   int ncols;                  // C columns of this unit (NT, or NT / nsplit for an N-split unit)
   bool valid;                 // false: padding entry of a static per-slot schedule
   int64_t ks0, kb0;  // first k-step / E block of the panel
@@ -294,7 +295,8 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
       w.kb_lo = a.z;
       w.kb_hi = a.w;
       w.nks = b.x;
-      w.ndk = b.y;
+      w.ndk = b.y & ~kPinCC;
+      w.ccp = (b.y & kPinCC) != 0;
       w.ks0 = b.z;
       w.kb0 = b.w;
       w.nkb_s = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
@@ -352,7 +354,8 @@ __device__ __forceinline__ Work decode_unit(const Prm& prm, int u, uint32_t rank
   w.nks = pi.x;
   w.ks0 = pi.y;
   w.kb0 = pi.z;
-  w.ndk = pi.w;
+  w.ndk = pi.w & ~kPinCC;
+  w.ccp = (pi.w & kPinCC) != 0;
   w.nkb_s = (w.nks + kStepsPerBlock - 1) / kStepsPerBlock;
   const int nkb = w.nkb_s + (w.ndk + kStepsPerBlock - 1) / kStepsPerBlock;
   w.piece = piece;
@@ -429,6 +432,41 @@ __device__ __forceinline__ void cc_accum(T (&acc)[W], const int2* __restrict__ e
       if (8 * j < width && col0 + 8 * j < N) {
         const uint4 b = __ldg(reinterpret_cast<const uint4*>(brow + 8 * j));
         const __half2* h = reinterpret_cast<const __half2*>(&b);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const float2 f = __half22float2(h[k]);
+          cc_set(acc[8 * j + 2 * k], fmaf(a, f.x, cc_f(acc[8 * j + 2 * k])));
+          cc_set(acc[8 * j + 2 * k + 1], fmaf(a, f.y, cc_f(acc[8 * j + 2 * k + 1])));
+        }
+      }
+    }
+  }
+}
+
+// Entries two at a time: both entries, then both B row segments are loaded
+// before the FMAs (two dependent chains in flight instead of one per entry).
+template <class T>
+__device__ __forceinline__ void cc_accum2(T (&acc)[32], const int2* __restrict__ ent, int e0, int e1,
+                                          const __half* __restrict__ B, int64_t N, int64_t col0, int width) {
+  for (int e = e0; e < e1; e += 2) {
+    const int n = min(e1 - e, 2);
+    int2 en[2];
+#pragma unroll
+    for (int i = 0; i < 2; ++i) en[i] = i < n ? __ldg(ent + e + i) : make_int2(0, 0);
+    uint4 b[2][4];
+#pragma unroll
+    for (int i = 0; i < 2; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        b[i][j] = (i < n && 8 * j < width && col0 + 8 * j < N)
+                      ? __ldg(reinterpret_cast<const uint4*>(B + (int64_t)en[i].x * N + col0 + 8 * j))
+                      : make_uint4(0, 0, 0, 0);
+#pragma unroll
+    for (int i = 0; i < 2; ++i) {
+      const float a = __half2float(__ushort_as_half((unsigned short)en[i].y));  // 0 for the padding entry
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const __half2* h = reinterpret_cast<const __half2*>(&b[i][j]);
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const float2 f = __half22float2(h[k]);
@@ -942,6 +980,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it % C_::kAccBufs;
       const int ncols = wk.ncols;                        // C columns of this unit
+      // CUDA-core entries of this lane's row (f3): fetched, and their B row
+      // segments prefetched into L2, while the accumulator is still being built
+      int ce0 = 0, ce1 = 0;
+      if (!kSplit && wk.ccp) {
+        const int64_t pr = wk.row0 + q * 32 + lane;  // padded panel-row index
+        ce0 = wk.ccoff[pr];
+        ce1 = wk.ccoff[pr + 1];
+        for (int e = ce0; e < ce1 && e < ce0 + 8; ++e)
+          bulk_prefetch_l2(wk.B + (int64_t)__ldg(wk.ccent + e).x * N + n0, (uint32_t)ncols * 2u);
+      }
       if (has_acc) {
         mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
         tc_fence_after();
@@ -977,12 +1025,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             const int mrow = __shfl_sync(kFullMask, crow, 8 * i + (lane >> 2));
             srow[i] = lrow < M ? (wk.rowmap ? (int64_t)mrow : lrow) : -1;
           }
-        }
-        int ce0 = 0, ce1 = 0;  // this lane's CUDA-core entries (f3)
-        if (wk.ccent) {
-          const int64_t pr = wk.row0 + q * 32 + lane;  // padded panel-row index
-          ce0 = wk.ccoff[pr];
-          ce1 = wk.ccoff[pr + 1];
         }
         const int npc = wk.npieces;
         if (npc > 1) {
@@ -1046,8 +1088,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
               }
             }
           }
-          if (ce1 > ce0)
-            cc_accum(v, wk.ccent, ce0, ce1, wk.B, N, n0 + ucol(c0 / 32), ncols - c0);
+          if (ce1 > ce0)  // CUDA-core entries (f3)
+            cc_accum2(v, wk.ccent, ce0, ce1, wk.B, N, n0 + ucol(c0 / 32), ncols - c0);
           // Transposed through shared memory so that each store instruction
           // writes 8 rows x 64 contiguous bytes (4 lanes per row) instead of 32
           // rows x 16 bytes; 16-byte chunks swizzled by (row >> 1) & 3.
@@ -1153,7 +1195,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           }
           const int64_t lrow = (int64_t)p * 128 + rank * rpo + i;
           const int64_t colg = n0 + c8 * 8;
-          if (wk.ccent) {  // CUDA-core entries of this row (f3)
+          if (wk.ccp) {  // CUDA-core entries of this row (f3)
             const int e0 = wk.ccoff[lrow], e1 = wk.ccoff[lrow + 1];
             if (e1 > e0) cc_accum(acc, wk.ccent, e0, e1, wk.B, N, colg, 8);
           }
@@ -1379,7 +1421,7 @@ static void fill_problem(Prm& prm, int i, const Format& f, const void* dB, int64
   Problem& P = prm.pr[i];
   P.pin0 = i == 0 ? 0 : prm.pr[i - 1].pin0 + prm.pr[i - 1].npanels;
   if (P.pin0 + f.npanels <= Prm::kMaxPin)
-    std::copy(f.pin.begin(), f.pin.end(), prm.pin + P.pin0);
+    for (int64_t p = 0; p < f.npanels; ++p) prm.pin[P.pin0 + p] = f.pin_dev(p);
   else
     prm.use_pin = 0;
   P.Aimg = f.d_Aimg;
@@ -1631,7 +1673,7 @@ jigsaw_status_t launch_spmm(const Format& f, const void* dB, int64_t N, void* dC
       const int4 pi = f.pin[p];  // {k-steps, first k-step, first E block, dense k-steps}
       const int nkb = (pi.x + 3) / 4 + (pi.w + 3) / 4;
       prm.ctab[c][0] = make_int4(p, n0, r * nkb / S, (r + 1) * nkb / S);
-      prm.ctab[c][1] = make_int4(pi.x, pi.w, pi.y, pi.z);
+      prm.ctab[c][1] = make_int4(pi.x, f.pin_dev(p).w, pi.y, pi.z);
     }
     prm.use_ctab = 1;
   }
@@ -1800,6 +1842,15 @@ static jigsaw_status_t launch_group(const Format* const* fs, const void* const* 
           maxlen = std::max(maxlen, q[h.second].size());
           std::push_heap(heap.begin(), heap.end(), cmp);
         }
+        // Units of panels with CUDA-core entries (f3) go first in their slot's
+        // queue: their epilogue (the entries' B loads) then overlaps the next
+        // units' mainloops instead of extending the slot's tail.  The set of
+        // units per slot -- the LPT balance -- is unchanged.
+        for (auto& qc : q)
+          std::stable_partition(qc.begin(), qc.end(), [&](uint32_t code) {
+            const Format& f = *fs[i0 + (int)(code >> 26)];
+            return !f.ccT.empty() && f.ccT[((code >> 15) & 0x7FFu) % f.npanels] > 0;
+          });
         if (JIG_DEV && kn.debug_sched) {
           int64_t lo = INT64_MAX, hi = 0;
           for (const auto& h : heap) lo = std::min(lo, h.first), hi = std::max(hi, h.first);
