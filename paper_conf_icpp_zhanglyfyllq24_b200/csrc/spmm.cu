@@ -478,7 +478,61 @@ __device__ __forceinline__ void cc_accum2(T (&acc)[32], const int2* __restrict__
   }
 }
 
-template <int NT, bool kSplit, bool kPair, class Prm>
+// Adds the CUDA-core entries of the warp's 32 rows (lane = row; panel-row index
+// pr) to the fp32 accumulator in TMEM (taddr: the warp's lane quarter, column 0
+// of the unit's buffer): tcgen05.ld -> FMAs -> tcgen05.st per 32 columns.
+__device__ __noinline__ void cc_tmem_add(uint32_t taddr, int ncols, const int32_t* __restrict__ ccoff,
+                                         const int2* __restrict__ ent, const __half* __restrict__ B, int64_t N,
+                                         int64_t n0, int64_t pr) {
+  const int e0 = ccoff[pr], e1 = ccoff[pr + 1];
+  if (!__any_sync(kFullMask, e1 > e0)) return;
+  for (int c0 = 0; c0 < ncols; c0 += 32) {
+    uint32_t v[32];
+    tc_ld_32x32b_x32(taddr + (uint32_t)c0, v);
+    tc_wait_ld();
+    if (e1 > e0) cc_accum2(v, ent, e0, e1, B, N, n0 + c0, ncols - c0);
+    tc_st_32x32b_x32(taddr + (uint32_t)c0, v);
+    tc_wait_st();
+  }
+}
+
+// A unit whose panel has no tensor-core tile (every tile moved to the CUDA
+// cores): this lane's C row (crow, -1: a padding row) is the sum of its
+// entries, written directly (fp16 RN or fp32), 32 columns at a time.
+__device__ __noinline__ void cc_only_store(void* C, int c32, int64_t crow, int ncols, int64_t N, int64_t n0,
+                                           const int32_t* __restrict__ ccoff, const int2* __restrict__ ent,
+                                           const __half* __restrict__ B, int64_t pr) {
+  const int e0 = ccoff[pr], e1 = ccoff[pr + 1];
+  for (int c0 = 0; c0 < ncols; c0 += 32) {
+    float v[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) v[j] = 0.f;
+    if (e1 > e0) cc_accum2(v, ent, e0, e1, B, N, n0 + c0, ncols - c0);
+    if (crow < 0) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int64_t col = n0 + c0 + 8 * j;
+      if (8 * j >= ncols - c0 || col >= N) continue;
+      if (c32) {
+        float4* dst = reinterpret_cast<float4*>(static_cast<float*>(C) + crow * N + col);
+        dst[0] = make_float4(v[8 * j], v[8 * j + 1], v[8 * j + 2], v[8 * j + 3]);
+        dst[1] = make_float4(v[8 * j + 4], v[8 * j + 5], v[8 * j + 6], v[8 * j + 7]);
+      } else {
+        uint4 pk;
+        pk.x = pack_h2(v[8 * j], v[8 * j + 1]);
+        pk.y = pack_h2(v[8 * j + 2], v[8 * j + 3]);
+        pk.z = pack_h2(v[8 * j + 4], v[8 * j + 5]);
+        pk.w = pack_h2(v[8 * j + 6], v[8 * j + 7]);
+        *reinterpret_cast<uint4*>(static_cast<__half*>(C) + crow * N + col) = pk;
+      }
+    }
+  }
+}
+
+// kCC: the launch has CUDA-core entries (f3).  A separate instantiation, so the
+// launches without them run the epilogue without the entry code (inlined or as a
+// call, it cost C4 1-1.5 %: profiles/r02ab_*).
+template <int NT, bool kSplit, bool kPair, class Prm, bool kCC>
 __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
   static_assert(!(kSplit && kPair), "split-K and CTA pairs are separate variants");
   using C_ = Cfg<NT, kSplit, kPair>;
@@ -980,19 +1034,33 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       const int r = q * 32 + lane;                       // row of the panel (= TMEM lane)
       const int a = it % C_::kAccBufs;
       const int ncols = wk.ncols;                        // C columns of this unit
-      // CUDA-core entries of this lane's row (f3): fetched, and their B row
-      // segments prefetched into L2, while the accumulator is still being built
-      int ce0 = 0, ce1 = 0;
-      if (!kSplit && wk.ccp) {
-        const int64_t pr = wk.row0 + q * 32 + lane;  // padded panel-row index
-        ce0 = wk.ccoff[pr];
-        ce1 = wk.ccoff[pr + 1];
-        for (int e = ce0; e < ce1 && e < ce0 + 8; ++e)
-          bulk_prefetch_l2(wk.B + (int64_t)__ldg(wk.ccent + e).x * N + n0, (uint32_t)ncols * 2u);
+      if (kCC && !kSplit && wk.ccp) {
+        // CUDA-core entries of this lane's row (f3): their B row segments are
+        // prefetched into L2 while the accumulator is still being built
+        const int64_t pr = wk.row0 + q * 32 + lane;
+        const int e0 = wk.ccoff[pr], e1 = wk.ccoff[pr + 1];
+        for (int e = e0; e < e1 && e < e0 + 8; ++e)
+          bulk_prefetch_l2(wk.B + (int64_t)__ldg(wk.ccent + e).x * N + n0, (uint32_t)wk.ncols * 2u);
       }
       if (has_acc) {
         mbar_wait(&tfull[a], (uint32_t)(it / C_::kAccBufs) & 1);
         tc_fence_after();
+      }
+      // CUDA-core entries (f3, kCC launches only): added into the TMEM
+      // accumulator once per unit (piece 0 of a k-range split), or -- a panel
+      // with no tensor-core tile -- written to C directly
+      bool cc_done = false;
+      if (kCC && !kSplit && wk.ccp) {
+        const int64_t pr = wk.row0 + q * 32 + lane;  // padded panel-row index
+        if (has_acc) {
+          if (wk.piece == 0)
+            cc_tmem_add(tbase + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * C_::kAccCols), wk.ncols, wk.ccoff,
+                        wk.ccent, wk.B, N, n0, pr);
+        } else if (wk.npieces == 1) {
+          cc_only_store(wk.C, wk.c32, pr < M ? (wk.rowmap ? (int64_t)wk.rowmap[pr] : pr) : -1, wk.ncols, N, n0,
+                        wk.ccoff, wk.ccent, wk.B, pr);
+          cc_done = true;
+        }
       }
       // 32-column chunk k of the unit: its TMEM column and its C column offset
       auto tcol = [&](int k) -> uint32_t { return (uint32_t)(a * C_::kAccCols + 32 * k); };
@@ -1010,7 +1078,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       if (warp == 2 && lane == 0 && it == 0) JIG_TRACE(6);
       if constexpr (!kSplit) {
         const uint32_t stg = smem_u32(sC + q * (32 * 64));
-        bool write_c = true;
+        bool write_c = !cc_done;
         // C rows of the 4 rows this lane stores (rr = 8i + lane / 4 of the warp's
         // 32): row-clustered panels scatter panel row r to C row rowmap[r]; once
         // per unit, outside the store loop (M < 2^31 by validation)
@@ -1088,8 +1156,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
               }
             }
           }
-          if (ce1 > ce0)  // CUDA-core entries (f3)
-            cc_accum2(v, wk.ccent, ce0, ce1, wk.B, N, n0 + ucol(c0 / 32), ncols - c0);
           // Transposed through shared memory so that each store instruction
           // writes 8 rows x 64 contiguous bytes (4 lanes per row) instead of 32
           // rows x 16 bytes; 16-byte chunks swizzled by (row >> 1) & 3.
@@ -1195,7 +1261,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           }
           const int64_t lrow = (int64_t)p * 128 + rank * rpo + i;
           const int64_t colg = n0 + c8 * 8;
-          if (wk.ccp) {  // CUDA-core entries of this row (f3)
+          if (kCC && wk.ccp) {  // CUDA-core entries of this row (f3)
             const int e0 = wk.ccoff[lrow], e1 = wk.ccoff[lrow + 1];
             if (e1 > e0) cc_accum(acc, wk.ccent, e0, e1, wk.B, N, colg, 8);
           }
@@ -1292,12 +1358,13 @@ const Knobs& knobs() {
   }();
   return k;
 }
-std::atomic<bool> g_attr_set[64][16] = {};  // [device][variant]
+std::atomic<bool> g_attr_set[64][32] = {};  // [device][variant (+16: kCC)]
 
-template <int NT, bool kSplit, bool kPair, class Prm>
+template <int NT, bool kSplit, bool kPair, bool kCC, class Prm>
 jigsaw_status_t launch_variant(const Prm& prm, int grid, int S, int dev, int vid, cudaStream_t s) {
   using C_ = Cfg<NT, kSplit, kPair>;
-  auto kern = k_spmm<NT, kSplit, kPair, Prm>;
+  auto kern = k_spmm<NT, kSplit, kPair, Prm, kCC>;
+  vid += kCC ? 16 : 0;
   if (dev >= 0 && dev < 64 && !g_attr_set[dev][vid].load(std::memory_order_acquire)) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::kSmem);
     if (e != cudaSuccess) return cuda_status(e, "cudaFuncSetAttribute(k_spmm)");
@@ -1562,6 +1629,23 @@ static void set_workspace(Prm& prm, const Workspace& w) {
 // Launches k_spmm for the parameter block.  `pslots` split-piece slots of
 // `tile_bytes` each need workspace; the dynamic scheduler is used when a
 // single-CTA launch has more units than CTAs.
+// The kernel instantiation for a launch shape (tile width, split-K, CTA pairs).
+template <bool kCC, class Prm>
+static jigsaw_status_t launch_shape(const Prm& prm, int NT, int S, int grid, int dev, bool pair, int vb,
+                                    cudaStream_t s) {
+  if (pair)
+    return NT == 256 ? launch_variant<256, false, true, kCC>(prm, grid, 2, dev, vb + 5, s)
+                     : launch_variant<128, false, true, kCC>(prm, grid, 2, dev, vb + 4, s);
+  if (NT == 256) return launch_variant<256, false, false, kCC>(prm, grid, 1, dev, vb + 3, s);
+  if (NT == 128) return launch_variant<128, false, false, kCC>(prm, grid, 1, dev, vb + 0, s);
+  if (NT == 32 && S == 1) return launch_variant<32, false, false, kCC>(prm, grid, 1, dev, vb + 6, s);
+  if (S == 1) return launch_variant<64, false, false, kCC>(prm, grid, 1, dev, vb + 1, s);
+  if constexpr (std::is_same<Prm, ParamsOne>::value)
+    return NT == 32 ? launch_variant<32, true, false, kCC>(prm, grid, S, dev, vb + 7, s)
+                    : launch_variant<64, true, false, kCC>(prm, grid, S, dev, vb + 2, s);
+  return set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
+}
+
 template <class Prm>
 static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev, bool pair, cudaStream_t s,
                                      int npieces_total = -1, int pslots = 0, size_t tile_bytes = 0) {
@@ -1603,23 +1687,10 @@ static jigsaw_status_t launch_params(Prm& prm, int NT, int S, int grid, int dev,
   d.graph_owned_workspace = w.graph_owned ? 1 : 0;
   d.launches += 1;
   constexpr int vb = std::is_same<Prm, ParamsOne>::value ? 0 : 8;
-  jigsaw_status_t st;
-  if (pair)
-    st = NT == 256 ? launch_variant<256, false, true>(prm, grid, 2, dev, vb + 5, s)
-                   : launch_variant<128, false, true>(prm, grid, 2, dev, vb + 4, s);
-  else if (NT == 256)
-    st = launch_variant<256, false, false>(prm, grid, 1, dev, vb + 3, s);
-  else if (NT == 128)
-    st = launch_variant<128, false, false>(prm, grid, 1, dev, vb + 0, s);
-  else if (NT == 32 && S == 1)
-    st = launch_variant<32, false, false>(prm, grid, 1, dev, vb + 6, s);
-  else if (S == 1)
-    st = launch_variant<64, false, false>(prm, grid, 1, dev, vb + 1, s);
-  else if constexpr (std::is_same<Prm, ParamsOne>::value)
-    st = NT == 32 ? launch_variant<32, true, false>(prm, grid, S, dev, vb + 7, s)
-                  : launch_variant<64, true, false>(prm, grid, S, dev, vb + 2, s);
-  else
-    st = set_status(JIGSAW_ERROR_INTERNAL, "split-K is only built for single products");
+  bool cc = false;  // some product of the launch has CUDA-core entries (f3)
+  for (int i = 0; i < prm.nprob; ++i) cc = cc || prm.pr[i].ccent != nullptr;
+  jigsaw_status_t st = cc ? launch_shape<true>(prm, NT, S, grid, dev, pair, vb, s)
+                          : launch_shape<false>(prm, NT, S, grid, dev, pair, vb, s);
   if (w.graph_owned) {
     cudaError_t e = cudaFreeAsync(w.base, s);  // free node right after the kernel node
     if (st == JIGSAW_SUCCESS && e != cudaSuccess) st = cuda_status(e, "workspace free node");
