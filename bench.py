@@ -52,6 +52,16 @@ import synth  # noqa: E402
 
 METRIC = "SpMM effective TFLOP/s and speedup vs cuBLAS fp16 GEMM vs sparsity, v=2/4/8"
 FLUSH_BYTES = 256 << 20
+# The paper's own speedups over cuBLAS HGemm (average / max over the DLMC
+# matrices), NVIDIA A100 40 GB, fp16 -- PAPER.md Table 2, quoted as
+# context only (other GPU, other matrices, other baseline build).
+PAPER_TABLE2 = {
+    "source": "PAPER.md Table 2 (P:244-259): Jigsaw vs cuBLAS HGemm, A100 40 GB, DLMC, fp16 (avg, max)",
+    "v2_s80": [0.77, 1.27], "v4_s80": [0.89, 1.34], "v8_s80": [1.00, 1.67],
+    "v2_s90": [1.00, 1.58], "v4_s90": [1.13, 1.95], "v8_s90": [1.35, 1.85],
+    "v2_s95": [1.19, 1.73], "v4_s95": [1.44, 2.83], "v8_s95": [1.78, 4.12],
+    "v2_s98": [1.43, 1.89], "v4_s98": [1.72, 4.14], "v8_s98": [2.14, 5.45],
+}
 
 
 # ------------------------------------------------------------------ workloads
@@ -518,6 +528,7 @@ def cublas_compare(b: Batch, flush, stream, torch, jig, jig_step_ms, steps, warm
         tj_sum += tj
         tc_sum += tc
     out["speedup_geomean_by_v_s"] = {k: float(np.exp(np.mean(np.log(x)))) for k, x in sorted(sp.items())}
+    out["paper_context"] = PAPER_TABLE2
     out["per_matrix_speedup_total_time"] = tc_sum / tj_sum
     out["per_matrix_how"] = ("each product alone: jigsaw_spmm vs cublasGemmEx (best of COMPUTE_16F / 32F) on "
                              "the dense A, [graph of 8 x (L2 flush, call)] - [graph of 8 x flush], / 8, median of 7")
