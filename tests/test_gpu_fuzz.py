@@ -1,7 +1,9 @@
 """Seeded randomised GPU parity sweep over the option / launch-shape matrix:
 shape (ragged M, K, N), v, sparsity, mask kind, panel height, residual mode,
 C element type, row order, and a forced launch shape (tile width, split-K,
-piece mode) -- each configuration's format bit-exact against the oracle on a
+piece mode), and (for half the seeds) a CUDA-core threshold cc_max_nnz taken
+from the configuration's own tile nonzero counts -- each configuration's format
+bit-exact against the oracle on a
 sampled panel and C within the north-star tolerance (integer inputs: exact).
 The interactions of the options, not each option alone (tested elsewhere)."""
 import numpy as np
@@ -15,6 +17,7 @@ pytestmark = pytest.mark.gpu
 
 import paper_conf_icpp_zhanglyfyllq24_b200 as jig  # noqa: E402
 from test_gpu_parity import _dev, _host, assert_format_equal, int_exact, spmm_check  # noqa: E402
+from test_gpu_cuda_core import tile_nnz  # noqa: E402
 
 
 @pytest.fixture(scope="module", autouse=True)
@@ -49,14 +52,25 @@ def test_fuzz_options(seed):
     M, K, N, v, s, kind, P, mode, c_dtype, row_order, ov = _config(seed)
     A = synth.vector_sparse(M, K, v, s, 3000 + seed, kind=kind)
     B = synth.dense_b(K, N, 3000 + seed, kind="int" if kind == "int" else "uniform")
-    h = jig.reorder(_dev(A), v, panel_rows=P, residual_mode=mode, c_dtype=c_dtype, row_order=row_order)
+    ref = oracle.reorder(A, P=P, mode=mode, row_order=row_order)
+    Ap = A[ref.rowmap] if row_order else A
+    Z = 0  # CUDA-core threshold (f3), from a separate stream so the other draws stay as they were
+    rc = np.random.default_rng(5000 + seed)
+    if rc.random() < 0.5 and int(ref.T.sum()) > 0:
+        cnt = np.sort(tile_nnz(Ap, ref))
+        Z = max(1, int(cnt[int(rc.integers(0, len(cnt)))]))
+    h = jig.reorder(_dev(A), v, panel_rows=P, residual_mode=mode, c_dtype=c_dtype, row_order=row_order,
+                    cc_max_nnz=Z)
     g = h.export()
     npan = (M + P - 1) // P
     p = seed % npan
-    ref = oracle.reorder(A, P=P, mode=mode, row_order=row_order)
     assert np.array_equal(g["rowmap"], ref.rowmap)
-    assert_format_equal(g, oracle.reorder(A[ref.rowmap] if row_order else A, P=P, mode=mode, panels=(p, p + 1)),
-                        panels=(p, p + 1))
+    sub = oracle.reorder(Ap, P=P, mode=mode, panels=(p, p + 1), cc_max_nnz=Z)
+    assert_format_equal(g, sub, panels=(p, p + 1))
+    assert g["cc_T"][p] == sub.cc_T[0]
+    e0, e1 = int(g["cc_eoff"][p]), int(g["cc_eoff"][p + 1])
+    for k in ("cc_row", "cc_col", "cc_val"):
+        assert np.array_equal(g[k][e0:e1], getattr(sub, k)), k
     with jig.launch_override(**ov):
         C = h.spmm(_dev(B))
         torch.cuda.synchronize()
