@@ -141,6 +141,7 @@ __global__ void k_compact(const RowMask* __restrict__ masks, int64_t K, int32_t*
 constexpr int kMaxBig = 256;
 struct TileSmem {
   uint32_t bitmap[2048];  // compat[S] for every 4-subset S, indexed by the 16-bit slot mask
+  uint32_t half[2048];    // cover_dp: 8-slot unions g0 | g1 of two disjoint compatible groups
   uint16_t big[kMaxBig];  // compatible 3- and 4-subsets of the real slots (existence test)
   int nbig;
   RowMask m[16];          // row masks per slot (PAD: 0)
@@ -199,14 +200,70 @@ __device__ bool complete_cover(const TileSmem& s, uint32_t used, uint32_t& o1, u
   return false;
 }
 
+// Exact existence test for a cover of all 16 slots by 4 disjoint compatible
+// groups, by levels (the oracle's DFS memoises dead used-sets instead; both only
+// decide existence): level 2 marks every union g0 | g1 of a compatible group g0
+// holding slot 0 and a compatible g1 holding the smallest slot outside g0 (at
+// most C(16,8) distinct 8-slot sets, deduplicated in a bitmap); a cover exists
+// iff the 8 remaining slots of some marked set split into two compatible groups
+// (the one holding their smallest slot, and the rest).  Work is bounded
+// (<= 455 x 165 level-2 checks, <= 12870 x 35 level-3 checks per warp), unlike
+// the depth-first search of complete_cover when no cover exists.
+__device__ bool cover_dp(TileSmem& s, uint32_t realset, int hmax, int lane) {
+  for (int i = lane; i < 2048; i += 32) s.half[i] = 0;
+  __syncwarp();
+  for (int k = lane; k < kNumG0; k += 32) {
+    const uint32_t g0 = g_subs[k];
+    // (exact pruning, as in complete_cover: no compatible group holds more than
+    // hmax real columns, so the real columns left must fit hmax per group)
+    if (!compat(s, g0) || __popc(realset & ~g0) > 3 * hmax) continue;
+    const int l1 = __ffs(~g0 & 0xFFFFu) - 1;
+    const uint32_t av = ~g0 & 0xFFFFu & ~(1u << l1);
+    for (uint32_t x = av; x; x &= x - 1) {
+      const uint32_t bb = x & (0u - x);
+      for (uint32_t y = x & (x - 1); y; y &= y - 1) {
+        const uint32_t cb = y & (0u - y);
+        for (uint32_t z = y & (y - 1); z; z &= z - 1) {
+          const uint32_t g1 = (1u << l1) | bb | cb | (z & (0u - z));
+          if (compat(s, g1) && __popc(realset & ~(g0 | g1)) <= 2 * hmax) {
+            const uint32_t u = g0 | g1;
+            atomicOr(&s.half[u >> 5], 1u << (u & 31));
+          }
+        }
+      }
+    }
+  }
+  __syncwarp();
+  bool found = false;
+  for (int w = lane; w < 2048 && !__any_sync(kFull, found); w += 32) {
+    for (uint32_t bits = s.half[w]; bits && !found; bits &= bits - 1) {
+      const uint32_t u = (uint32_t)w * 32u + (uint32_t)(__ffs(bits) - 1);
+      const uint32_t rest = ~u & 0xFFFFu;
+      const int l2 = __ffs(rest) - 1;
+      const uint32_t av = rest & ~(1u << l2);
+      for (uint32_t x = av; x && !found; x &= x - 1) {
+        const uint32_t bb = x & (0u - x);
+        for (uint32_t y = x & (x - 1); y && !found; y &= y - 1) {
+          const uint32_t cb = y & (0u - y);
+          for (uint32_t z = y & (y - 1); z && !found; z &= z - 1) {
+            const uint32_t g2 = (1u << l2) | bb | cb | (z & (0u - z));
+            if (compat(s, g2) && compat(s, rest & ~g2)) found = true;
+          }
+        }
+      }
+    }
+  }
+  return __any_sync(kFull, found) != 0;
+}
+
 // Exact existence test for a cover (used to skip exhaustive searches that must
 // fail; it never changes WHICH cover is chosen).  PAD slots are interchangeable
 // zero columns and any group with <= 2 real columns is compatible, so a cover
 // exists iff some k <= 4 disjoint compatible "big" groups (3 or 4 real columns)
 // hold enough real columns that the rest fits 2 per remaining group:
-// sum(|b_i| - 2) >= nreal - 8.  Falls back to "maybe" (true) when the
-// candidate list or the search budget overflows.
-__device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
+// sum(|b_i| - 2) >= nreal - 8.  When the candidate list or the search budget
+// overflows, the level-wise exact test cover_dp decides.
+__device__ bool cover_exists(TileSmem& s, uint32_t realset, int hmax, int lane) {
   if (lane == 0) {
     s.nbig = 0;
     s.stop = 0;
@@ -241,13 +298,14 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
   // common case once a tile has more than 8 hard columns -- is exhausted 32
   // lanes at a time instead of by one thread
   int found = 0;
+  bool maybe = false;
   const int n = s.nbig, need = __popc(realset) - 8;
   if (n > kMaxBig) {
-    found = 1;
+    maybe = true;
   } else {
     int budget = 1 << 13;  // per lane; exceeding it answers "maybe" (exactness kept)
     volatile int* stop = &s.stop;
-    for (int i0 = lane; i0 < n && !found && !*stop; i0 += 32) {
+    for (int i0 = lane; i0 < n && !found && !maybe && !*stop; i0 += 32) {
       const uint32_t b0 = s.big[i0];
       int idx[3];
       uint32_t used[4];
@@ -258,7 +316,7 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
       int d = 0;
       idx[0] = i0 + 1;
       while (d >= 0) {
-        if (--budget < 0) { found = 1; break; }
+        if (--budget < 0) { maybe = true; break; }
         if ((budget & 63) == 0 && *stop) break;  // another lane already answered
         if (idx[d] >= n) {                    // level exhausted: backtrack
           --d;
@@ -272,10 +330,13 @@ __device__ bool cover_exists(TileSmem& s, uint32_t realset, int lane) {
         if (exc[d + 1] >= need) { found = 1; break; }
         if (d + 1 < 3) { idx[d + 1] = idx[d] + 1; ++d; } else { ++idx[d]; }
       }
-      if (found) *stop = 1;
+      if (found || maybe) *stop = 1;  // answered (or inconclusive: the exact test decides)
     }
   }
-  return __any_sync(kFull, found) != 0;
+  if (__any_sync(kFull, found)) return true;
+  // inconclusive (candidate list or search budget exceeded): the exact test below
+  if (__any_sync(kFull, maybe)) return cover_dp(s, realset, hmax, lane);
+  return false;
 }
 
 // Alg. 1 + reorder retry on one tile, executed by one full warp.  On entry
@@ -343,8 +404,11 @@ __device__ void tile_search(TileSmem& s, int lane) {
     // every slot lies in some compatible group; 4 groups can hold all real columns.
     bool coverable = __all_sync(kFull, lane >= 16 || fr > 0) && hmax * 4 >= __popc(realset);
     const int nreal = __popc(realset);
-    if (nreal > 8) {
-      const bool ex = cover_exists(s, realset, lane);
+    // (hmax >= 3 and a necessary condition already failed: no cover, and some
+    // compatible group holds 3+ real columns, so the shortcut below cannot apply --
+    // the existence test is skipped, the result is the same)
+    if (nreal > 8 && (hmax < 3 || coverable)) {
+      const bool ex = cover_exists(s, realset, hmax, lane);
       if (s.nbig == 0) {
         // No compatible group holds 3+ real columns, and none will after more
         // evictions: every real column is in the same number of compatible groups
@@ -432,7 +496,7 @@ __device__ void store_tile(const TileSmem& s, const Scratch& sc, int p, int t, i
 }
 
 // ------------------------------------------------------------------ R3
-constexpr int kR3Warps = 4;
+constexpr int kR3Warps = 2;  // 2 x sizeof(TileSmem) (~17.6 KB) of static shared memory
 __global__ void __launch_bounds__(32 * kR3Warps) k_main_tiles(const RowMask* __restrict__ masks,
                                                               const int32_t* __restrict__ S,
                                                               const int32_t* __restrict__ Kp,
