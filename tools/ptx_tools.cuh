@@ -6,6 +6,16 @@
 #include "../paper_conf_icpp_zhanglyfyllq24_b200/csrc/ptx.cuh"
 
 namespace jig {
+// Non-blocking parity test of an mbarrier phase.
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
 // Wait with back-off (mbar_test polling).
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, uint32_t ns) {
   while (!mbar_test(bar, parity)) __nanosleep(ns);
