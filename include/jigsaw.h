@@ -293,7 +293,7 @@ JIGSAW_API jigsaw_status_t jigsaw_last_launch(jigsaw_launch_desc_t* out);
  * the library's choice.  Fields: tile_n (0 or 32/64/128/256 columns per unit),
  * split_k (0 or 1/2/4/8: single products of 128-row panels on split-K clusters
  * of that size, tile 64 or 32), no_pieces (1: no k-range pieces in grouped
- * launches), host_chunks (0 = 16, else the chunk count of
+ * launches), host_chunks (0 = library choice: ~6 MB chunks, 2..16; else the chunk count of
  * jigsaw_spmm_batched_host), k_pieces (1: split long units of grouped launches
  * into k-range pieces reduced through the workspace, instead of the default
  * column slices).  Results are identical up to fp32 summation order. */

@@ -320,6 +320,11 @@ def debug_trace(max_ctas: int = 1024) -> np.ndarray:
     return out[:n]
 
 
+def _addr(x: np.ndarray) -> int:
+    """Data address of a host array (cheaper than ``x.ctypes.data``)."""
+    return x.__array_interface__["data"][0]
+
+
 def spmm_batched_host(handles, Bs, outs=None, stream=None):
     """jigsaw_spmm_batched_host: the batch with host B's in and host C's out
     (pinned arrays, e.g. from torch pin_memory, let the copies overlap)."""
@@ -327,18 +332,17 @@ def spmm_batched_host(handles, Bs, outs=None, stream=None):
     if len(Bs) != n or (outs is not None and len(outs) != n):
         raise ValueError("handles, Bs and outs must have the same length")
     Bs = [_host16(b, "B") for b in Bs]
-    for h, b in zip(handles, Bs):
-        if b.shape[0] != h.K:
-            raise ValueError(f"B has {b.shape[0]} rows, A has K = {h.K}")
     if outs is None:
         outs = [np.empty((h.M, b.shape[1]), dtype=h.c_numpy_dtype) for h, b in zip(handles, Bs)]
     for h, b, c in zip(handles, Bs, outs):
+        if b.shape[0] != h.K:
+            raise ValueError(f"B has {b.shape[0]} rows, A has K = {h.K}")
         if (c.shape != (h.M, b.shape[1]) or not c.flags.c_contiguous
-                or c.itemsize != np.dtype(h.c_numpy_dtype).itemsize):
+                or c.itemsize != (4 if h.c_dtype == C_F32 else 2)):
             raise ValueError("each out must be a contiguous M x N array of its handle's C element size")
-    hs = (ctypes.c_void_p * n)(*[h.ptr.value for h in handles])
-    bp = (ctypes.c_void_p * n)(*[b.ctypes.data for b in Bs])
-    cp = (ctypes.c_void_p * n)(*[c.ctypes.data for c in outs])
+    hs = (ctypes.c_void_p * n)(*[h._h.value for h in handles])
+    bp = (ctypes.c_void_p * n)(*[_addr(b) for b in Bs])
+    cp = (ctypes.c_void_p * n)(*[_addr(c) for c in outs])
     ns = (ctypes.c_int64 * n)(*[b.shape[1] for b in Bs])
     _raise_if(lib().jigsaw_spmm_batched_host(hs, bp, ns, cp, n, _stream_ptr(stream) if stream is not None else None))
     return outs

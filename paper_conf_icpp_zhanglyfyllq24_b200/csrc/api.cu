@@ -588,7 +588,11 @@ static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_hand
   // override jigsaw_set_launch_override host_chunks): copy-in of chunk k+1 and copy-out of chunk
   // k-1 overlap the grouped launch of chunk k (16 measured best with one copy
   // per product and direction, profiles/r01zt_e2e_chunks.txt)
-  const int nchunks = launch_override().host_chunks > 0 ? launch_override().host_chunks : 16;
+  // chunk count: ~6 MB chunks, 2..16 (per-copy costs ~6 us on this link: C2's
+  // 47 MB run best in 8 chunks, C4's 382 MB in 16; profiles/r02_e2e_floor*.jsonl)
+  const int nchunks = launch_override().host_chunks > 0
+                          ? launch_override().host_chunks
+                          : (int)std::min<size_t>(16, std::max<size_t>(2, ((bb + cb) + (3u << 20)) / (6u << 20)));
   const size_t target = std::max<size_t>((bb + cb) / nchunks, 1);
   std::vector<const Format*> fs;
   std::vector<const void*> pb;
@@ -596,13 +600,30 @@ static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_hand
   std::vector<void*> pc;
   jigsaw_status_t st = JIGSAW_SUCCESS;
   std::vector<cudaEvent_t> evs;
-  for (int i0 = 0; i0 < count && st == JIGSAW_SUCCESS;) {
+  // Chunks are runs of consecutive products (so packed host buffers still merge
+  // into one copy per chunk and direction), taken alternately from the front and
+  // the back of the batch: a batch ordered from B-heavy to C-heavy products (the
+  // C2 batch: 512 x 2048 products, then 2048 x 512) otherwise keeps one copy
+  // direction idle for half of the call -- with the ends interleaved both
+  // directions of the link stay busy (C2: 0.92 -> see DESIGN.md §8).
+  std::vector<std::pair<int, int>> runs;
+  for (int i0 = 0; i0 < count;) {
     int i1 = i0;
     size_t acc = 0;
     while (i1 < count && (i1 == i0 || acc < target)) {
       acc += (size_t)hs[i1]->f.K * Ns[i1] * 2 + (size_t)hs[i1]->f.M * Ns[i1] * c_elem_bytes(hs[i1]->f);
       ++i1;
     }
+    runs.push_back({i0, i1});
+    i0 = i1;
+  }
+  std::vector<std::pair<int, int>> order;
+  for (size_t lo = 0, hi = runs.size(); lo < hi;) {
+    order.push_back(runs[lo++]);
+    if (lo < hi) order.push_back(runs[--hi]);
+  }
+  for (size_t r = 0; r < order.size() && st == JIGSAW_SUCCESS; ++r) {
+    const int i0 = order[r].first, i1 = order[r].second;
     std::vector<void*> cd, cs;
     std::vector<size_t> cz;
     std::vector<char> jn;
@@ -638,7 +659,6 @@ static jigsaw_status_t spmm_batched_host_on(const HostPipe& P, const jigsaw_hand
       jn.push_back(i > i0 && cjoin[i]);
     }
     if (e == cudaSuccess && st == JIGSAW_SUCCESS) e = copy_batch(cd, cs, cz, jn, cudaMemcpyDeviceToHost, P.d2h);
-    i0 = i1;
   }
   // staging goes back to the pool after the last copy-out
   cudaEvent_t fin;
