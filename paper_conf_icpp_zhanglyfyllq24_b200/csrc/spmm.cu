@@ -56,6 +56,9 @@
 #ifndef JIG_DEV
 #define JIG_DEV 0  // developer build (-DJIG_DEV=1): timing-only JIGSAW_DBG modes and schedule experiments
 #endif
+#ifndef JIG_AE_SPLIT
+#define JIG_AE_SPLIT 1  // static schedules: metadata copies on warp 9, gather lists on warp 13 (else all on warp 0)
+#endif
 
 namespace jig {
 
@@ -589,7 +592,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       }
     }
   };
-  if (warp >= 2 && warp <= 5) decode_first();
+  // Static schedules split warp 0's per-k-block issue work (each mbarrier /
+  // bulk-copy operation costs ~100 cycles from one thread, and warp 0 paced the
+  // k-blocks: its copies left ~1,000 cycles after the B producers saw the same
+  // free stage, profiles/r02ac_kblock_timeline_c4.txt): warp 0 the compressed A,
+  // warp 9 the metadata blocks, warp 13 the gather-list ring (9 and 13 were idle).
+  const bool split_ae = JIG_AE_SPLIT && JIG_SPARE_SMSP1 && !dyn;
+  if ((warp >= 2 && warp <= 5) || (split_ae && (warp == 9 || warp == 13))) decode_first();
 
   // Barrier initialisation spread over the lanes of warp 0 (~50 barriers; one
   // thread initialising them all costs ~0.5 us of kernel start).  The barriers
@@ -600,7 +609,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     for (int i = lane; i < nb; i += 32) {
       int k = i;
       uint32_t cnt;
-      if (k < C_::kStages) cnt = 1 + 32 * C_::kWPG;        // full: A/E expect_tx + the B group's cp.async arrivals
+      if (k < C_::kStages) cnt = (split_ae ? 2 : 1) + 32 * C_::kWPG;  // full: A (and E) expect_tx + the B group's cp.async
       else if ((k -= C_::kStages) < C_::kStages) cnt = 1;  // empty
       else if ((k -= C_::kStages) < C_::kGS) cnt = 1;      // gfull
       else if ((k -= C_::kGS) < C_::kGS) cnt = C_::kWPG;   // gempty
@@ -659,6 +668,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
         mbar_arrive_expect_tx(&full[l], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
         bulk_g2s(sA + l * kStageA, w0.Aimg + w0.gks(kb) * kKStepBytesA, steps * kKStepBytesA, &full[l]);
         if (!dense) bulk_g2s(sE + l * kStageE, w0.Eimg + (w0.kb0 + kb) * kEBlockBytes, kStageE, &full[l]);
+        if (split_ae) mbar_arrive(&full[l]);  // the metadata warp's arrival for this stage
       }
       if (warp == 3 && nA0 > 0) JIG_TRACE(2);
     }
@@ -777,13 +787,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
             bulk_prefetch_l2(wk.Eimg + (kb0 + wk.kb_lo) * kEBlockBytes, (uint32_t)(kbe - wk.kb_lo) * kEBlockBytes);
         }
         for (int kb = wk.kb_lo + (mq == 1 ? nA0 : 0); kb < wk.kb_hi; ++kb) {
-          g_issue_upto(mi + 1 + C_::kGAhead);
+          if (!split_ae) g_issue_upto(mi + 1 + C_::kGAhead);
           const int steps = wk.steps(kb);
           const bool dense = wk.dense(kb);
           const int64_t gks = wk.gks(kb);
           mbar_wait(&empty[stage], phase ^ 1);
           if (JIG_DEV && (prm.dbg & 16)) {  // timing only: no A / metadata loads
             mbar_arrive(&full[stage]);
+          } else if (split_ae) {
+            mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA));
+            bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
           } else {
             mbar_arrive_expect_tx(&full[stage], (uint32_t)(steps * kKStepBytesA + (dense ? 0 : kStageE)));
             bulk_g2s(sA + stage * kStageA, wk.Aimg + gks * kKStepBytesA, steps * kKStepBytesA, &full[stage]);
@@ -809,6 +822,52 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
       // workspace / scheduler accesses still wait for this grid to complete.
       if (JIG_EARLY_TRIGGER == 1) griddep_launch_dependents();
     }
+  } else if (split_ae && warp == 9) {
+    // ------------------------------------------------------------ metadata producer (static schedules)
+    // The same (unit, k-block) sequence and stage ring as warp 0: per k-block one
+    // metadata bulk copy (its own expect_tx), or a plain arrival for a DENSE
+    // k-block; the first unit's first nA0 stages were filled by the initial fill.
+    if (lane == 0) {
+      int stage = nA0 % C_::kStages, hint = 0;
+      uint32_t phase = nA0 == C_::kStages ? 1u : 0u;
+      for (int us = cluster_id; us < prm.nunits; us += nclusters) {
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
+        if (!wk.valid) continue;
+        for (int kb = wk.kb_lo + (us == cluster_id ? nA0 : 0); kb < wk.kb_hi; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          if (wk.dense(kb) || (JIG_DEV && (prm.dbg & 16))) {
+            mbar_arrive(&full[stage]);
+          } else {
+            mbar_arrive_expect_tx(&full[stage], (uint32_t)kStageE);
+            bulk_g2s(sE + stage * kStageE, wk.Eimg + (wk.kb0 + kb) * kEBlockBytes, kStageE, &full[stage]);
+          }
+          if (++stage == C_::kStages) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+    __syncwarp();
+  } else if (split_ae && warp == 13) {
+    // ------------------------------------------------------------ gather-list producer (static schedules)
+    // Fills the gather-list ring in (unit, k-block) order, paced only by the ring
+    // (kGS = 2 x stages slots freed by the B producers): the lists land long
+    // before their B rows are needed; the initial fill issued the
+    // first unit's first nG0 lists.
+    if (lane == 0) {
+      int gslot = nG0 % C_::kGS, hint = 0;
+      uint32_t gph = nG0 == C_::kGS ? 1u : 0u;
+      for (int us = cluster_id; us < prm.nunits; us += nclusters) {
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
+        if (!wk.valid) continue;
+        for (int kb = wk.kb_lo + (us == cluster_id ? nG0 : 0); kb < wk.kb_hi; ++kb) {
+          const int steps = wk.steps(kb);
+          mbar_wait(&gempty[gslot], gph ^ 1);
+          mbar_arrive_expect_tx(&gfull[gslot], (uint32_t)(steps * 128));
+          bulk_g2s(sG + gslot * kRowsPerBlock, wk.G + wk.gks(kb) * 32, steps * 128, &gfull[gslot]);
+          if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
+        }
+      }
+    }
+    __syncwarp();
   } else if (bprod_index(warp) >= 0) {
     // ------------------------------------------------------------ B producers
     // Group grp copies the B rows of the k-blocks j with j % kBGroups == grp; warp

@@ -30,6 +30,7 @@ __global__ void __launch_bounds__(512, 1) probe(const uint8_t* __restrict__ B, u
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t bars[16][4];
+  __shared__ uint64_t cbar[4];  // MODE 5: one CTA-wide barrier per batch slot
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // per warp: one 32-row x 256 B = 8 KB region, rewritten by every batch (the
   // contents do not matter here, only the throughput)
@@ -38,11 +39,15 @@ __global__ void __launch_bounds__(512, 1) probe(const uint8_t* __restrict__ B, u
     for (int d = 0; d < D; ++d) mbar_init(&bars[warp][d], 1);
   if (MODE == 4 && lane == 0)
     for (int d = 0; d < D; ++d) mbar_init(&bars[warp][d], 32);
+  if (MODE == 5 && threadIdx.x == 0)
+    for (int d = 0; d < D; ++d) mbar_init(&cbar[d], 32 * nwarps);
+  if (MODE == 6 && lane == 0)
+    for (int d = 0; d < D; ++d) mbar_init(&bars[warp][d], 1);
   fence_barrier_init();
   __syncthreads();
   const long long t0 = clock64();
   if (warp >= nwarps) {
-  } else if (MODE == 0 || MODE == 4) {
+  } else if (MODE == 0 || MODE == 4 || MODE == 5 || MODE == 6) {
     // 16 lanes per row: 2 rows per instruction, 16 instructions per 32-row batch
     const int c = lane & 15;
     for (int it = 0; it < kIters; ++it) {
@@ -54,11 +59,25 @@ __global__ void __launch_bounds__(512, 1) probe(const uint8_t* __restrict__ B, u
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(B + (size_t)g * pitch + c * 16)
                      : "memory");
       }
-      if (MODE == 4) {  // completion through an mbarrier (k_spmm's cp.async.mbarrier.arrive.noinc)
+      if (MODE == 4 || MODE == 5) {  // completion through an mbarrier (k_spmm's cp.async.mbarrier.arrive.noinc)
         const int s = it % D;
-        cp_async_mbar_arrive_noinc(&bars[warp][s]);
+        uint64_t* bb = MODE == 4 ? bars[warp] : cbar;
+        cp_async_mbar_arrive_noinc(&bb[s]);
         if (it >= D - 1) {
           const int so = (it - (D - 1)) % D;
+          mbar_wait(&bb[so], (uint32_t)(((it - (D - 1)) / D) & 1));
+        }
+        continue;
+      }
+      if (MODE == 6) {  // commit groups; one plain arrive per warp once a group has landed
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        if (it >= D - 1) {
+          if (D == 4) asm volatile("cp.async.wait_group 3;" ::: "memory");
+          else if (D == 2) asm volatile("cp.async.wait_group 1;" ::: "memory");
+          else asm volatile("cp.async.wait_group 0;" ::: "memory");
+          __syncwarp();
+          const int so = (it - (D - 1)) % D;
+          if (lane == 0) mbar_arrive(&bars[warp][so]);
           mbar_wait(&bars[warp][so], (uint32_t)(((it - (D - 1)) / D) & 1));
         }
         continue;
@@ -70,10 +89,10 @@ __global__ void __launch_bounds__(512, 1) probe(const uint8_t* __restrict__ B, u
         else asm volatile("cp.async.wait_group 0;" ::: "memory");
       }
     }
-    if (MODE == 0) asm volatile("cp.async.wait_group 0;" ::: "memory");
+    if (MODE == 0 || MODE == 6) asm volatile("cp.async.wait_group 0;" ::: "memory");
     else
       for (int it = kIters - (D - 1); it < kIters; ++it)
-        if (it >= 0) mbar_wait(&bars[warp][it % D], (uint32_t)((it / D) & 1));
+        if (it >= 0) mbar_wait(MODE == 4 ? &bars[warp][it % D] : &cbar[it % D], (uint32_t)((it / D) & 1));
   } else if (MODE == 1 || MODE == 2) {
     // each lane loads D 16-byte pieces (rows r = 2i + lane/16) before storing them
     const int c = lane & 15;
@@ -150,23 +169,18 @@ void run(const char* name, const uint8_t* dB, uint32_t K, uint32_t pitch, int nw
 int main() {
   uint8_t* dB;
   long long* dout;
-  const size_t bytes = 1024u << 20;  // 1 GB: rows beyond the 16 MB window miss L2
+  const size_t bytes = 64u << 20;
   cudaMalloc(&dB, bytes);
   cudaMemset(dB, 1, bytes);
   cudaMalloc(&dout, 148 * 8);
-  for (size_t window : {(size_t)16 << 20, (size_t)1024 << 20}) {  // L2-resident rows, DRAM rows
-    printf("-- rows drawn from a %zu MB window\n", window >> 20);
-    for (uint32_t pitch : {512u, 4096u}) {
-      const uint32_t K = (uint32_t)(window / pitch);
-      for (int nw : {8, 16}) {
-        run<0, 1>("cp.async 16 B, wait_group, 1 batch/warp", dB, K, pitch, nw, dout);
-        run<0, 4>("cp.async 16 B, wait_group, 4 batches/warp", dB, K, pitch, nw, dout);
-        run<4, 2>("cp.async 16 B, mbarrier, 2 batches/warp", dB, K, pitch, nw, dout);
-        run<4, 4>("cp.async 16 B, mbarrier, 4 batches/warp", dB, K, pitch, nw, dout);
-        run<1, 4>("ld.global.v4 + st.shared, 4 loads/lane", dB, K, pitch, nw, dout);
-        run<3, 2>("bulk copy 256 B per lane, 2 batches/warp", dB, K, pitch, nw, dout);
-      }
-    }
+  const uint32_t pitch = 512, K = (uint32_t)((16u << 20) / pitch);
+  for (int nw : {8, 16}) {
+    run<4, 2>("noinc arrive, per-warp barrier, 2 in flight", dB, K, pitch, nw, dout);
+    run<4, 4>("noinc arrive, per-warp barrier, 4 in flight", dB, K, pitch, nw, dout);
+    run<5, 2>("noinc arrive, ONE CTA barrier, 2 in flight", dB, K, pitch, nw, dout);
+    run<5, 4>("noinc arrive, ONE CTA barrier, 4 in flight", dB, K, pitch, nw, dout);
+    run<6, 2>("wait_group + 1 arrive/warp, 2 in flight", dB, K, pitch, nw, dout);
+    run<6, 4>("wait_group + 1 arrive/warp, 4 in flight", dB, K, pitch, nw, dout);
   }
   return 0;
 }
