@@ -9,7 +9,9 @@
 //     warp 0      A/E producer : cp.async.bulk of the compressed A image (4 KB per
 //                               k-step) and of the TMEM metadata block (2 KB); a
 //                               second cursor fills the gather-list ring ahead
-//     warps 6-15  B producers  : 8 warps (9 and 13 idle: SM sub-partition 1 is
+//     warps 9, 13  (static schedules) metadata blocks / gather-list ring, split
+//                               off warp 0, whose one thread paced the k-blocks
+//     warps 6-15  B producers  : 8 warps (9 and 13 not: SM sub-partition 1 is
 //     except 9,13               left to the MMA warp) gather the B rows of the
 //                               k-block with 16-byte cp.async straight into the
 //                               SW128 MN-major UMMA layout (PAD rows / columns
