@@ -61,10 +61,6 @@
 #ifndef JIG_AE_SPLIT
 #define JIG_AE_SPLIT 1  // static schedules: metadata copies on warp 9, gather lists on warp 13 (else all on warp 0)
 #endif
-#ifndef JIG_L2_AHEAD
-#define JIG_L2_AHEAD 1  // warp 13 also prefetches into L2 the A / metadata of the k-blocks it lists, and the B rows
-                        // of the list it wrote 4 k-blocks earlier
-#endif
 
 namespace jig {
 
@@ -857,56 +853,23 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
     // Fills the gather-list ring in (unit, k-block) order, paced only by the ring
     // (kGS = 2 x stages slots freed by the B producers): the lists land long
     // before their B rows are needed; the initial fill issued the
-    // first unit's first nG0 lists.  JIG_L2_AHEAD: running several k-blocks ahead
-    // of the copies, the warp also prefetches into L2 the compressed A and
-    // metadata of each k-block it lists (bulk prefetches, lane 0) and the B row
-    // segments of the list it wrote 4 k-blocks earlier (landed by then; all lanes),
-    // so the stage copies find them in L2 instead of DRAM.
-    constexpr int kLag = 4;
-    int gslot = nG0 % C_::kGS, hint = 0, nl = 0;
-    uint32_t gph = nG0 == C_::kGS ? 1u : 0u;
-    struct Lag {
-      const char* base;  // B + this CTA's first column of the unit (bytes)
-      int64_t pitch;     // B row pitch (bytes)
-      int32_t K, bytes, rows;
-    };
-    Lag lag[kLag];
-    for (int us = cluster_id; us < prm.nunits; us += nclusters) {
-      const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
-      if (!wk.valid) continue;
-      for (int kb = wk.kb_lo + (us == cluster_id ? nG0 : 0); kb < wk.kb_hi; ++kb) {
-        const int steps = wk.steps(kb);
-        if (lane == 0) {
+    // first unit's first nG0 lists.
+    if (lane == 0) {
+      int gslot = nG0 % C_::kGS, hint = 0;
+      uint32_t gph = nG0 == C_::kGS ? 1u : 0u;
+      for (int us = cluster_id; us < prm.nunits; us += nclusters) {
+        const Work wk = decode_unit<NT, kPair, Prm>(prm, us, rank, S, hint);
+        if (!wk.valid) continue;
+        for (int kb = wk.kb_lo + (us == cluster_id ? nG0 : 0); kb < wk.kb_hi; ++kb) {
+          const int steps = wk.steps(kb);
           mbar_wait(&gempty[gslot], gph ^ 1);
           mbar_arrive_expect_tx(&gfull[gslot], (uint32_t)(steps * 128));
           bulk_g2s(sG + gslot * kRowsPerBlock, wk.G + wk.gks(kb) * 32, steps * 128, &gfull[gslot]);
-          if (JIG_L2_AHEAD) {
-            bulk_prefetch_l2(wk.Aimg + wk.gks(kb) * kKStepBytesA, (uint32_t)(steps * kKStepBytesA));
-            if (!wk.dense(kb)) bulk_prefetch_l2(wk.Eimg + (wk.kb0 + kb) * kEBlockBytes, kEBlockBytes);
-          }
+          if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
         }
-        if (JIG_L2_AHEAD) {
-          if (nl >= kLag) {  // the list written kLag k-blocks ago: its B row segments into L2
-            if (nl == kLag) griddep_wait();  // B may be the previous kernel's output
-            const int ls = (gslot - kLag + C_::kGS) % C_::kGS;
-            const uint32_t lph = ((uint32_t)((nl - kLag + nG0) / C_::kGS)) & 1u;
-            const Lag& l = lag[nl % kLag];
-            mbar_wait(&gfull[ls], lph);
-            for (int r = lane; r < l.rows; r += 32) {
-              const int32_t g = ld_shared_s32(smem_u32(sG + ls * kRowsPerBlock + r));
-              if (g < l.K)
-                for (int o = 0; o < l.bytes; o += 128) prefetch_l2(l.base + (int64_t)g * l.pitch + o);
-            }
-          }
-          const int wl = kPair ? wk.ncols / 2 : wk.ncols;  // B columns this CTA stages
-          lag[nl % kLag] = Lag{reinterpret_cast<const char*>(wk.B) + (int64_t)(wk.n0 + (kPair ? (int)rank * wl : 0)) * 2,
-                               wk.N * 2, (int32_t)wk.K, (int32_t)min((int64_t)wl, wk.N - wk.n0) * 2, steps * 32};
-          ++nl;
-        }
-        __syncwarp();
-        if (++gslot == C_::kGS) { gslot = 0; gph ^= 1; }
       }
     }
+    __syncwarp();
   } else if (bprod_index(warp) >= 0) {
     // ------------------------------------------------------------ B producers
     // Group grp copies the B rows of the k-blocks j with j % kBGroups == grp; warp
