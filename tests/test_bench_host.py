@@ -49,3 +49,32 @@ def test_venom_workload_points_are_natively_24():
     nz = (A & 0x7FFF) != 0
     assert nz.reshape(256, -1, 4).sum(axis=2).max() <= 2
     assert abs(nz.mean() - 2 / 20) < 1e-12
+
+
+def test_algorithmic_bytes_and_flops():
+    """Roofline numerator: per tile 16P values +
+    2P metadata + 64 B gather list, the touched B rows once, C once; executed
+    flops 2*P*16*N per tile; CUDA-core entries (f3) add 8 B each plus the per-row
+    offsets and 2*N flops each."""
+    info = dict(panel_rows=128, ntiles=10, npanels=2, cc_entries=0)
+    ab, ef = bench.algorithmic(info, M=200, K=300, N=64, rows_touched=250)
+    assert ab == (16 * 128 + 2 * 128 + 64) * 10 + 2 * 64 * 250 + 2 * 200 * 64
+    assert ef == 2 * 128 * 16 * 10 * 64
+    info["cc_entries"] = 7
+    ab2, ef2 = bench.algorithmic(info, M=200, K=300, N=64, rows_touched=250)
+    assert ab2 - ab == 8 * 7 + 4 * (2 * 128 + 1) and ef2 - ef == 2 * 7 * 64
+    ab3, _ = bench.algorithmic(info, M=200, K=300, N=64, rows_touched=250, c_bytes_per_elem=4)
+    assert ab3 - ab2 == 2 * 200 * 64
+
+
+def test_paper_context_is_table2():
+    """The paper's Table 2 cuBLAS column, quoted as context:
+    twelve (v, s) cells, avg <= max, increasing with sparsity for every v."""
+    t = bench.PAPER_TABLE2
+    cells = {k: v for k, v in t.items() if k != "source"}
+    assert len(cells) == 12 and "P:244-259" in t["source"]
+    for v in (2, 4, 8):
+        avgs = [cells[f"v{v}_s{s}"][0] for s in (80, 90, 95, 98)]
+        assert avgs == sorted(avgs)
+        assert all(a <= m for a, m in (cells[f"v{v}_s{s}"] for s in (80, 90, 95, 98)))
+    assert cells["v8_s98"] == [2.14, 5.45] and cells["v2_s80"] == [0.77, 1.27]
