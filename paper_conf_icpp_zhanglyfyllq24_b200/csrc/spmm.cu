@@ -1023,6 +1023,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_spmm(const Prm prm) {
           // cluster-scope acquire would add an L1 invalidate (CCTL.IVALL) per k-block.
           if (kPair) mbar_wait(&pfull[stage], phase);
           if (JIG_TRACE_KB_ON && prm.trace) wait_cycles += clock64() - tw0;
+          // the stage's B rows were written by cp.async (generic proxy) and are
+          // read by the tensor core (async proxy): proxy fence after observing them
+          fence_proxy_async();
           tc_fence_after();
           if (it == 0 && kb == kb_lo) JIG_TRACE(4);
           JIG_TRACE_KB(2, nkb_mma);
